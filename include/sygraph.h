@@ -1,0 +1,156 @@
+/*
+ * sygraph.h — C ABI of the B200-native Two-Layer-Bitmap frontier advance
+ * (SYgraph, De Caro/Cordasco/Cosenza, ICPP'25; /root/reference/PAPER.md = "P:<line>").
+ *
+ * Plain C: pointers + sizes, no torch/C++ types.  Every function returns an int status
+ * (SG_OK = 0, < 0 on error) and never throws; sg_last_error() gives a thread-local message.
+ * Handles are not thread-safe (one host thread per handle at a time).  Device pointers are
+ * CUDA device addresses on the current device; `stream` arguments are cudaStream_t values
+ * (NULL = legacy default stream).
+ *
+ * Data layout (readings C1-C3):
+ *   graph     symmetric CSR, vertex ids int32, row_ptr int64[n+1], col_idx int32[nnz] with
+ *             every row sorted ascending, no self-loops or multi-edges (§3.1; C8, C9);
+ *             optional weights uint8[nnz] (SSSP; w(u,v) = w(v,u); C11).
+ *   frontier  Two-Layer Bitmap (§4.3): layer 1 = uint64 bits[ceil(n/64)], vertex v is
+ *             bit (v & 63) of word (v >> 6) (LSB first; §4.1); layer 2 = uint64
+ *             summ[ceil(n/4096)], bit (w & 63) of word (w >> 6) is set iff bits[w] != 0.
+ *             Bits >= n are always 0.
+ */
+#ifndef SYGRAPH_H
+#define SYGRAPH_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SG_API __attribute__((visibility("default")))
+
+enum sg_status {
+    SG_OK = 0,
+    SG_ERR_INVALID = -1,      /* bad argument (range, NULL, malformed CSR under SG_F_VALIDATE) */
+    SG_ERR_OOM = -2,          /* device allocation failed */
+    SG_ERR_CUDA = -3,         /* CUDA runtime/launch error (message in sg_last_error) */
+    SG_ERR_NCCL = -4,         /* reserved: collective failure */
+    SG_ERR_UNSUPPORTED = -5,  /* valid request outside the implemented envelope */
+    SG_ERR_STATE = -6         /* missing functor state / iteration cap hit / handle misuse */
+};
+enum { SG_MEM_HOST = 0, SG_MEM_DEVICE = 1 };          /* where input arrays live */
+enum { SG_F_VALIDATE = 2 };                           /* graph_load_csr flags */
+enum { SG_FN_BFS = 0, SG_FN_SSSP = 1, SG_FN_CC = 2, SG_FN_BC_SIGMA = 3 };   /* advance functors */
+enum { SG_DIR_AUTO = 0, SG_DIR_PUSH = 1, SG_DIR_PULL = 2 };                 /* BFS direction */
+
+typedef struct sg_graph sg_graph;
+typedef struct sg_frontier sg_frontier;
+
+/* Functor states for advance(): device pointers + scalars (Table 2: an advance functor
+ * (src, dst, edge, weight) -> bool decides whether dst enters the output frontier). */
+typedef struct {              /* BFS (Listing 1): dst enters iff not yet visited; the   */
+    uint32_t *level;          /* inserting thread writes level[dst] = depth + 1 and sets visited.  */
+    uint64_t *visited;        /* layer-1-shaped bitmap (ceil(n/64) words), updated in place        */
+    uint32_t depth;
+} sg_bfs_state;
+typedef struct {              /* SSSP relax (P:161 Bellman-Ford): nd = dist[src] + w; dst enters  */
+    uint32_t *dist;           /* iff atomicMin(&dist[dst], nd) > nd.  Weights come from the graph. */
+} sg_sssp_state;
+typedef struct {              /* CC label propagation: dst enters iff                      */
+    int32_t *label;           /* atomicMin(&label[dst], label[src]) > label[src].                  */
+} sg_cc_state;
+typedef struct {              /* BC forward sigma (P:161 Brandes): dst not in `visited` (frozen for */
+    uint32_t *level;          /* the step) gets sigma[dst] += sigma[src] and enters the output; its */
+    uint64_t *visited;        /* inserting thread writes level[dst] = depth + 1.  The caller ORs   */
+    double *sigma;            /* the output into `visited` afterwards (frontier_or).               */
+    uint32_t depth;
+} sg_bc_state;
+
+typedef struct {
+    void *stream;             /* cudaStream_t; NULL = legacy default stream */
+    int direction;            /* SG_DIR_* for run_bfs (default AUTO = Beamer direction optimising) */
+    double alpha, beta;       /* Beamer thresholds (defaults 14, 24): push->pull when m_f > m_u/alpha,
+                                 pull->push when n_f < n/beta */
+    int64_t max_iters;        /* superstep cap (0 = n + 1); exceeding it returns SG_ERR_STATE */
+    int32_t heavy_degree;     /* push tiers: degree > heavy_degree goes to the CTA/grid tier (0 = default) */
+    int32_t small_degree;     /* degree <= small_degree uses the thread-granular packed tier (0 = default, <0 = none) */
+    int32_t reserved[8];
+} sg_opts;
+
+typedef struct {
+    int64_t iterations;       /* supersteps executed */
+    int64_t push_steps, pull_steps;
+    int64_t arcs_pushed;      /* sum of frontier degrees over push steps (arcs inspected by push) */
+    int64_t arcs_pulled;      /* arcs scanned by pull steps (early exit at the first parent) */
+    int64_t reached;          /* vertices with a finite result (BFS/SSSP) */
+    double device_ms;         /* CUDA-event time of the call on its stream */
+} sg_stats;
+
+/* ---- graph ---------------------------------------------------------------------------- */
+/* Copy a symmetric CSR to device memory owned by the returned handle (§3.1; timing of
+ * the paper excludes this transfer).  mem = SG_MEM_HOST | SG_MEM_DEVICE says where the
+ * three input arrays live; weights may be NULL.  n in [1, 2^31-1], nnz in [0, 2^40].
+ * SG_F_VALIDATE checks row_ptr monotone, row_ptr[0] = 0, row_ptr[n] = nnz and 0 <= col < n on
+ * the device (SG_ERR_INVALID on failure).  Synchronises `stream` before returning. */
+SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const int32_t *col_idx,
+                          const uint8_t *weights, int mem, int flags, void *stream, sg_graph **out);
+SG_API int graph_free(sg_graph *g);
+SG_API int graph_info(const sg_graph *g, int64_t *n, int64_t *nnz, const int64_t **row_ptr,
+                      const int32_t **col_idx, const uint8_t **weights);
+
+/* ---- frontier (§3.1, §3.2, Listing 1) -------------------------------------- */
+/* Empty 2LB frontier sized for g (library-owned device memory). */
+SG_API int frontier_init(const sg_graph *g, sg_frontier **out);
+SG_API int frontier_free(sg_frontier *f);
+/* Insert k vertex ids (host or device array per `mem`); ids outside [0,n) -> SG_ERR_INVALID
+ * (host arrays are checked; device arrays are range-masked on the device). Async. */
+SG_API int frontier_insert(sg_frontier *f, const int32_t *v, int64_t k, int mem, void *stream);
+/* All vertices active (advance::vertices, Table 2). Async. */
+SG_API int frontier_fill_all(sg_frontier *f, void *stream);
+SG_API int frontier_clear(sg_frontier *f, void *stream);
+/* Number of active vertices (popcount); synchronises `stream`. */
+SG_API int frontier_count(const sg_frontier *f, int64_t *out, void *stream);
+/* Device pointers of the two layers and their word counts (read/write views). */
+SG_API int frontier_view(const sg_frontier *f, uint64_t **bits, uint64_t **summ, int64_t *nw1, int64_t *nw2);
+/* Frontier set operators (§3.1, §4.1), word-parallel: dst = dst OP src,
+ * op 0 = union (OR), 1 = intersection (AND), 2 = subtraction (AND NOT), 3 = symmetric
+ * difference (XOR).  The summary layer is rebuilt. Async. */
+SG_API int frontier_op(sg_frontier *dst, const sg_frontier *src, int op, void *stream);
+/* OR the layer-1 words of f into a plain bitmap `dst` (ceil(n/64) words). Async. */
+SG_API int frontier_or_into(const sg_frontier *f, uint64_t *dst, void *stream);
+
+/* ---- advance (Table 2; §4.2-4.3) ----------------------------------- */
+/* One push advance superstep: compacts the summary layer of `in` into the offsets buffer
+ * (P:255), then expands every active vertex's adjacency with the degree-tiered load balance,
+ * applying `functor` (SG_FN_*) per edge with `functor_state` (pointer to the matching
+ * sg_*_state struct, host memory, read at call time).  Vertices for which the functor
+ * returns true are inserted into `out` (both layers); out may be NULL (advance without an
+ * output frontier).  `out` is not cleared first.  Stream-ordered, returns after
+ * enqueue (the paper's returned event). SG_FN_SSSP needs graph weights. */
+SG_API int advance(const sg_graph *g, const sg_frontier *in, sg_frontier *out, int functor,
+                   const void *functor_state, void *stream);
+
+/* ---- algorithms (§3.4) — return when the result is complete on opts->stream ------ */
+/* BFS levels from src (Listing 1): level[src] = 0, UINT32_MAX = unreached. level: device[n]. */
+SG_API int run_bfs(const sg_graph *g, int32_t src, uint32_t *level, const sg_opts *opts, sg_stats *stats);
+/* SSSP distances (Bellman-Ford by frontier relaxation, no delta-stepping).
+ * dist: device[n], UINT32_MAX = unreached. Needs weights; SG_ERR_UNSUPPORTED if
+ * max_weight * (n-1) >= 2^32-1. */
+SG_API int run_sssp(const sg_graph *g, int32_t src, uint32_t *dist, const sg_opts *opts, sg_stats *stats);
+/* Connected components by label propagation: label[v] = min id of v's component. */
+SG_API int run_cc(const sg_graph *g, int32_t *label, const sg_opts *opts, sg_stats *stats);
+/* Betweenness centrality (Brandes, forward sigma + backward delta): bc[v] = sum over
+ * the k host-array sources of delta_s(v), unnormalised (reading C14). bc: device[n], overwritten. */
+SG_API int run_bc(const sg_graph *g, const int32_t *sources, int32_t k, double *bc, const sg_opts *opts,
+                  sg_stats *stats);
+
+/* Defaults for sg_opts (stream NULL, AUTO direction, alpha 14, beta 24). */
+SG_API void sg_opts_default(sg_opts *o);
+/* Thread-local message of the last error on this thread ("" if none). */
+SG_API const char *sg_last_error(void);
+/* Library build/version string. */
+SG_API const char *sg_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SYGRAPH_H */

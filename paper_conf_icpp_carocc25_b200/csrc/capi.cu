@@ -1,0 +1,773 @@
+// capi.cu — the C ABI (include/sygraph.h) and the superstep drivers of BFS / SSSP / CC / BC.
+//
+// Execution model (§3 BSP; Listing 1): one advance per superstep,
+// the output frontier consistent at the end of the step, swap + clear, stop when the frontier
+// is empty.  Per superstep the host reads back one 128-byte control block (frontier sizes for
+// empty() and the direction policy); everything else stays on the device stream.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "sygraph.h"
+#include "kernels.h"
+
+using namespace sg;
+
+// ------------------------------------------------------------------------------------------
+// errors
+static thread_local std::string t_err;
+static int fail(int code, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    t_err = buf;
+    return code;
+}
+#define CK(x)                                                                                          \
+    do {                                                                                               \
+        cudaError_t e_ = (x);                                                                          \
+        if (e_ != cudaSuccess) {                                                                       \
+            return fail(e_ == cudaErrorMemoryAllocation ? SG_ERR_OOM : SG_ERR_CUDA, "%s: %s (%s:%d)", #x, \
+                        cudaGetErrorString(e_), __FILE__, __LINE__);                                   \
+        }                                                                                              \
+    } while (0)
+#define TRY(x)                 \
+    do {                       \
+        int r_ = (x);          \
+        if (r_ != SG_OK) return r_; \
+    } while (0)
+
+// ------------------------------------------------------------------------------------------
+// handles
+struct sg_frontier {
+    const sg_graph *g;
+    uint64_t *bits = nullptr;      // nw1 words
+    uint64_t *summ = nullptr;      // nw2 words
+    uint32_t *offsets = nullptr;   // nw1 entries
+    DevStats *st = nullptr;        // control block (device)
+    bool owns_st = true;
+};
+
+struct Workspace {
+    sg_frontier fr[2];
+    DevStats *st = nullptr;        // 2 contiguous control blocks (fr[0].st, fr[1].st)
+    DevStats *h_st = nullptr;      // pinned host mirror
+    uint64_t *visited = nullptr;   // nw1 words
+    HeavyItem *heavy = nullptr;
+    uint32_t heavy_cap = 0;
+    int32_t heavy_deg = 0;
+    unsigned long long *scratch = nullptr;   // 8 device u64 counters (BC max, stack top, underflow ...)
+    unsigned long long *h_scratch = nullptr;
+    int32_t *stack = nullptr;      // BC: BFS order
+    int32_t *exp_of_level = nullptr;
+    double *delta = nullptr;
+    double *sigma = nullptr;
+    uint32_t *level = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+};
+
+struct sg_graph {
+    GraphView v;
+    int64_t *rp = nullptr;
+    int32_t *col = nullptr;
+    uint8_t *w = nullptr;
+    uint32_t max_w = 0;
+    int device = 0;
+    Workspace *ws = nullptr;
+};
+
+static const int32_t kDefaultHeavy = 2048;
+static const int32_t kDefaultSmall = 32;
+
+static int alloc_frontier_bufs(sg_frontier *f, const sg_graph *g, bool own_st) {
+    f->g = g;
+    CK(cudaMalloc(&f->bits, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMalloc(&f->summ, sizeof(uint64_t) * (size_t)g->v.nw2));
+    CK(cudaMalloc(&f->offsets, sizeof(uint32_t) * (size_t)g->v.nw1));
+    if (own_st) CK(cudaMalloc(&f->st, sizeof(DevStats)));
+    f->owns_st = own_st;
+    CK(cudaMemset(f->bits, 0, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMemset(f->summ, 0, sizeof(uint64_t) * (size_t)g->v.nw2));
+    if (own_st) CK(cudaMemset(f->st, 0, sizeof(DevStats)));
+    return SG_OK;
+}
+
+static void free_frontier_bufs(sg_frontier *f) {
+    cudaFree(f->bits);
+    cudaFree(f->summ);
+    cudaFree(f->offsets);
+    if (f->owns_st) cudaFree(f->st);
+    f->bits = f->summ = nullptr;
+    f->offsets = nullptr;
+    f->st = nullptr;
+}
+
+static int ensure_ws(sg_graph *g) {
+    if (g->ws) return SG_OK;
+    Workspace *ws = new Workspace();
+    g->ws = ws;
+    CK(cudaMalloc(&ws->st, 2 * sizeof(DevStats)));
+    CK(cudaMemset(ws->st, 0, 2 * sizeof(DevStats)));
+    CK(cudaMallocHost(&ws->h_st, 2 * sizeof(DevStats)));
+    for (int i = 0; i < 2; i++) {
+        TRY(alloc_frontier_bufs(&ws->fr[i], g, false));
+        ws->fr[i].st = ws->st + i;
+    }
+    CK(cudaMalloc(&ws->visited, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMalloc(&ws->scratch, 8 * sizeof(unsigned long long)));
+    CK(cudaMallocHost(&ws->h_scratch, 8 * sizeof(unsigned long long)));
+    CK(cudaEventCreate(&ws->ev0));
+    CK(cudaEventCreate(&ws->ev1));
+    return SG_OK;
+}
+
+// heavy queue sized for the smallest heavy threshold used so far: sum over vertices with
+// deg > T of ceil(deg / CHUNK) <= nnz / CHUNK + nnz / T.
+static int ensure_heavy(sg_graph *g, int32_t heavy_deg) {
+    Workspace *ws = g->ws;
+    if (ws->heavy && ws->heavy_deg <= heavy_deg) return SG_OK;
+    const int64_t cap64 = g->v.nnz / HEAVY_CHUNK + g->v.nnz / heavy_deg + 64;
+    if (cap64 > 0xFFFFFFF0ll) return fail(SG_ERR_UNSUPPORTED, "heavy queue too large (heavy_degree too small)");
+    cudaFree(ws->heavy);
+    ws->heavy = nullptr;
+    CK(cudaMalloc(&ws->heavy, sizeof(HeavyItem) * (size_t)cap64));
+    ws->heavy_cap = (uint32_t)cap64;
+    ws->heavy_deg = heavy_deg;
+    return SG_OK;
+}
+
+static void free_ws(Workspace *ws) {
+    if (!ws) return;
+    for (int i = 0; i < 2; i++) free_frontier_bufs(&ws->fr[i]);
+    cudaFree(ws->st);
+    cudaFreeHost(ws->h_st);
+    cudaFree(ws->visited);
+    cudaFree(ws->heavy);
+    cudaFree(ws->scratch);
+    cudaFreeHost(ws->h_scratch);
+    cudaFree(ws->stack);
+    cudaFree(ws->exp_of_level);
+    cudaFree(ws->delta);
+    cudaFree(ws->sigma);
+    cudaFree(ws->level);
+    if (ws->ev0) cudaEventDestroy(ws->ev0);
+    if (ws->ev1) cudaEventDestroy(ws->ev1);
+    delete ws;
+}
+
+static int check_device(const void *p) {
+    if (!p) return SG_OK;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(SG_ERR_INVALID, "pointer %p is not a CUDA allocation", p);
+    }
+    if (a.type != cudaMemoryTypeDevice && a.type != cudaMemoryTypeManaged)
+        return fail(SG_ERR_INVALID, "pointer %p is not device memory", p);
+    return SG_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+extern "C" {
+
+SG_API const char *sg_last_error(void) { return t_err.c_str(); }
+SG_API const char *sg_version(void) { return "sygraph-b200 0.1 (sm_100a)"; }
+
+SG_API void sg_opts_default(sg_opts *o) {
+    if (!o) return;
+    memset(o, 0, sizeof *o);
+    o->direction = SG_DIR_AUTO;
+    o->alpha = 14.0;
+    o->beta = 24.0;
+}
+
+SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const int32_t *col_idx,
+                          const uint8_t *weights, int mem, int flags, void *stream, sg_graph **out) {
+    t_err.clear();
+    if (!out) return fail(SG_ERR_INVALID, "out is NULL");
+    *out = nullptr;
+    if (n <= 0 || n > 0x7FFFFFFFll) return fail(SG_ERR_INVALID, "n=%lld outside [1, 2^31-1]", (long long)n);
+    if (nnz < 0 || nnz > (1ll << 40)) return fail(SG_ERR_INVALID, "nnz=%lld outside [0, 2^40]", (long long)nnz);
+    if (!row_ptr || (nnz > 0 && !col_idx)) return fail(SG_ERR_INVALID, "row_ptr/col_idx NULL");
+    if (mem != SG_MEM_HOST && mem != SG_MEM_DEVICE) return fail(SG_ERR_INVALID, "mem must be SG_MEM_HOST or SG_MEM_DEVICE");
+    if (mem == SG_MEM_DEVICE) {
+        TRY(check_device(row_ptr));
+        TRY(check_device(col_idx));
+        TRY(check_device(weights));
+    } else {
+        if (row_ptr[0] != 0 || row_ptr[n] != nnz) return fail(SG_ERR_INVALID, "row_ptr[0] != 0 or row_ptr[n] != nnz");
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    sg_graph *g = new sg_graph();
+    CK(cudaGetDevice(&g->device));
+    g->v.n = n;
+    g->v.nnz = nnz;
+    g->v.nw1 = (n + 63) / 64;
+    g->v.nw2 = (g->v.nw1 + 63) / 64;
+    const cudaMemcpyKind kind = mem == SG_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+    // col_idx/weights get 64 B of zero padding: 16-B bulk copies may read up to 12 B past nnz
+    CK(cudaMalloc(&g->rp, sizeof(int64_t) * (size_t)(n + 1)));
+    CK(cudaMalloc(&g->col, sizeof(int32_t) * (size_t)nnz + 64));
+    CK(cudaMemsetAsync((char *)g->col + sizeof(int32_t) * (size_t)nnz, 0, 64, s));
+    CK(cudaMemcpyAsync(g->rp, row_ptr, sizeof(int64_t) * (size_t)(n + 1), kind, s));
+    if (nnz) CK(cudaMemcpyAsync(g->col, col_idx, sizeof(int32_t) * (size_t)nnz, kind, s));
+    if (weights) {
+        CK(cudaMalloc(&g->w, (size_t)nnz + 64));
+        CK(cudaMemsetAsync(g->w + nnz, 0, 64, s));
+        if (nnz) CK(cudaMemcpyAsync(g->w, weights, (size_t)nnz, kind, s));
+    }
+    g->v.rp = g->rp;
+    g->v.col = g->col;
+    g->v.w = g->w;
+    unsigned long long *dscr = nullptr;
+    CK(cudaMalloc(&dscr, 16));
+    CK(cudaMemsetAsync(dscr, 0, 16, s));
+    if (flags & SG_F_VALIDATE) launch_validate_csr(g->v, dscr, s);
+    if (g->w) launch_max_weight(g->w, nnz, reinterpret_cast<unsigned int *>(dscr + 1), s);
+    unsigned long long h[2] = {0, 0};
+    CK(cudaMemcpyAsync(h, dscr, 16, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    CK(cudaGetLastError());
+    cudaFree(dscr);
+    g->max_w = (uint32_t)(h[1] & 0xffffffffu);
+    if (h[0]) {
+        graph_free(g);
+        return fail(SG_ERR_INVALID, "CSR validation failed (%llu bad entries)", h[0]);
+    }
+    *out = g;
+    return SG_OK;
+}
+
+SG_API int graph_free(sg_graph *g) {
+    if (!g) return SG_OK;
+    free_ws(g->ws);
+    cudaFree(g->rp);
+    cudaFree(g->col);
+    cudaFree(g->w);
+    delete g;
+    return SG_OK;
+}
+
+SG_API int graph_info(const sg_graph *g, int64_t *n, int64_t *nnz, const int64_t **row_ptr, const int32_t **col_idx,
+                      const uint8_t **weights) {
+    if (!g) return fail(SG_ERR_INVALID, "graph is NULL");
+    if (n) *n = g->v.n;
+    if (nnz) *nnz = g->v.nnz;
+    if (row_ptr) *row_ptr = g->rp;
+    if (col_idx) *col_idx = g->col;
+    if (weights) *weights = g->w;
+    return SG_OK;
+}
+
+// ---- frontier ----------------------------------------------------------------------------
+SG_API int frontier_init(const sg_graph *g, sg_frontier **out) {
+    t_err.clear();
+    if (!g || !out) return fail(SG_ERR_INVALID, "NULL argument");
+    sg_frontier *f = new sg_frontier();
+    int r = alloc_frontier_bufs(f, g, true);
+    if (r != SG_OK) {
+        free_frontier_bufs(f);
+        delete f;
+        return r;
+    }
+    *out = f;
+    return SG_OK;
+}
+
+SG_API int frontier_free(sg_frontier *f) {
+    if (!f) return SG_OK;
+    free_frontier_bufs(f);
+    delete f;
+    return SG_OK;
+}
+
+SG_API int frontier_insert(sg_frontier *f, const int32_t *v, int64_t k, int mem, void *stream) {
+    t_err.clear();
+    if (!f || (k > 0 && !v) || k < 0) return fail(SG_ERR_INVALID, "bad frontier_insert arguments");
+    if (k == 0) return SG_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t n = f->g->v.n;
+    if (mem == SG_MEM_HOST) {
+        for (int64_t i = 0; i < k; i++)
+            if (v[i] < 0 || v[i] >= n) return fail(SG_ERR_INVALID, "vertex %d outside [0,%lld)", v[i], (long long)n);
+        int32_t *d = nullptr;
+        CK(cudaMallocAsync(&d, sizeof(int32_t) * (size_t)k, s));
+        CK(cudaMemcpyAsync(d, v, sizeof(int32_t) * (size_t)k, cudaMemcpyHostToDevice, s));
+        launch_insert(f->bits, f->summ, d, k, n, s);
+        CK(cudaFreeAsync(d, s));
+        CK(cudaStreamSynchronize(s));   // the host array may be released by the caller
+    } else if (mem == SG_MEM_DEVICE) {
+        launch_insert(f->bits, f->summ, v, k, n, s);
+    } else {
+        return fail(SG_ERR_INVALID, "bad mem");
+    }
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
+SG_API int frontier_fill_all(sg_frontier *f, void *stream) {
+    if (!f) return fail(SG_ERR_INVALID, "NULL frontier");
+    const GraphView &g = f->g->v;
+    launch_fill_all(f->bits, f->summ, g.n, g.nw1, g.nw2, (cudaStream_t)stream);
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
+static int clear_frontier(sg_frontier *f, cudaStream_t s) {
+    const GraphView &g = f->g->v;
+    CK(cudaMemsetAsync(f->bits, 0, sizeof(uint64_t) * (size_t)g.nw1, s));
+    CK(cudaMemsetAsync(f->summ, 0, sizeof(uint64_t) * (size_t)g.nw2, s));
+    return SG_OK;
+}
+
+SG_API int frontier_clear(sg_frontier *f, void *stream) {
+    if (!f) return fail(SG_ERR_INVALID, "NULL frontier");
+    return clear_frontier(f, (cudaStream_t)stream);
+}
+
+SG_API int frontier_count(const sg_frontier *f, int64_t *out, void *stream) {
+    if (!f || !out) return fail(SG_ERR_INVALID, "NULL argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    unsigned long long *d = nullptr, h = 0;
+    CK(cudaMallocAsync(&d, sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(d, 0, sizeof(unsigned long long), s));
+    launch_popcount(f->bits, f->g->v.nw1, d, s);
+    CK(cudaMemcpyAsync(&h, d, sizeof h, cudaMemcpyDeviceToHost, s));
+    CK(cudaFreeAsync(d, s));
+    CK(cudaStreamSynchronize(s));
+    CK(cudaGetLastError());
+    *out = (int64_t)h;
+    return SG_OK;
+}
+
+SG_API int frontier_view(const sg_frontier *f, uint64_t **bits, uint64_t **summ, int64_t *nw1, int64_t *nw2) {
+    if (!f) return fail(SG_ERR_INVALID, "NULL frontier");
+    if (bits) *bits = f->bits;
+    if (summ) *summ = f->summ;
+    if (nw1) *nw1 = f->g->v.nw1;
+    if (nw2) *nw2 = f->g->v.nw2;
+    return SG_OK;
+}
+
+SG_API int frontier_op(sg_frontier *dst, const sg_frontier *src, int op, void *stream) {
+    if (!dst || !src || dst->g->v.n != src->g->v.n || op < 0 || op > 3)
+        return fail(SG_ERR_INVALID, "bad frontier_op arguments");
+    cudaStream_t s = (cudaStream_t)stream;
+    const GraphView &g = dst->g->v;
+    launch_setop(dst->bits, src->bits, g.nw1, op, s);
+    launch_rebuild_summary(dst->bits, dst->summ, g.nw1, g.nw2, s);
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
+SG_API int frontier_or_into(const sg_frontier *f, uint64_t *dst, void *stream) {
+    if (!f || !dst) return fail(SG_ERR_INVALID, "NULL argument");
+    launch_or_all(f->bits, f->g->v.nw1, dst, (cudaStream_t)stream);
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------------------------------------------
+// superstep helpers
+struct Tiers {
+    int32_t heavy, small;
+};
+static Tiers tiers_from(const sg_opts *o) {
+    Tiers t{kDefaultHeavy, kDefaultSmall};
+    if (o && o->heavy_degree > 0) t.heavy = o->heavy_degree;
+    if (o && o->small_degree > 0) t.small = o->small_degree;
+    if (o && o->small_degree < 0) t.small = 0;           // no thread tier
+    if (t.small > t.heavy) t.small = t.heavy;
+    return t;
+}
+
+// zero the control block, compact the summary layer into offsets, optional n_f / m_f
+static int compact(const sg_graph *g, const sg_frontier *f, bool stats, cudaStream_t s) {
+    CK(cudaMemsetAsync(f->st, 0, sizeof(DevStats), s));
+    launch_compact(f->summ, g->v.nw2, f->offsets, f->st, s);
+    if (stats) launch_frontier_stats(g->v, f->bits, f->offsets, f->st, g->v.nw1, s);
+    return SG_OK;
+}
+
+static PushLaunch push_launch(const sg_graph *g, const sg_frontier *in, Tiers t, int64_t count_hint) {
+    PushLaunch L;
+    L.g = g->v;
+    L.in_bits = in->bits;
+    L.offsets = in->offsets;
+    L.st = in->st;
+    L.heavy = g->ws->heavy;
+    L.heavy_cap = g->ws->heavy_cap;
+    L.heavy_deg = t.heavy;
+    L.small_deg = t.small;
+    const int maxg = push_max_grid_words();
+    if (count_hint < 0) {
+        L.batch = 32;
+        L.grid_words = maxg;
+    } else {
+        int64_t cf = count_hint / ((int64_t)maxg * 8 * 2);
+        if (cf < 1) cf = 1;
+        if (cf > 8) cf = 8;
+        L.batch = (int32_t)(8 * cf);
+        int64_t gw = (count_hint + L.batch - 1) / L.batch;
+        if (gw < 1) gw = 1;
+        if (gw > maxg) gw = maxg;
+        L.grid_words = (int)gw;
+    }
+    L.grid_heavy = push_max_grid_heavy();
+    return L;
+}
+
+static int read_stats(Workspace *ws, cudaStream_t s) {
+    CK(cudaMemcpyAsync(ws->h_st, ws->st, 2 * sizeof(DevStats), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
+static cudaStream_t stream_of(const sg_opts *o) { return o ? (cudaStream_t)o->stream : (cudaStream_t)0; }
+
+extern "C" {
+
+// ---- generic advance ---------------------------------------------------------------------
+SG_API int advance(const sg_graph *gc, const sg_frontier *in, sg_frontier *out, int functor, const void *state,
+                   void *stream) {
+    t_err.clear();
+    if (!gc || !in || !state) return fail(SG_ERR_INVALID, "NULL argument");
+    if (in->g != gc || (out && out->g != gc)) return fail(SG_ERR_INVALID, "frontier belongs to another graph");
+    sg_graph *g = const_cast<sg_graph *>(gc);
+    cudaStream_t s = (cudaStream_t)stream;
+    TRY(ensure_ws(g));
+    const Tiers t{kDefaultHeavy, kDefaultSmall};
+    TRY(ensure_heavy(g, t.heavy));
+    TRY(compact(g, in, false, s));
+    const PushLaunch L = push_launch(g, in, t, -1);
+    uint64_t *ob = out ? out->bits : nullptr, *os = out ? out->summ : nullptr;
+    switch (functor) {
+        case SG_FN_BFS: {
+            const sg_bfs_state *st = (const sg_bfs_state *)state;
+            if (!st->level || !st->visited) return fail(SG_ERR_STATE, "BFS state needs level and visited");
+            launch_push_bfs(L, BfsArgs{st->visited, st->level, st->depth + 1, ob, os}, s);
+            break;
+        }
+        case SG_FN_SSSP: {
+            const sg_sssp_state *st = (const sg_sssp_state *)state;
+            if (!st->dist) return fail(SG_ERR_STATE, "SSSP state needs dist");
+            if (!g->w) return fail(SG_ERR_INVALID, "SSSP needs graph weights");
+            launch_push_sssp(L, SsspArgs{st->dist, ob, os}, s);
+            break;
+        }
+        case SG_FN_CC: {
+            const sg_cc_state *st = (const sg_cc_state *)state;
+            if (!st->label) return fail(SG_ERR_STATE, "CC state needs label");
+            launch_push_cc(L, CcArgs{st->label, ob, os}, s);
+            break;
+        }
+        case SG_FN_BC_SIGMA: {
+            const sg_bc_state *st = (const sg_bc_state *)state;
+            if (!st->level || !st->visited || !st->sigma) return fail(SG_ERR_STATE, "BC state needs level, visited, sigma");
+            if (!out) return fail(SG_ERR_STATE, "BC sigma advance needs an output frontier");
+            launch_push_bc(L, BcArgs{st->visited, st->sigma, st->level, st->depth + 1, ob, os}, s);
+            break;
+        }
+        default:
+            return fail(SG_ERR_INVALID, "unknown functor %d", functor);
+    }
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
+// ---- BFS (Listing 1 + Beamer direction optimisation) --------------------------------------
+SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_opts *opts, sg_stats *stats) {
+    t_err.clear();
+    if (!gc || !level) return fail(SG_ERR_INVALID, "NULL argument");
+    sg_graph *g = const_cast<sg_graph *>(gc);
+    const GraphView &G = g->v;
+    if (src < 0 || src >= G.n) return fail(SG_ERR_INVALID, "src %d outside [0,%lld)", src, (long long)G.n);
+    sg_opts o;
+    if (opts) o = *opts; else sg_opts_default(&o);
+    if (o.alpha <= 0) o.alpha = 14.0;
+    if (o.beta <= 0) o.beta = 24.0;
+    const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
+    cudaStream_t s = stream_of(&o);
+    TRY(ensure_ws(g));
+    const Tiers t = tiers_from(&o);
+    TRY(ensure_heavy(g, t.heavy));
+    Workspace *ws = g->ws;
+    CK(cudaEventRecord(ws->ev0, s));
+    CK(cudaMemsetAsync(level, 0xFF, sizeof(uint32_t) * (size_t)G.n, s));
+    launch_set_u32(level, src, 0u, s);
+    sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
+    TRY(clear_frontier(in, s));
+    TRY(clear_frontier(out, s));
+    CK(cudaMemsetAsync(ws->visited, 0, sizeof(uint64_t) * (size_t)G.nw1, s));
+    launch_seed(in->bits, in->summ, ws->visited, src, s);      // in = {src}, visited = {src}
+    const bool auto_dir = o.direction == SG_DIR_AUTO;
+    TRY(compact(g, in, true, s));
+    TRY(read_stats(ws, s));
+    int64_t mu = G.nnz;
+    bool pull = o.direction == SG_DIR_PULL;
+    int64_t iters = 0, push_steps = 0, pull_steps = 0, arcs_pushed = 0, arcs_pulled = 0;
+    int64_t reached = 1;
+    uint32_t d = 0;
+    int in_idx = 0;
+    for (;;) {
+        const DevStats &hs = ws->h_st[in_idx];
+        const int64_t count = (int64_t)hs.count;
+        if (count == 0) break;
+        if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
+        const int64_t nf = (int64_t)hs.nf, mf = (int64_t)hs.mf;
+        if (iters > 0) reached += nf;
+        mu -= mf;
+        if (auto_dir) {
+            if (!pull && (double)mf > (double)mu / o.alpha) pull = true;
+            else if (pull && (double)nf < (double)G.n / o.beta) pull = false;
+        }
+        if (pull) {
+            launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, level, d + 1, in->st, s);
+            pull_steps++;
+        } else {
+            const PushLaunch L = push_launch(g, in, t, count);
+            launch_push_bfs(L, BfsArgs{ws->visited, level, d + 1, out->bits, out->summ}, s);
+            push_steps++;
+            arcs_pushed += mf;
+        }
+        TRY(clear_frontier(in, s));
+        TRY(compact(g, out, true, s));
+        TRY(read_stats(ws, s));
+        if (pull) arcs_pulled += (int64_t)ws->h_st[in_idx].arcs;
+        std::swap(in, out);
+        in_idx ^= 1;
+        d++;
+        iters++;
+    }
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    if (stats) {
+        stats->iterations = iters;
+        stats->push_steps = push_steps;
+        stats->pull_steps = pull_steps;
+        stats->arcs_pushed = arcs_pushed;
+        stats->arcs_pulled = arcs_pulled;
+        stats->reached = reached;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
+// ---- SSSP (frontier Bellman-Ford) --------------------------------------------------
+SG_API int run_sssp(const sg_graph *gc, int32_t src, uint32_t *dist, const sg_opts *opts, sg_stats *stats) {
+    t_err.clear();
+    if (!gc || !dist) return fail(SG_ERR_INVALID, "NULL argument");
+    sg_graph *g = const_cast<sg_graph *>(gc);
+    const GraphView &G = g->v;
+    if (src < 0 || src >= G.n) return fail(SG_ERR_INVALID, "src %d outside [0,%lld)", src, (long long)G.n);
+    if (!g->w) return fail(SG_ERR_INVALID, "SSSP needs graph weights");
+    if ((double)g->max_w * (double)(G.n - 1) >= 4294967295.0)
+        return fail(SG_ERR_UNSUPPORTED, "max_weight*(n-1) does not fit uint32 distances");
+    sg_opts o;
+    if (opts) o = *opts; else sg_opts_default(&o);
+    const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
+    cudaStream_t s = stream_of(&o);
+    TRY(ensure_ws(g));
+    const Tiers t = tiers_from(&o);
+    TRY(ensure_heavy(g, t.heavy));
+    Workspace *ws = g->ws;
+    CK(cudaEventRecord(ws->ev0, s));
+    CK(cudaMemsetAsync(dist, 0xFF, sizeof(uint32_t) * (size_t)G.n, s));
+    launch_set_u32(dist, src, 0u, s);
+    sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
+    TRY(clear_frontier(in, s));
+    TRY(clear_frontier(out, s));
+    launch_seed(in->bits, in->summ, nullptr, src, s);
+    TRY(compact(g, in, false, s));
+    TRY(read_stats(ws, s));
+    int64_t iters = 0, arcs = 0;
+    int in_idx = 0;
+    for (;;) {
+        const int64_t count = (int64_t)ws->h_st[in_idx].count;
+        if (count == 0) break;
+        if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
+        const PushLaunch L = push_launch(g, in, t, count);
+        launch_push_sssp(L, SsspArgs{dist, out->bits, out->summ}, s);
+        TRY(clear_frontier(in, s));
+        TRY(compact(g, out, false, s));
+        TRY(read_stats(ws, s));
+        arcs += (int64_t)ws->h_st[in_idx].arcs;
+        std::swap(in, out);
+        in_idx ^= 1;
+        iters++;
+    }
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->iterations = iters;
+        stats->push_steps = iters;
+        stats->arcs_pushed = arcs;
+        stats->reached = -1;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
+// ---- CC (label propagation) --------------------------------------------------------
+SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_stats *stats) {
+    t_err.clear();
+    if (!gc || !label) return fail(SG_ERR_INVALID, "NULL argument");
+    sg_graph *g = const_cast<sg_graph *>(gc);
+    const GraphView &G = g->v;
+    sg_opts o;
+    if (opts) o = *opts; else sg_opts_default(&o);
+    const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
+    cudaStream_t s = stream_of(&o);
+    TRY(ensure_ws(g));
+    const Tiers t = tiers_from(&o);
+    TRY(ensure_heavy(g, t.heavy));
+    Workspace *ws = g->ws;
+    CK(cudaEventRecord(ws->ev0, s));
+    launch_iota_i32(label, G.n, s);
+    sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
+    launch_fill_all(in->bits, in->summ, G.n, G.nw1, G.nw2, s);    // advance::vertices
+    TRY(clear_frontier(out, s));
+    TRY(compact(g, in, false, s));
+    TRY(read_stats(ws, s));
+    int64_t iters = 0, arcs = 0;
+    int in_idx = 0;
+    for (;;) {
+        const int64_t count = (int64_t)ws->h_st[in_idx].count;
+        if (count == 0) break;
+        if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
+        const PushLaunch L = push_launch(g, in, t, count);
+        launch_push_cc(L, CcArgs{label, out->bits, out->summ}, s);
+        TRY(clear_frontier(in, s));
+        TRY(compact(g, out, false, s));
+        TRY(read_stats(ws, s));
+        arcs += (int64_t)ws->h_st[in_idx].arcs;
+        std::swap(in, out);
+        in_idx ^= 1;
+        iters++;
+    }
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->iterations = iters;
+        stats->push_steps = iters;
+        stats->arcs_pushed = arcs;
+        stats->reached = G.n;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
+// ---- BC (Brandes forward sigma + backward delta) -----------------------------------
+SG_API int run_bc(const sg_graph *gc, const int32_t *sources, int32_t k, double *bc, const sg_opts *opts,
+                  sg_stats *stats) {
+    t_err.clear();
+    if (!gc || !bc || (k > 0 && !sources) || k < 0) return fail(SG_ERR_INVALID, "bad run_bc arguments");
+    sg_graph *g = const_cast<sg_graph *>(gc);
+    const GraphView &G = g->v;
+    for (int32_t i = 0; i < k; i++)
+        if (sources[i] < 0 || sources[i] >= G.n) return fail(SG_ERR_INVALID, "source %d outside [0,%lld)", sources[i], (long long)G.n);
+    sg_opts o;
+    if (opts) o = *opts; else sg_opts_default(&o);
+    cudaStream_t s = stream_of(&o);
+    TRY(ensure_ws(g));
+    const Tiers t = tiers_from(&o);
+    TRY(ensure_heavy(g, t.heavy));
+    Workspace *ws = g->ws;
+    if (!ws->sigma) {
+        CK(cudaMalloc(&ws->sigma, sizeof(double) * (size_t)G.n));
+        CK(cudaMalloc(&ws->delta, sizeof(double) * (size_t)G.n));
+        CK(cudaMalloc(&ws->level, sizeof(uint32_t) * (size_t)G.n));
+        CK(cudaMalloc(&ws->stack, sizeof(int32_t) * (size_t)G.n));
+        CK(cudaMalloc(&ws->exp_of_level, sizeof(int32_t) * (size_t)(G.n + 1)));
+    }
+    CK(cudaEventRecord(ws->ev0, s));
+    CK(cudaMemsetAsync(bc, 0, sizeof(double) * (size_t)G.n, s));
+    int64_t total_iters = 0, arcs = 0;
+    std::vector<int64_t> level_off;
+    unsigned long long *d_max = ws->scratch, *d_top = ws->scratch + 1, *d_under = ws->scratch + 2;
+    for (int32_t si = 0; si < k; si++) {
+        const int32_t src = sources[si];
+        CK(cudaMemsetAsync(ws->level, 0xFF, sizeof(uint32_t) * (size_t)G.n, s));
+        CK(cudaMemsetAsync(ws->sigma, 0, sizeof(double) * (size_t)G.n, s));
+        CK(cudaMemsetAsync(ws->visited, 0, sizeof(uint64_t) * (size_t)G.nw1, s));
+        CK(cudaMemsetAsync(ws->scratch, 0, 8 * sizeof(unsigned long long), s));
+        CK(cudaMemsetAsync(ws->exp_of_level, 0, sizeof(int32_t), s));
+        launch_set_u32(ws->level, src, 0u, s);
+        launch_set_f64(ws->sigma, src, 1.0, s);
+        launch_set_i32(ws->stack, 0, src, s);
+        launch_set_u32(reinterpret_cast<uint32_t *>(d_top), 0, 1u, s);
+        sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
+        TRY(clear_frontier(in, s));
+        TRY(clear_frontier(out, s));
+        launch_seed(in->bits, in->summ, ws->visited, src, s);
+        TRY(compact(g, in, false, s));
+        TRY(read_stats(ws, s));
+        level_off.assign(1, 0);
+        level_off.push_back(1);
+        uint32_t d = 0;
+        int in_idx = 0;
+        for (;;) {
+            const int64_t count = (int64_t)ws->h_st[in_idx].count;
+            if (count == 0) break;
+            if ((int64_t)d > G.n) return fail(SG_ERR_STATE, "BC level cap reached");
+            const PushLaunch L = push_launch(g, in, t, count);
+            launch_push_bc(L, BcArgs{ws->visited, ws->sigma, ws->level, d + 1, out->bits, out->summ}, s);
+            TRY(clear_frontier(in, s));
+            TRY(compact(g, out, false, s));
+            // finish level d+1: visited |= out, per-level scale, BFS stack
+            launch_or_listed(out->bits, out->offsets, out->st, ws->visited, G.nw1, s);
+            CK(cudaMemsetAsync(d_max, 0, sizeof(unsigned long long), s));
+            launch_bc_level_max(ws->sigma, out->bits, out->offsets, out->st, G.nw1, d_max, s);
+            launch_bc_level_scale_and_stack(ws->sigma, out->bits, out->offsets, out->st, G.nw1, d_max,
+                                            ws->exp_of_level, d + 1, ws->stack, d_top, d_under, s);
+            CK(cudaMemcpyAsync(ws->h_scratch, ws->scratch, 8 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+            TRY(read_stats(ws, s));
+            arcs += (int64_t)ws->h_st[in_idx].arcs;
+            std::swap(in, out);
+            in_idx ^= 1;
+            d++;
+            total_iters++;
+            if (ws->h_st[in_idx].count) level_off.push_back((int64_t)ws->h_scratch[1]);
+        }
+        if (ws->h_scratch[2]) return fail(SG_ERR_UNSUPPORTED, "sigma dynamic range within a BFS level exceeds fp64");
+        // backward: levels depth-1 .. 1 (level 0 = the source: delta_s(s) excluded)
+        const int64_t depth = (int64_t)level_off.size() - 1;   // number of levels
+        for (int64_t lv = depth - 1; lv >= 1; lv--)
+            launch_bc_backward_level(G, ws->stack, level_off[lv], level_off[lv + 1], ws->level, ws->sigma, ws->delta,
+                                     ws->exp_of_level, (uint32_t)lv, bc, src, s);
+        total_iters += depth;
+    }
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->iterations = total_iters;
+        stats->push_steps = total_iters;
+        stats->arcs_pushed = arcs;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
+}  // extern "C"

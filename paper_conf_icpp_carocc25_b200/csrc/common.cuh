@@ -1,0 +1,107 @@
+// common.cuh — shared device/host definitions of the B200 Two-Layer-Bitmap advance.
+// Layout (DESIGN.md §4, §4.1 and :253 §4.3, readings C1-C3):
+//   layer 1  uint64 bits[nw1], nw1 = ceil(n/64): vertex v = bit (v & 63) of word (v >> 6)
+//   layer 2  uint64 summ[nw2], nw2 = ceil(nw1/64): bit (w & 63) of word (w >> 6) <=> bits[w] != 0
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace sg {
+
+constexpr uint32_t INF32 = 0xFFFFFFFFu;
+constexpr int WARP = 32;
+
+// Graph as the kernels see it (device pointers).
+struct GraphView {
+    const int64_t *__restrict__ rp;    // row_ptr[n+1]
+    const int32_t *__restrict__ col;   // col_idx[nnz] (+16 B zero padding for 16-B bulk copies)
+    const uint8_t *__restrict__ w;     // weights[nnz] or nullptr
+    int64_t n, nnz;
+    int64_t nw1, nw2;
+};
+
+// Per-superstep control block, device resident; host reads it back with one 64-B copy.
+struct DevStats {
+    unsigned long long count;        // non-zero layer-1 words listed in offsets (summary compaction)
+    unsigned long long nf;           // active vertices (popcount) — direction policy
+    unsigned long long mf;           // sum of active vertices' degrees — direction policy
+    unsigned long long arcs;         // arcs inspected by the advance
+    unsigned long long batch;        // push: next word batch (dynamic CTA scheduling)
+    unsigned long long heavy_count;  // push: CTA/grid-tier chunks queued
+    unsigned long long changed;      // algorithm-specific flag/counter
+    unsigned long long pad;
+};
+
+// One CTA/grid-tier work unit: a contiguous piece of one vertex's adjacency list.
+struct HeavyItem {
+    int64_t begin;   // first arc index
+    int32_t len;     // number of arcs (<= HEAVY_CHUNK)
+    int32_t u;       // source vertex
+};
+
+constexpr int HEAVY_CHUNK = 4096;     // arcs per CTA-tier work unit (16 KB of col_idx)
+
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+__device__ __forceinline__ unsigned long long atomic_or_u64(uint64_t *p, uint64_t m) {
+    return atomicOr(reinterpret_cast<unsigned long long *>(p), (unsigned long long)m);
+}
+
+// Insert v into a 2LB frontier; returns true iff this call flipped v's bit (0 -> 1).
+// The summary bit is touched only on the word's 0 -> non-zero transition.
+__device__ __forceinline__ bool insert_2lb(uint64_t *bits, uint64_t *summ, int32_t v) {
+    const uint64_t m = 1ull << (v & 63);
+    const unsigned long long old = atomic_or_u64(bits + (v >> 6), m);
+    if (old == 0ull) atomic_or_u64(summ + (v >> 12), 1ull << ((v >> 6) & 63));
+    return (old & m) == 0ull;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_inclusive_scan(T x) {
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        T y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane_id() >= o) x += y;
+    }
+    return x;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T x) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+    return x;
+}
+
+// Plain (L1-cacheable) 64-bit load of a word that other threads may be updating with
+// atomics during the kernel: a stale value only costs an extra atomic, never correctness.
+__device__ __forceinline__ uint64_t ld_word(const uint64_t *p) { return *p; }
+
+// Load row_ptr bounds for the (up to) two vertices a = 64w + lane, b = 64w + 32 + lane of a
+// word.  Dense words read rp[64w .. 64w+64] coalesced (3 warp loads); sparse words let only
+// active lanes read their two entries.
+__device__ __forceinline__ void word_bounds(const GraphView &g, int64_t w, uint64_t x, int64_t &sa, int64_t &ea,
+                                            int64_t &sb, int64_t &eb) {
+    const int lane = lane_id();
+    const bool act_a = (x >> lane) & 1ull, act_b = (x >> (lane + 32)) & 1ull;
+    const int64_t base = w * 64;
+    if (__popcll(x) > 12) {
+        const int64_t n = g.n;
+        const int64_t r0 = __ldg(g.rp + min(base + lane, n));
+        const int64_t r1 = __ldg(g.rp + min(base + 32 + lane, n));
+        const int64_t r2 = __ldg(g.rp + min(base + 64, n));
+        const int64_t r0n = __shfl_down_sync(0xffffffffu, r0, 1);
+        const int64_t r1n = __shfl_down_sync(0xffffffffu, r1, 1);
+        const int64_t r1f = __shfl_sync(0xffffffffu, r1, 0);
+        sa = r0; ea = lane < 31 ? r0n : r1f;
+        sb = r1; eb = lane < 31 ? r1n : r2;
+        if (!act_a) ea = sa;
+        if (!act_b) eb = sb;
+    } else {
+        sa = ea = sb = eb = 0;
+        if (act_a) { sa = __ldg(g.rp + base + lane); ea = __ldg(g.rp + base + lane + 1); }
+        if (act_b) { sb = __ldg(g.rp + base + 32 + lane); eb = __ldg(g.rp + base + 33 + lane); }
+    }
+}
+
+}  // namespace sg

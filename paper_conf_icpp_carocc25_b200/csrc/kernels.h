@@ -1,0 +1,70 @@
+// kernels.h — host-side launchers of the sm_100a kernels (internal to libsygraph).
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+#include "common.cuh"
+
+namespace sg {
+
+struct PushParams;
+
+// frontier.cu
+void launch_fill_all(uint64_t *bits, uint64_t *summ, int64_t n, int64_t nw1, int64_t nw2, cudaStream_t s);
+void launch_insert(uint64_t *bits, uint64_t *summ, const int32_t *v, int64_t k, int64_t n, cudaStream_t s);
+void launch_setop(uint64_t *dst, const uint64_t *src, int64_t nw1, int op, cudaStream_t s);
+void launch_rebuild_summary(const uint64_t *bits, uint64_t *summ, int64_t nw1, int64_t nw2, cudaStream_t s);
+void launch_compact(const uint64_t *summ, int64_t nw2, uint32_t *offsets, DevStats *st, cudaStream_t s);
+void launch_frontier_stats(const GraphView &g, const uint64_t *bits, const uint32_t *offsets, DevStats *st,
+                           int64_t max_words, cudaStream_t s);
+void launch_popcount(const uint64_t *bits, int64_t nw1, unsigned long long *out, cudaStream_t s);
+void launch_or_listed(const uint64_t *bits, const uint32_t *offsets, const DevStats *st, uint64_t *dst,
+                      int64_t max_words, cudaStream_t s);
+void launch_or_all(const uint64_t *bits, int64_t nw1, uint64_t *dst, cudaStream_t s);
+void launch_set_u32(uint32_t *p, int64_t i, uint32_t v, cudaStream_t s);
+void launch_set_i32(int32_t *p, int64_t i, int32_t v, cudaStream_t s);
+void launch_set_f64(double *p, int64_t i, double v, cudaStream_t s);
+void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s);
+void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, cudaStream_t s);
+void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s);
+void launch_max_weight(const uint8_t *w, int64_t nnz, unsigned int *out, cudaStream_t s);
+
+// push.cu — one push advance = k_push_words (+ k_push_heavy), functor selected by `fn`.
+struct PushLaunch {
+    GraphView g;
+    const uint64_t *in_bits;
+    const uint32_t *offsets;
+    DevStats *st;
+    HeavyItem *heavy;
+    uint32_t heavy_cap;
+    int32_t heavy_deg, small_deg;
+    int32_t batch;      // words per CTA grab (coarsening factor x 8 warps)
+    int grid_words;     // CTAs for k_push_words
+    int grid_heavy;     // CTAs for k_push_heavy
+};
+struct BfsArgs { uint64_t *visited; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; };
+struct SsspArgs { uint32_t *dist; uint64_t *out_bits, *out_summ; };
+struct CcArgs { int32_t *label; uint64_t *out_bits, *out_summ; };
+struct BcArgs { const uint64_t *visited; double *sigma; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; };
+void launch_push_bfs(const PushLaunch &L, const BfsArgs &a, cudaStream_t s);
+void launch_push_sssp(const PushLaunch &L, const SsspArgs &a, cudaStream_t s);
+void launch_push_cc(const PushLaunch &L, const CcArgs &a, cudaStream_t s);
+void launch_push_bc(const PushLaunch &L, const BcArgs &a, cudaStream_t s);
+int push_max_grid_words();
+int push_max_grid_heavy();
+
+// pull.cu — bottom-up BFS step (direction-optimising, Beamer)
+void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
+                     uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s);
+
+// bc.cu — Brandes helpers
+void launch_bc_level_max(const double *sigma, const uint64_t *bits, const uint32_t *offsets, const DevStats *st,
+                         int64_t max_words, unsigned long long *max_bits, cudaStream_t s);
+void launch_bc_level_scale_and_stack(double *sigma, const uint64_t *bits, const uint32_t *offsets,
+                                     const DevStats *st, int64_t max_words, const unsigned long long *max_bits,
+                                     int32_t *exp_of_level, uint32_t level_idx, int32_t *stack,
+                                     unsigned long long *stack_top, unsigned long long *underflow, cudaStream_t s);
+void launch_bc_backward_level(const GraphView &g, const int32_t *stack, int64_t lo, int64_t hi, const uint32_t *level,
+                              const double *sigma, double *delta, const int32_t *exp_of_level, uint32_t d,
+                              double *bc, int32_t src, cudaStream_t s);
+
+}  // namespace sg

@@ -1,0 +1,324 @@
+// push.cuh — the load-balanced push advance over a Two-Layer-Bitmap frontier
+// (PAPER.md:231-233 §4.2 workload mapping, :249-262 §4.3 2LB + offsets buffer).
+//
+// B200 design:
+//   * the offsets buffer (non-zero layer-1 words, from k_compact) is consumed by persistent
+//     CTAs that grab batches of PUSH_BATCH words with one atomic per batch (the paper's
+//     "set number of workgroups iterating over the offsets buffer", with its
+//     coarsening factor);
+//   * one warp owns one 64-bit word (2 bits per lane: the paper's MSI for 64-bit words)
+//     and splits its active vertices into degree tiers:
+//       - thread tier  (deg <= small_deg): the warp packs all such vertices' arcs into one
+//         list and gives each lane single arcs (ballot/popc start-mask mapping, no search),
+//         so a word with one or two low-degree vertices does not idle 31 lanes (Fig. 5b);
+//       - warp tier    (small_deg < deg <= heavy_deg): the warp streams the list with
+//         16-byte vectorised col_idx loads, 8 arcs in flight per lane;
+//       - CTA/grid tier (deg > heavy_deg): the list is cut into HEAVY_CHUNK-arc chunks queued
+//         in global memory and expanded by k_push_heavy, whose CTAs stage each chunk into
+//         shared memory with cp.async.bulk (TMA bulk copy, mbarrier completion) in a
+//         HEAVY_STAGES-deep ring; a hub's chunks spread across all CTAs (grid tier);
+//   * per arc: probe (one random load: visited word / dist / label) issued for all arcs in
+//     flight before any decision, then the functor's act (atomics on 64-bit words, summary
+//     bit only on the word's 0 -> non-zero transition).
+#pragma once
+#include "common.cuh"
+#include "functors.cuh"
+
+namespace sg {
+
+constexpr int PUSH_THREADS = 256;
+constexpr int PUSH_WARPS = PUSH_THREADS / 32;
+constexpr int HEAVY_THREADS = 256;
+constexpr int HEAVY_STAGES = 4;
+constexpr int HEAVY_BUF_INTS = HEAVY_CHUNK + 8;   // alignment slack for 16-B bulk copies
+constexpr size_t HEAVY_SMEM = (size_t)HEAVY_STAGES * HEAVY_BUF_INTS * 4 + HEAVY_STAGES * 8;
+
+struct PushParams {
+    GraphView g;
+    const uint64_t *in_bits;
+    const uint32_t *offsets;
+    DevStats *st;          // count (input), batch / heavy_count / arcs (scratch, zeroed by host)
+    HeavyItem *heavy;
+    uint32_t heavy_cap;
+    int32_t heavy_deg;
+    int32_t small_deg;
+    int32_t batch;         // words per CTA grab (multiple of PUSH_WARPS)
+};
+
+template <class F>
+struct PushWarpSmem {
+    int64_t start[64];
+    uint32_t pre[64];
+    typename F::Ctx ctx[64];
+};
+
+template <class F>
+__device__ __forceinline__ uint32_t load_w(const GraphView &g, int64_t i) {
+    if constexpr (F::kWeights) return __ldg(g.w + i);
+    else return 0u;
+}
+
+// ---- warp tier -------------------------------------------------------------------------
+template <class F>
+__device__ __forceinline__ void warp_expand(const GraphView &g, const F &f, int64_t s, int64_t e,
+                                            typename F::Ctx c) {
+    const int lane = lane_id();
+    int64_t a = (s + 3) & ~3ll;
+    if (a > e) a = e;
+    const int64_t b = a + ((e - a) & ~3ll);
+    {   // ragged head [s, a) on lanes 0..2 and tail [b, e) on lanes 4..6
+        int64_t i = -1;
+        if (lane < a - s) i = s + lane;
+        else if (lane >= 4 && lane - 4 < e - b) i = b + (lane - 4);
+        if (i >= 0) {
+            const int32_t v = __ldg(g.col + i);
+            const uint32_t w = load_w<F>(g, i);
+            f.act(c, v, w, f.probe(v));
+        }
+    }
+    for (int64_t i = a + 4 * lane; i < b; i += 256) {
+        const bool two = i + 128 < b;
+        const int4 v0 = __ldg(reinterpret_cast<const int4 *>(g.col + i));
+        int4 v1 = make_int4(0, 0, 0, 0);
+        if (two) v1 = __ldg(reinterpret_cast<const int4 *>(g.col + i + 128));
+        uint32_t w0 = 0, w1 = 0;
+        if constexpr (F::kWeights) {
+            w0 = __ldg(reinterpret_cast<const uint32_t *>(g.w + i));
+            if (two) w1 = __ldg(reinterpret_cast<const uint32_t *>(g.w + i + 128));
+        }
+        typename F::Probe p0 = f.probe(v0.x), p1 = f.probe(v0.y), p2 = f.probe(v0.z), p3 = f.probe(v0.w);
+        typename F::Probe q0{}, q1{}, q2{}, q3{};
+        if (two) { q0 = f.probe(v1.x); q1 = f.probe(v1.y); q2 = f.probe(v1.z); q3 = f.probe(v1.w); }
+        f.act(c, v0.x, w0 & 0xff, p0);
+        f.act(c, v0.y, (w0 >> 8) & 0xff, p1);
+        f.act(c, v0.z, (w0 >> 16) & 0xff, p2);
+        f.act(c, v0.w, w0 >> 24, p3);
+        if (two) {
+            f.act(c, v1.x, w1 & 0xff, q0);
+            f.act(c, v1.y, (w1 >> 8) & 0xff, q1);
+            f.act(c, v1.z, (w1 >> 16) & 0xff, q2);
+            f.act(c, v1.w, w1 >> 24, q3);
+        }
+    }
+}
+
+// ---- CTA/grid tier enqueue -------------------------------------------------------------
+__device__ __forceinline__ void enqueue_heavy(const PushParams &p, int32_t u, int64_t s, int64_t e) {
+    const int64_t d = e - s;
+    const uint32_t nch = (uint32_t)((d + HEAVY_CHUNK - 1) / HEAVY_CHUNK);
+    const unsigned long long pos = atomicAdd(&p.st->heavy_count, (unsigned long long)nch);
+    for (uint32_t j = 0; j < nch; j++) {
+        if (pos + j >= p.heavy_cap) break;      // cannot happen: capacity bound in DESIGN.md
+        HeavyItem it;
+        it.begin = s + (int64_t)j * HEAVY_CHUNK;
+        it.len = (int32_t)min((int64_t)HEAVY_CHUNK, e - it.begin);
+        it.u = u;
+        p.heavy[pos + j] = it;
+    }
+}
+
+// ---- one word on one warp ----------------------------------------------------------------
+template <class F>
+__device__ __forceinline__ unsigned long long push_word(const PushParams &p, const F &f, int64_t w,
+                                                        PushWarpSmem<F> &sm) {
+    const int lane = lane_id();
+    const uint64_t x = __ldg(p.in_bits + w);
+    int64_t sa, ea, sb, eb;
+    word_bounds(p.g, w, x, sa, ea, sb, eb);
+    const int32_t ua = (int32_t)(w * 64 + lane), ub = ua + 32;
+    const int64_t da = ea - sa, db = eb - sb;
+    const bool ha = da > p.heavy_deg, hb = db > p.heavy_deg;
+    if (ha) enqueue_heavy(p, ua, sa, ea);
+    if (hb) enqueue_heavy(p, ub, sb, eb);
+    const bool ma = !ha && da > p.small_deg, mb = !hb && db > p.small_deg;
+    const bool ta = da > 0 && da <= p.small_deg, tb = db > 0 && db <= p.small_deg;
+    typename F::Ctx ca{}, cb{};
+    if (ma || ta) ca = f.ctx(ua);
+    if (mb || tb) cb = f.ctx(ub);
+
+    // warp tier: one vertex at a time, whole warp
+    uint32_t mm = __ballot_sync(0xffffffffu, ma);
+    while (mm) {
+        const int src = __ffs(mm) - 1;
+        mm &= mm - 1;
+        warp_expand(p.g, f, __shfl_sync(0xffffffffu, sa, src), __shfl_sync(0xffffffffu, ea, src),
+                    __shfl_sync(0xffffffffu, ca, src));
+    }
+    mm = __ballot_sync(0xffffffffu, mb);
+    while (mm) {
+        const int src = __ffs(mm) - 1;
+        mm &= mm - 1;
+        warp_expand(p.g, f, __shfl_sync(0xffffffffu, sb, src), __shfl_sync(0xffffffffu, eb, src),
+                    __shfl_sync(0xffffffffu, cb, src));
+    }
+
+    // thread tier: pack the low-degree vertices' arcs, one arc per lane per window
+    const uint32_t la = ta ? (uint32_t)da : 0u, lb = tb ? (uint32_t)db : 0u;
+    const uint32_t mine = la + lb;
+    const uint32_t incl = warp_inclusive_scan(mine);
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    if (total) {
+        const uint32_t pa = incl - mine, pb = pa + la;
+        const uint32_t bal_a = __ballot_sync(0xffffffffu, ta), bal_b = __ballot_sync(0xffffffffu, tb);
+        const uint32_t lt = (1u << lane) - 1u;
+        const int slot_a = __popc(bal_a & lt) + __popc(bal_b & lt);
+        const int slot_b = slot_a + (ta ? 1 : 0);
+        if (ta) { sm.start[slot_a] = sa; sm.pre[slot_a] = pa; sm.ctx[slot_a] = ca; }
+        if (tb) { sm.start[slot_b] = sb; sm.pre[slot_b] = pb; sm.ctx[slot_b] = cb; }
+        __syncwarp();
+        int kb = -1;
+        for (uint32_t base = 0; base < total; base += 64) {
+            // bit (P_k - base) marks vertex k's first arc inside this 64-arc window
+            uint64_t m = 0;
+            if (ta && pa >= base && pa < base + 64) m |= 1ull << (pa - base);
+            if (tb && pb >= base && pb < base + 64) m |= 1ull << (pb - base);
+            const uint32_t lo = __reduce_or_sync(0xffffffffu, (uint32_t)m);
+            const uint32_t hi = __reduce_or_sync(0xffffffffu, (uint32_t)(m >> 32));
+            const uint64_t mask = (uint64_t)lo | ((uint64_t)hi << 32);
+            const int k0 = kb + __popcll(mask & ((2ull << lane) - 1ull));
+            const int k1 = kb + __popcll(mask & ((2ull << (lane + 32)) - 1ull));
+            const uint32_t e0 = base + lane, e1 = base + 32 + lane;
+            const bool ok0 = e0 < total, ok1 = e1 < total;
+            int32_t v0 = 0, v1 = 0;
+            uint32_t w0 = 0, w1 = 0;
+            typename F::Ctx c0{}, c1{};
+            if (ok0) {
+                const int64_t i = sm.start[k0] + (e0 - sm.pre[k0]);
+                v0 = __ldg(p.g.col + i);
+                w0 = load_w<F>(p.g, i);
+                c0 = sm.ctx[k0];
+            }
+            if (ok1) {
+                const int64_t i = sm.start[k1] + (e1 - sm.pre[k1]);
+                v1 = __ldg(p.g.col + i);
+                w1 = load_w<F>(p.g, i);
+                c1 = sm.ctx[k1];
+            }
+            typename F::Probe p0{}, p1{};
+            if (ok0) p0 = f.probe(v0);
+            if (ok1) p1 = f.probe(v1);
+            if (ok0) f.act(c0, v0, w0, p0);
+            if (ok1) f.act(c1, v1, w1, p1);
+            kb += __popcll(mask);
+        }
+        __syncwarp();
+    }
+    return (unsigned long long)(da + db);
+}
+
+template <class F>
+__global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) {
+    __shared__ PushWarpSmem<F> s_warp[PUSH_WARPS];
+    __shared__ uint32_t s_batch;
+    __shared__ unsigned long long s_arcs[PUSH_WARPS];
+    const uint32_t count = (uint32_t)p.st->count;
+    const int wid = threadIdx.x >> 5;
+    unsigned long long arcs = 0;
+    for (;;) {
+        if (threadIdx.x == 0) s_batch = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)p.batch);
+        __syncthreads();
+        const uint32_t b0 = s_batch;
+        __syncthreads();
+        if (b0 >= count) break;
+        const uint32_t b1 = min(b0 + (uint32_t)p.batch, count);
+        for (uint32_t i = b0 + wid; i < b1; i += PUSH_WARPS) arcs += push_word(p, f, p.offsets[i], s_warp[wid]);
+    }
+    arcs = warp_sum(arcs);
+    if (lane_id() == 0) s_arcs[wid] = arcs;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t = 0;
+        for (int i = 0; i < PUSH_WARPS; i++) t += s_arcs[i];
+        if (t) atomicAdd(&p.st->arcs, t);
+    }
+}
+
+// ---- CTA/grid tier: TMA-bulk-staged chunks ---------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void *ptr) {
+    return (uint32_t)__cvta_generic_to_shared(ptr);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase) {
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(phase)
+            : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void bulk_g2s(void *dst_smem, const void *src_gmem, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst_smem)),
+        "l"(src_gmem), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+template <class F>
+__global__ void __launch_bounds__(HEAVY_THREADS) k_push_heavy(PushParams p, F f) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    int32_t *buf = reinterpret_cast<int32_t *>(smem_raw);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem_raw + (size_t)HEAVY_STAGES * HEAVY_BUF_INTS * 4);
+    const unsigned long long hc = p.st->heavy_count;
+    const uint32_t nitems = (uint32_t)(hc < p.heavy_cap ? hc : p.heavy_cap);
+    const uint32_t G = gridDim.x;
+    const uint32_t my_n = nitems > blockIdx.x ? (nitems - blockIdx.x + G - 1) / G : 0u;
+    if (my_n == 0) return;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < HEAVY_STAGES; s++) mbar_init(bar + s, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    auto issue = [&](uint32_t j) {
+        const HeavyItem it = p.heavy[blockIdx.x + (size_t)j * G];
+        const int64_t a = it.begin & ~3ll;
+        const int64_t b = (it.begin + it.len + 3) & ~3ll;
+        const uint32_t bytes = (uint32_t)((b - a) * 4);
+        const int s = j % HEAVY_STAGES;
+        mbar_expect_tx(bar + s, bytes);
+        bulk_g2s(buf + (size_t)s * HEAVY_BUF_INTS, p.g.col + a, bytes, bar + s);
+    };
+    if (threadIdx.x == 0)
+        for (uint32_t j = 0; j < my_n && j < (uint32_t)HEAVY_STAGES; j++) issue(j);
+    for (uint32_t j = 0; j < my_n; j++) {
+        const int s = j % HEAVY_STAGES;
+        const uint32_t phase = (j / HEAVY_STAGES) & 1u;
+        const HeavyItem it = p.heavy[blockIdx.x + (size_t)j * G];
+        const typename F::Ctx c = f.ctx(it.u);
+        mbar_wait(bar + s, phase);
+        const int32_t *src = buf + (size_t)s * HEAVY_BUF_INTS + (it.begin & 3);
+        for (int i = threadIdx.x; i < it.len; i += HEAVY_THREADS * 4) {
+            int32_t v[4];
+            uint32_t w[4];
+            bool ok[4];
+            typename F::Probe pr[4];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                const int ii = i + k * HEAVY_THREADS;
+                ok[k] = ii < it.len;
+                v[k] = ok[k] ? src[ii] : 0;
+                w[k] = ok[k] ? load_w<F>(p.g, it.begin + ii) : 0u;
+            }
+#pragma unroll
+            for (int k = 0; k < 4; k++)
+                if (ok[k]) pr[k] = f.probe(v[k]);
+#pragma unroll
+            for (int k = 0; k < 4; k++)
+                if (ok[k]) f.act(c, v[k], w[k], pr[k]);
+        }
+        __syncthreads();   // buffer s fully consumed
+        if (threadIdx.x == 0 && j + HEAVY_STAGES < my_n) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            issue(j + HEAVY_STAGES);
+        }
+    }
+}
+
+}  // namespace sg

@@ -1,0 +1,312 @@
+"""GPU parity: the CUDA path (through the C ABI) against the pinned oracle, element by element.
+
+BFS levels, SSSP distances and CC labels must be bit-exact; BC within
+|g - o| <= 1e-9 * max(|o|, 1) (north_star; reading C21).  Sizes span several tiles
+and ragged tails; tier-forcing options must not change any result."""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from golden import twolayer_example
+
+pytestmark = pytest.mark.gpu
+
+INF = 0xFFFFFFFF
+
+
+@pytest.fixture(scope="module")
+def sg():
+    import torch
+    import paper_conf_icpp_carocc25_b200 as m
+    torch.cuda.set_device(0)
+    return m
+
+
+def load(sg, g):
+    return sg.graph_load_csr(g.row_ptr, g.col_idx, g.weights, validate=True)
+
+
+def bc_close(got, ref, tol=1e-9):
+    return np.all(np.abs(got - ref) <= tol * np.maximum(np.abs(ref), 1.0))
+
+
+# ------------------------------------------------------------------ frontier / 2LB layout
+def test_frontier_layout_matches_handworked_fixture(sg):
+    import torch
+    n, active, words, summ = twolayer_example()
+    g = gen.empty_graph(n)
+    G = load(sg, g)
+    f = sg.frontier_init(G)
+    sg.frontier_insert(f, active.astype(np.int32))
+    bits, sm = sg.frontier_view(f)
+    torch.cuda.synchronize()
+    assert np.array_equal(bits.cpu().numpy().view(np.uint64), words)
+    assert np.array_equal(sm.cpu().numpy().view(np.uint64), summ)
+    assert sg.frontier_count(f) == len(active)
+
+
+@pytest.mark.parametrize("n", [1, 63, 64, 65, 4095, 4096, 4097, 100_003])
+def test_fill_all_tail_and_count(sg, n):
+    g = gen.empty_graph(n)
+    G = load(sg, g)
+    f = sg.frontier_init(G)
+    sg.frontier_fill_all(f)
+    bits, summ = sg.frontier_view(f)
+    mask = np.ones(n, bool)
+    w = oracle.bitmap_words(mask) if n <= 5000 else None
+    b = bits.cpu().numpy().view(np.uint64)
+    if w is not None:
+        assert np.array_equal(b, w)
+        assert np.array_equal(summ.cpu().numpy().view(np.uint64), oracle.summary_words(w))
+    assert sg.frontier_count(f) == n
+    sg.frontier_clear(f)
+    assert sg.frontier_count(f) == 0
+
+
+def test_frontier_set_ops(sg):
+    n = 20_000
+    rng = np.random.default_rng(5)
+    a = rng.random(n) < 0.1
+    b = rng.random(n) < 0.05
+    G = load(sg, gen.empty_graph(n))
+    for op, fn in enumerate([np.logical_or, np.logical_and, lambda x, y: x & ~y, np.logical_xor]):
+        fa, fb = sg.frontier_init(G), sg.frontier_init(G)
+        sg.frontier_insert(fa, np.nonzero(a)[0].astype(np.int32))
+        sg.frontier_insert(fb, np.nonzero(b)[0].astype(np.int32))
+        sg.frontier_op(fa, fb, op)
+        bits, summ = sg.frontier_view(fa)
+        exp = oracle.bitmap_words(fn(a, b))
+        assert np.array_equal(bits.cpu().numpy().view(np.uint64), exp)
+        assert np.array_equal(summ.cpu().numpy().view(np.uint64), oracle.summary_words(exp))
+
+
+# ------------------------------------------------------------------------------- BFS
+DIRS = ["push", "pull", "auto"]
+
+
+def _dir(sg, d):
+    return {"push": sg.SG_DIR_PUSH, "pull": sg.SG_DIR_PULL, "auto": sg.SG_DIR_AUTO}[d]
+
+
+@pytest.mark.parametrize("direction", DIRS)
+def test_bfs_config1(sg, direction):
+    g = gen.rmat(10, 16)
+    G = load(sg, g)
+    lv, st = sg.run_bfs(G, 0, direction=_dir(sg, direction))
+    assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, 0))
+
+
+@pytest.mark.parametrize("opts", [dict(), dict(heavy_degree=1), dict(heavy_degree=40), dict(small_degree=-1),
+                                  dict(small_degree=100000, heavy_degree=100000), dict(small_degree=3, heavy_degree=7)])
+def test_bfs_tier_forcing_invariant(sg, opts):
+    g = gen.rmat(14, 16, permute=True)
+    G = load(sg, g)
+    for s in gen.sources(g, 3):
+        lv, _ = sg.run_bfs(G, int(s), direction=sg.SG_DIR_PUSH, **opts)
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (opts, s)
+
+
+@pytest.mark.parametrize("make", [lambda: gen.path(5000), lambda: gen.cycle(4097), lambda: gen.grid(97, 131),
+                                  lambda: gen.hypercube(16), lambda: gen.complete(300), lambda: gen.star(70_000),
+                                  lambda: gen.lattice(300, 400, 0.6)])
+@pytest.mark.parametrize("direction", DIRS)
+def test_bfs_closed_form_families(sg, make, direction):
+    g = make()
+    G = load(sg, g)
+    for s in [0, g.n // 2, g.n - 1]:
+        lv, _ = sg.run_bfs(G, s, direction=_dir(sg, direction))
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, s))
+
+
+@pytest.mark.parametrize("deg", [1, 31, 32, 33, 2047, 2048, 2049, 4095, 4096, 4097, 65536, 200_001])
+def test_bfs_degree_tier_boundaries(sg, deg):
+    # a hub of degree `deg` plus a tail path so several levels exist
+    n = deg + 1 + 50
+    u = np.concatenate([np.zeros(deg, np.int64), np.arange(deg, n - 1)])
+    v = np.concatenate([np.arange(1, deg + 1), np.arange(deg + 1, n)])
+    g = gen.from_edges(n, u, v)
+    G = load(sg, g)
+    for s in (0, 1, n - 1):
+        for d in (sg.SG_DIR_PUSH, sg.SG_DIR_AUTO):
+            lv, _ = sg.run_bfs(G, s, direction=d)
+            assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, s)), (deg, s, d)
+
+
+def test_bfs_isolated_source_and_empty_graph(sg):
+    g = gen.rmat(10, 16)
+    iso = int(np.nonzero(g.degrees() == 0)[0][0])
+    G = load(sg, g)
+    lv, st = sg.run_bfs(G, iso)
+    exp = np.full(g.n, INF, np.uint32)
+    exp[iso] = 0
+    assert np.array_equal(sg.as_u32(lv), exp) and st.iterations == 1
+    G0 = load(sg, gen.empty_graph(1))
+    lv, _ = sg.run_bfs(G0, 0)
+    assert sg.as_u32(lv)[0] == 0
+
+
+def test_bfs_rejects_bad_source(sg):
+    G = load(sg, gen.path(10))
+    with pytest.raises(sg.SgError):
+        sg.run_bfs(G, 10)
+    with pytest.raises(sg.SgError):
+        sg.run_bfs(G, -1)
+
+
+@pytest.mark.parametrize("direction", DIRS)
+def test_bfs_rmat16_many_sources(sg, direction):
+    g = gen.rmat(16, 32, permute=True)
+    G = load(sg, g)
+    for s in gen.sources(g, 5):
+        lv, _ = sg.run_bfs(G, int(s), direction=_dir(sg, direction))
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s)))
+
+
+# ---------------------------------------------------------------------- one advance step
+def test_single_bfs_advance_step_set_semantics(sg):
+    import torch
+    g = gen.rmat(13, 16, permute=True)
+    G = load(sg, g)
+    s = int(gen.sources(g, 1)[0])
+    lvl = oracle.bfs(g, s)
+    fin, fout = sg.frontier_init(G), sg.frontier_init(G)
+    level = torch.full((g.n,), -1, dtype=torch.int32, device="cuda")
+    visited = torch.zeros((g.n + 63) // 64, dtype=torch.int64, device="cuda")
+    for d in range(int(lvl[lvl != INF].max()) + 1):
+        frontier = lvl == d
+        vis = lvl <= d
+        # state before step d: visited = levels <= d, level set for those
+        visited.copy_(torch.from_numpy(oracle.bitmap_words(vis).view(np.int64)))
+        lv_host = np.where(vis, lvl, INF).astype(np.uint32)
+        level.copy_(torch.from_numpy(lv_host.view(np.int32)))
+        sg.frontier_clear(fin)
+        sg.frontier_clear(fout)
+        sg.frontier_insert(fin, np.nonzero(frontier)[0].astype(np.int32))
+        sg.advance(G, fin, fout, sg.SG_FN_BFS, dict(level=level, visited=visited, depth=d))
+        bits, summ = sg.frontier_view(fout)
+        exp = oracle.bfs_advance_step(g, frontier, vis)
+        ew = oracle.bitmap_words(exp)
+        assert np.array_equal(bits.cpu().numpy().view(np.uint64), ew)
+        assert np.array_equal(summ.cpu().numpy().view(np.uint64), oracle.summary_words(ew))
+        got_lv = sg.as_u32(level)
+        assert np.array_equal(got_lv[exp], np.full(exp.sum(), d + 1, np.uint32))
+
+
+def test_single_relax_step_invariants(sg):
+    """SSSP/CC steps are non-unique under asynchronous updates (reading C12): check
+    out == {v: value decreased}, final >= fixed point, and <= the Jacobi step bound."""
+    import torch
+    g = gen.with_weights(gen.rmat(12, 16, permute=True), seed=4)
+    G = load(sg, g)
+    s = int(gen.sources(g, 1)[0])
+    ref = oracle.sssp(g, s).astype(np.int64)
+    dist = np.full(g.n, INF, np.int64)
+    dist[s] = 0
+    front = np.zeros(g.n, bool)
+    front[s] = True
+    fin, fout = sg.frontier_init(G), sg.frontier_init(G)
+    dd = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    for _ in range(200):
+        if not front.any():
+            break
+        dd.copy_(torch.from_numpy(dist.astype(np.uint32).view(np.int32)))
+        sg.frontier_clear(fin)
+        sg.frontier_clear(fout)
+        sg.frontier_insert(fin, np.nonzero(front)[0].astype(np.int32))
+        sg.advance(G, fin, fout, sg.SG_FN_SSSP, dict(dist=dd))
+        new = sg.as_u32(dd).astype(np.int64)
+        bits, _ = sg.frontier_view(fout)
+        out = oracle.words_to_mask(bits.cpu().numpy().view(np.uint64), g.n)
+        assert np.array_equal(out, new < dist)
+        assert (new >= ref).all()
+        assert (new <= oracle.jacobi_relax_step(g, front, dist, g.weights)).all()
+        dist, front = new, out
+    assert np.array_equal(dist, ref)
+
+
+# ------------------------------------------------------------------------------ SSSP
+@pytest.mark.parametrize("scale,ef,perm", [(10, 16, False), (14, 16, True), (16, 8, False)])
+def test_sssp_rmat(sg, scale, ef, perm):
+    g = gen.with_weights(gen.rmat(scale, ef, permute=perm), seed=1)
+    G = load(sg, g)
+    for s in [0] + list(gen.sources(g, 3)):
+        d, _ = sg.run_sssp(G, int(s))
+        assert np.array_equal(sg.as_u32(d), oracle.sssp(g, int(s)))
+
+
+@pytest.mark.parametrize("opts", [dict(heavy_degree=1), dict(small_degree=-1), dict(small_degree=5000, heavy_degree=5000)])
+def test_sssp_tiers(sg, opts):
+    g = gen.with_weights(gen.rmat(13, 16), seed=2)
+    G = load(sg, g)
+    d, _ = sg.run_sssp(G, 0, **opts)
+    assert np.array_equal(sg.as_u32(d), oracle.sssp(g, 0))
+
+
+def test_sssp_lattice_and_unit_weights(sg):
+    g = gen.with_weights(gen.lattice(200, 300, 0.7), seed=9)
+    G = load(sg, g)
+    s = int(gen.sources(g, 1, stream=6)[0])
+    d, _ = sg.run_sssp(G, s)
+    assert np.array_equal(sg.as_u32(d), oracle.sssp(g, s))
+    g2 = gen.rmat(12, 16)
+    g2.weights = np.ones(g2.nnz, np.uint8)
+    G2 = load(sg, g2)
+    d, _ = sg.run_sssp(G2, 0)
+    assert np.array_equal(sg.as_u32(d), oracle.bfs(g2, 0))
+
+
+def test_sssp_requires_weights(sg):
+    G = load(sg, gen.path(10))
+    with pytest.raises(sg.SgError):
+        sg.run_sssp(G, 0)
+
+
+# -------------------------------------------------------------------------------- CC
+@pytest.mark.parametrize("make", [lambda: gen.gnm(300_000, 150_000, seed=3), lambda: gen.gnm(100_000, 1_200_000),
+                                  lambda: gen.rmat(15, 8, permute=True), lambda: gen.lattice(300, 300, 0.5),
+                                  lambda: gen.empty_graph(1000), lambda: gen.path(3000)])
+def test_cc(sg, make):
+    g = make()
+    G = load(sg, g)
+    lab, _ = sg.run_cc(G)
+    assert np.array_equal(lab.cpu().numpy(), oracle.cc(g))
+
+
+def test_cc_tiers(sg):
+    g = gen.rmat(13, 16)
+    G = load(sg, g)
+    ref = oracle.cc(g)
+    for opts in (dict(heavy_degree=1), dict(small_degree=-1), dict(small_degree=100000, heavy_degree=100000)):
+        lab, _ = sg.run_cc(G, **opts)
+        assert np.array_equal(lab.cpu().numpy(), ref)
+
+
+# -------------------------------------------------------------------------------- BC
+@pytest.mark.parametrize("make,k", [(lambda: gen.random_simple(60, 0.08, 3), 60), (lambda: gen.path(300), 10),
+                                    (lambda: gen.hypercube(10), 5), (lambda: gen.rmat(12, 16, permute=True), 8),
+                                    (lambda: gen.lattice(80, 120, 0.6, seed=2), 6)])
+def test_bc(sg, make, k):
+    g = make()
+    G = load(sg, g)
+    srcs = gen.sources(g, k) if k < g.n else np.arange(g.n, dtype=np.int32)
+    bc, _ = sg.run_bc(G, srcs)
+    assert bc_close(bc.cpu().numpy(), oracle.bc(g, srcs))
+
+
+def test_bc_sigma_beyond_fp64_range(sg):
+    """Full 600x600 grid from a corner: sigma reaches ~2^1193 > DBL_MAX (reading C20); the
+    per-level exponent scaling must keep BC exact to 1e-9."""
+    g = gen.grid(600, 600)
+    G = load(sg, g)
+    srcs = np.array([0, 600 * 600 - 1], np.int32)
+    bc, _ = sg.run_bc(G, srcs)
+    assert bc_close(bc.cpu().numpy(), oracle.bc(g, srcs))
+
+
+def test_bc_duplicates_and_isolated(sg):
+    g = gen.from_edges(8, [0, 1, 2, 3], [1, 2, 3, 4])
+    G = load(sg, g)
+    srcs = [0, 0, 7, 2]
+    bc, _ = sg.run_bc(G, srcs)
+    assert bc_close(bc.cpu().numpy(), oracle.bc(g, srcs))
