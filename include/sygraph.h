@@ -143,6 +143,20 @@ SG_API int run_cc(const sg_graph *g, int32_t *label, const sg_opts *opts, sg_sta
 SG_API int run_bc(const sg_graph *g, const int32_t *sources, int32_t k, double *bc, const sg_opts *opts,
                   sg_stats *stats);
 
+/* ---- measurement (bench.py roofline; not needed for correctness) ----------------------- */
+enum { SG_K_COMPACT = 0, SG_K_STATS = 1, SG_K_PUSH = 2, SG_K_PULL = 3, SG_K_BC = 4, SG_K_COUNT = 5 };
+typedef struct {
+    double ms;                /* summed CUDA-event time of the class's launches (launching stream) */
+    double bytes;             /* summed algorithmic HBM bytes */
+    int64_t launches;         /* profiled launches (a push advance = its word + CTA-tier kernels) */
+} sg_kprof;
+/* Enable (1) / disable (0) per-kernel-class event timing for run_bfs on g; resets totals. */
+SG_API int sg_profile(sg_graph *g, int enable);
+/* Copy the SG_K_COUNT per-class totals. */
+SG_API int sg_profile_read(const sg_graph *g, sg_kprof *out);
+/* Kernel launches issued by this library since load (host-side counter). */
+SG_API int64_t sg_launch_count(void);
+
 /* Defaults for sg_opts (stream NULL, AUTO direction, alpha 14, beta 24). */
 SG_API void sg_opts_default(sg_opts *o);
 /* Thread-local message of the last error on this thread ("" if none). */

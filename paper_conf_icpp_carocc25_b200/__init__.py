@@ -14,7 +14,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "lib", "libsygraph.so")
+LIB_PATH = os.environ.get("SYGRAPH_LIB") or os.path.join(_PKG, "lib", "libsygraph.so")
 
 SG_OK, SG_ERR_INVALID, SG_ERR_OOM, SG_ERR_CUDA, SG_ERR_NCCL, SG_ERR_UNSUPPORTED, SG_ERR_STATE = 0, -1, -2, -3, -4, -5, -6
 SG_MEM_HOST, SG_MEM_DEVICE = 0, 1
@@ -62,11 +62,18 @@ class SgBcState(ctypes.Structure):
                 ("depth", ctypes.c_uint32)]
 
 
+class SgKprof(ctypes.Structure):
+    _fields_ = [("ms", ctypes.c_double), ("bytes", ctypes.c_double), ("launches", ctypes.c_int64)]
+
+
+SG_K_COMPACT, SG_K_STATS, SG_K_PUSH, SG_K_PULL, SG_K_BC, SG_K_COUNT = 0, 1, 2, 3, 4, 5
+K_NAMES = ["compact", "stats", "advance_push", "advance_pull", "bc"]
+
 # every symbol include/sygraph.h declares (checked by tests/test_abi.py)
 EXPORTS = ["graph_load_csr", "graph_free", "graph_info", "frontier_init", "frontier_free", "frontier_insert",
            "frontier_fill_all", "frontier_clear", "frontier_count", "frontier_view", "frontier_op",
            "frontier_or_into", "advance", "run_bfs", "run_sssp", "run_cc", "run_bc", "sg_opts_default",
-           "sg_last_error", "sg_version"]
+           "sg_last_error", "sg_version", "sg_profile", "sg_profile_read", "sg_launch_count"]
 
 _lib = None
 
@@ -102,6 +109,9 @@ def load():
         "sg_opts_default": (None, [ctypes.POINTER(SgOpts)]),
         "sg_last_error": (ctypes.c_char_p, []),
         "sg_version": (ctypes.c_char_p, []),
+        "sg_profile": (c_int, [vp, c_int]),
+        "sg_profile_read": (c_int, [vp, ctypes.POINTER(SgKprof)]),
+        "sg_launch_count": (i64, []),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -325,6 +335,20 @@ def run_bc(g: Graph, sources, bc=None, o: SgOpts | None = None, **kw):
 def as_u32(t) -> np.ndarray:
     """Device int32 tensor holding uint32 values -> host numpy uint32."""
     return t.cpu().numpy().view(np.uint32)
+
+
+def profile(g: Graph, enable: bool = True):
+    _check(load().sg_profile(g.handle, int(enable)))
+
+
+def profile_read(g: Graph) -> dict:
+    arr = (SgKprof * SG_K_COUNT)()
+    _check(load().sg_profile_read(g.handle, arr))
+    return {K_NAMES[i]: dict(ms=arr[i].ms, bytes=arr[i].bytes, launches=arr[i].launches) for i in range(SG_K_COUNT)}
+
+
+def launch_count() -> int:
+    return int(load().sg_launch_count())
 
 
 def version() -> str:

@@ -42,19 +42,23 @@ def _stamp() -> str:
     return h.hexdigest()
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defines=(), lib: str | None = None) -> str:
+    """defines: extra -D macros (tuning variants); lib: output path (default lib/libsygraph.so)."""
+    LIB = lib or globals()["LIB"]
+    BUILD = globals()["BUILD"] + ("_" + hashlib.sha256(" ".join(defines).encode()).hexdigest()[:8] if defines else "")
     stamp_file = LIB + ".stamp"
-    stamp = _stamp()
+    stamp = _stamp() + " ".join(defines)
     if not force and os.path.exists(LIB) and os.path.exists(stamp_file):
         with open(stamp_file) as f:
             if f.read().strip() == stamp:
                 return LIB
     os.makedirs(BUILD, exist_ok=True)
-    os.makedirs(LIB_DIR, exist_ok=True)
+    os.makedirs(os.path.dirname(LIB), exist_ok=True)
 
     def compile_one(src):
         obj = os.path.join(BUILD, os.path.basename(src)[:-3] + ".o")
-        cmd = [NVCC, *ARCH, *FLAGS, "-Xptxas", "-v" if verbose else "-O3", "-c", src, "-o", obj]
+        cmd = [NVCC, *ARCH, *FLAGS, *["-D" + d for d in defines], "-Xptxas", "-v" if verbose else "-O3", "-c", src,
+               "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr}")

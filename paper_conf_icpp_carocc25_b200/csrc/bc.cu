@@ -93,12 +93,14 @@ static int grid_for(int64_t items, int threads, int max_blocks) {
 
 void launch_bc_level_max(const double *sigma, const uint64_t *bits, const uint32_t *offsets, const DevStats *st,
                          int64_t max_words, unsigned long long *max_bits, cudaStream_t s) {
+    note_launch();
     k_bc_level_max<<<grid_for(max_words, 256, 148 * 4), 256, 0, s>>>(sigma, bits, offsets, st, max_bits);
 }
 void launch_bc_level_scale_and_stack(double *sigma, const uint64_t *bits, const uint32_t *offsets,
                                      const DevStats *st, int64_t max_words, const unsigned long long *max_bits,
                                      int32_t *exp_of_level, uint32_t level_idx, int32_t *stack,
                                      unsigned long long *stack_top, unsigned long long *underflow, cudaStream_t s) {
+    note_launch();
     k_bc_scale_stack<<<grid_for(max_words, 256, 148 * 4), 256, 0, s>>>(sigma, bits, offsets, st, max_bits,
                                                                         exp_of_level, level_idx, stack, stack_top,
                                                                         underflow);
@@ -107,6 +109,7 @@ void launch_bc_backward_level(const GraphView &g, const int32_t *stack, int64_t 
                               const double *sigma, double *delta, const int32_t *exp_of_level, uint32_t d,
                               double *bc, int32_t src, cudaStream_t s) {
     if (hi <= lo) return;
+    note_launch();
     k_bc_backward<<<grid_for(hi - lo, 256, 148 * 8), 256, 0, s>>>(g, stack, lo, hi, level, sigma, delta,
                                                                    exp_of_level, d, bc, src);
 }

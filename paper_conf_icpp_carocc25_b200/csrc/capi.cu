@@ -4,8 +4,10 @@
 // the output frontier consistent at the end of the step, swap + clear, stop when the frontier
 // is empty.  Per superstep the host reads back one 128-byte control block (frontier sizes for
 // empty() and the direction policy); everything else stays on the device stream.
+#include <atomic>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -14,6 +16,11 @@
 #include "kernels.h"
 
 using namespace sg;
+
+namespace sg {
+static std::atomic<long long> g_launches{0};
+void note_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+}  // namespace sg
 
 // ------------------------------------------------------------------------------------------
 // errors
@@ -52,7 +59,25 @@ struct sg_frontier {
     bool owns_st = true;
 };
 
+// Optional per-kernel-class timing (CUDA events on the launching stream) + algorithmic bytes
+// (DESIGN.md §6 "Measurement").  Off by default; bench.py turns it on for the roofline.
+struct ProfRec {
+    int cls;
+    cudaEvent_t a, b;
+    double bytes;
+};
+struct Prof {
+    bool on = false;
+    std::vector<cudaEvent_t> pool;
+    size_t used = 0;
+    std::vector<ProfRec> recs;
+    double ms[SG_K_COUNT] = {0};
+    double bytes[SG_K_COUNT] = {0};
+    int64_t launches[SG_K_COUNT] = {0};
+};
+
 struct Workspace {
+    Prof prof;
     sg_frontier fr[2];
     DevStats *st = nullptr;        // 2 contiguous control blocks (fr[0].st, fr[1].st)
     DevStats *h_st = nullptr;      // pinned host mirror
@@ -75,6 +100,8 @@ struct sg_graph {
     int64_t *rp = nullptr;
     int32_t *col = nullptr;
     uint8_t *w = nullptr;
+    uint8_t *deg8 = nullptr;
+    uint64_t *isolated = nullptr;   // bit v <=> deg(v) == 0
     uint32_t max_w = 0;
     int device = 0;
     Workspace *ws = nullptr;
@@ -156,6 +183,7 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->level);
     if (ws->ev0) cudaEventDestroy(ws->ev0);
     if (ws->ev1) cudaEventDestroy(ws->ev1);
+    for (cudaEvent_t e : ws->prof.pool) cudaEventDestroy(e);
     delete ws;
 }
 
@@ -223,6 +251,11 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     g->v.rp = g->rp;
     g->v.col = g->col;
     g->v.w = g->w;
+    CK(cudaMalloc(&g->deg8, (size_t)g->v.nw1 * 64));
+    launch_deg8(g->rp, n, g->v.nw1 * 64, g->deg8, s);
+    g->v.deg8 = g->deg8;
+    CK(cudaMalloc(&g->isolated, sizeof(uint64_t) * (size_t)g->v.nw1));
+    launch_isolated(g->deg8, n, g->v.nw1, g->isolated, s);
     unsigned long long *dscr = nullptr;
     CK(cudaMalloc(&dscr, 16));
     CK(cudaMemsetAsync(dscr, 0, 16, s));
@@ -248,6 +281,8 @@ SG_API int graph_free(sg_graph *g) {
     cudaFree(g->rp);
     cudaFree(g->col);
     cudaFree(g->w);
+    cudaFree(g->deg8);
+    cudaFree(g->isolated);
     delete g;
     return SG_OK;
 }
@@ -391,7 +426,7 @@ static Tiers tiers_from(const sg_opts *o) {
 static int compact(const sg_graph *g, const sg_frontier *f, bool stats, cudaStream_t s) {
     CK(cudaMemsetAsync(f->st, 0, sizeof(DevStats), s));
     launch_compact(f->summ, g->v.nw2, f->offsets, f->st, s);
-    if (stats) launch_frontier_stats(g->v, f->bits, f->offsets, f->st, g->v.nw1, s);
+    if (stats) launch_frontier_stats(g->v, f->bits, f->st, s);
     return SG_OK;
 }
 
@@ -406,15 +441,16 @@ static PushLaunch push_launch(const sg_graph *g, const sg_frontier *in, Tiers t,
     L.heavy_deg = t.heavy;
     L.small_deg = t.small;
     const int maxg = push_max_grid_words();
+    // batch = words per warp grab (coarsening factor): ~4 grabs per warp, 1..8 words
     if (count_hint < 0) {
-        L.batch = 32;
+        L.batch = 4;
         L.grid_words = maxg;
     } else {
-        int64_t cf = count_hint / ((int64_t)maxg * 8 * 2);
+        int64_t cf = count_hint / ((int64_t)maxg * 8 * 4);
         if (cf < 1) cf = 1;
         if (cf > 8) cf = 8;
-        L.batch = (int32_t)(8 * cf);
-        int64_t gw = (count_hint + L.batch - 1) / L.batch;
+        L.batch = (int32_t)cf;
+        int64_t gw = (count_hint + 8 * L.batch - 1) / (8 * L.batch);
         if (gw < 1) gw = 1;
         if (gw > maxg) gw = maxg;
         L.grid_words = (int)gw;
@@ -428,6 +464,46 @@ static int read_stats(Workspace *ws, cudaStream_t s) {
     CK(cudaStreamSynchronize(s));
     CK(cudaGetLastError());
     return SG_OK;
+}
+
+static cudaEvent_t prof_event(Prof &P) {
+    if (P.used == P.pool.size()) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        P.pool.push_back(e);
+    }
+    return P.pool[P.used++];
+}
+// returns the record index (or -1 when profiling is off)
+static int prof_begin(Workspace *ws, int cls, cudaStream_t s) {
+    Prof &P = ws->prof;
+    if (!P.on) return -1;
+    ProfRec r{cls, prof_event(P), prof_event(P), 0.0};
+    if (!r.a || !r.b) return -1;
+    cudaEventRecord(r.a, s);
+    P.recs.push_back(r);
+    return (int)P.recs.size() - 1;
+}
+static void prof_end(Workspace *ws, int idx, cudaStream_t s) {
+    if (idx >= 0) cudaEventRecord(ws->prof.recs[idx].b, s);
+}
+static void prof_bytes(Workspace *ws, int idx, double bytes) {
+    if (idx >= 0) ws->prof.recs[idx].bytes = bytes;
+}
+// after the stream is synchronised: fold the records into the per-class totals
+static void prof_flush(Workspace *ws) {
+    Prof &P = ws->prof;
+    for (const ProfRec &r : P.recs) {
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, r.a, r.b) == cudaSuccess) {
+            P.ms[r.cls] += ms;
+            P.bytes[r.cls] += r.bytes;
+            P.launches[r.cls] += 1;
+        }
+    }
+    cudaGetLastError();
+    P.recs.clear();
+    P.used = 0;
 }
 
 static cudaStream_t stream_of(const sg_opts *o) { return o ? (cudaStream_t)o->stream : (cudaStream_t)0; }
@@ -505,12 +581,14 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
     TRY(clear_frontier(in, s));
     TRY(clear_frontier(out, s));
-    CK(cudaMemsetAsync(ws->visited, 0, sizeof(uint64_t) * (size_t)G.nw1, s));
-    launch_seed(in->bits, in->summ, ws->visited, src, s);      // in = {src}, visited = {src}
+    // visited starts as the isolated vertices (unreachable: level stays INF) plus src
+    CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, s));
+    launch_seed(in->bits, in->summ, ws->visited, src, s);      // in = {src}, visited |= {src}
     const bool auto_dir = o.direction == SG_DIR_AUTO;
+    static const bool trace = getenv("SG_TRACE") != nullptr;
     TRY(compact(g, in, true, s));
     TRY(read_stats(ws, s));
-    int64_t mu = G.nnz;
+    int64_t mu = G.nnz, nf_prev = 0;
     bool pull = o.direction == SG_DIR_PULL;
     int64_t iters = 0, push_steps = 0, pull_steps = 0, arcs_pushed = 0, arcs_pulled = 0;
     int64_t reached = 1;
@@ -524,10 +602,14 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         const int64_t nf = (int64_t)hs.nf, mf = (int64_t)hs.mf;
         if (iters > 0) reached += nf;
         mu -= mf;
-        if (auto_dir) {
-            if (!pull && (double)mf > (double)mu / o.alpha) pull = true;
-            else if (pull && (double)nf < (double)G.n / o.beta) pull = false;
+        if (auto_dir) {   // Beamer: push -> pull on a growing frontier with m_f > m_u / alpha,
+                          // pull -> push on a shrinking frontier with n_f < n / beta
+            if (!pull && nf > nf_prev && (double)mf > (double)mu / o.alpha) pull = true;
+            else if (pull && nf < nf_prev && (double)nf < (double)G.n / o.beta) pull = false;
         }
+        nf_prev = nf;
+        const int64_t reached_before = reached;
+        const int pr = prof_begin(ws, pull ? SG_K_PULL : SG_K_PUSH, s);
         if (pull) {
             launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, level, d + 1, in->st, s);
             pull_steps++;
@@ -535,12 +617,36 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
             const PushLaunch L = push_launch(g, in, t, count);
             launch_push_bfs(L, BfsArgs{ws->visited, level, d + 1, out->bits, out->summ}, s);
             push_steps++;
-            arcs_pushed += mf;
         }
+        prof_end(ws, pr, s);
         TRY(clear_frontier(in, s));
+        const int pc = prof_begin(ws, SG_K_COMPACT, s);
         TRY(compact(g, out, true, s));
+        prof_end(ws, pc, s);
         TRY(read_stats(ws, s));
+        {
+            // algorithmic bytes of this step: col_idx 4 B/arc, row_ptr 16 B per
+            // expanded vertex, 8 B per input word, level 4 B + 8 B output word per new vertex/word
+            const DevStats &ho = ws->h_st[in_idx ^ 1];
+            const double n_new = (double)ho.nf, c_out = (double)ho.count;
+            double bytes;
+            if (pull) {
+                const double unvisited = (double)(G.n - reached_before);
+                bytes = 4.0 * (double)ws->h_st[in_idx].arcs + 16.0 * unvisited + 8.0 * (double)G.nw1 +
+                        4.0 * n_new + 16.0 * c_out;
+            } else {
+                bytes = 4.0 * (double)ws->h_st[in_idx].arcs + 16.0 * (double)nf + 8.0 * (double)count + 4.0 * n_new +
+                        8.0 * c_out;
+            }
+            prof_bytes(ws, pr, bytes);
+            prof_bytes(ws, pc, 8.0 * (double)G.nw2 + 12.0 * c_out + 16.0 * n_new);
+        }
         if (pull) arcs_pulled += (int64_t)ws->h_st[in_idx].arcs;
+        else arcs_pushed += (int64_t)ws->h_st[in_idx].arcs;
+        if (trace)
+            fprintf(stderr, "[sygraph bfs] level %u %s in: words %lld n_f %lld m_f~%lld | arcs %llu | out: n_f %llu\n", d,
+                    pull ? "pull" : "push", (long long)count, (long long)nf, (long long)mf,
+                    (unsigned long long)ws->h_st[in_idx].arcs, (unsigned long long)ws->h_st[in_idx ^ 1].nf);
         std::swap(in, out);
         in_idx ^= 1;
         d++;
@@ -551,6 +657,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
     CK(cudaGetLastError());
+    prof_flush(ws);
     if (stats) {
         stats->iterations = iters;
         stats->push_steps = push_steps;
@@ -769,5 +876,33 @@ SG_API int run_bc(const sg_graph *gc, const int32_t *sources, int32_t k, double 
     }
     return SG_OK;
 }
+
+// ---- measurement ---------------------------------------------------------------------------
+SG_API int sg_profile(sg_graph *g, int enable) {
+    if (!g) return fail(SG_ERR_INVALID, "NULL graph");
+    TRY(ensure_ws(g));
+    Prof &P = g->ws->prof;
+    P.on = enable != 0;
+    P.recs.clear();
+    P.used = 0;
+    for (int i = 0; i < SG_K_COUNT; i++) {
+        P.ms[i] = 0;
+        P.bytes[i] = 0;
+        P.launches[i] = 0;
+    }
+    return SG_OK;
+}
+
+SG_API int sg_profile_read(const sg_graph *g, sg_kprof *out) {
+    if (!g || !out) return fail(SG_ERR_INVALID, "NULL argument");
+    for (int i = 0; i < SG_K_COUNT; i++) {
+        out[i].ms = g->ws ? g->ws->prof.ms[i] : 0.0;
+        out[i].bytes = g->ws ? g->ws->prof.bytes[i] : 0.0;
+        out[i].launches = g->ws ? g->ws->prof.launches[i] : 0;
+    }
+    return SG_OK;
+}
+
+SG_API int64_t sg_launch_count(void) { return (int64_t)g_launches.load(); }
 
 }  // extern "C"

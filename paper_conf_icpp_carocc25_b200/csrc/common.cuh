@@ -16,6 +16,7 @@ struct GraphView {
     const int64_t *__restrict__ rp;    // row_ptr[n+1]
     const int32_t *__restrict__ col;   // col_idx[nnz] (+16 B zero padding for 16-B bulk copies)
     const uint8_t *__restrict__ w;     // weights[nnz] or nullptr
+    const uint8_t *__restrict__ deg8;  // 8-bit log-coded degrees, nw1*64 bytes (direction policy only)
     int64_t n, nnz;
     int64_t nw1, nw2;
 };

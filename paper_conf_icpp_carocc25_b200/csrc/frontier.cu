@@ -61,63 +61,90 @@ __global__ void k_rebuild_summary(const uint64_t *bits, uint64_t *summ, int64_t 
 }
 
 // ---------------------------------------------------------------------------------------
-// Summary compaction: one thread per summary word, block-wide exclusive scan of the
-// popcounts, one atomicAdd per block to reserve output space; each thread then writes its
-// word indices in ascending order (ascending within a block, arbitrary across blocks:
-// reading C4).  st->count receives the number of non-zero layer-1 words.
-constexpr int COMPACT_THREADS = 512;
+// Summary compaction: one warp per summary word (lane l owns bits l and l+32), a
+// block-wide exclusive scan of the 32 warps' popcounts and one atomicAdd per block to reserve
+// output space.  Offsets come out ascending within a block, blocks in arbitrary order
+// (reading C4).  st->count receives the number of non-zero layer-1 words.
+constexpr int COMPACT_THREADS = 1024;
+constexpr int COMPACT_WARPS = COMPACT_THREADS / 32;
 __global__ void __launch_bounds__(COMPACT_THREADS)
 k_compact(const uint64_t *__restrict__ summ, int64_t nw2, uint32_t *__restrict__ offsets, DevStats *st) {
-    __shared__ uint32_t s_warp[COMPACT_THREADS / 32];
+    __shared__ uint32_t s_cnt[COMPACT_WARPS];
     __shared__ uint32_t s_base;
-    const int64_t stride = (int64_t)gridDim.x * COMPACT_THREADS;
-    for (int64_t s0 = blockIdx.x * (int64_t)COMPACT_THREADS; s0 < nw2; s0 += stride) {
-        const int64_t s = s0 + threadIdx.x;
+    const int wid = threadIdx.x >> 5, lane = lane_id();
+    for (int64_t s0 = blockIdx.x * (int64_t)COMPACT_WARPS; s0 < nw2; s0 += (int64_t)gridDim.x * COMPACT_WARPS) {
+        const int64_t s = s0 + wid;
         const uint64_t x = s < nw2 ? summ[s] : 0ull;
-        const uint32_t c = __popcll(x);
-        const uint32_t incl = warp_inclusive_scan(c);
-        const int wid = threadIdx.x >> 5;
-        if (lane_id() == 31) s_warp[wid] = incl;
+        if (lane == 0) s_cnt[wid] = __popcll(x);
         __syncthreads();
         if (wid == 0) {
-            uint32_t t = lane_id() < COMPACT_THREADS / 32 ? s_warp[lane_id()] : 0u;
+            const uint32_t t = s_cnt[lane];
             const uint32_t ti = warp_inclusive_scan(t);
-            if (lane_id() < COMPACT_THREADS / 32) s_warp[lane_id()] = ti - t;
-            if (lane_id() == 31) s_base = ti ? (uint32_t)atomicAdd(&st->count, (unsigned long long)ti) : 0u;
+            s_cnt[lane] = ti - t;
+            if (lane == 31) s_base = ti ? (uint32_t)atomicAdd(&st->count, (unsigned long long)ti) : 0u;
         }
         __syncthreads();
-        uint32_t pos = s_base + s_warp[wid] + (incl - c);
-        uint64_t y = x;
-        while (y) {
-            const int b = __ffsll((long long)y) - 1;
-            offsets[pos++] = (uint32_t)(s * 64 + b);
-            y &= y - 1;
-        }
+        const uint32_t base = s_base + s_cnt[wid];
+        if ((x >> lane) & 1ull) offsets[base + __popcll(x & ((1ull << lane) - 1ull))] = (uint32_t)(s * 64 + lane);
+        if ((x >> (lane + 32)) & 1ull)
+            offsets[base + __popcll(x & ((1ull << (lane + 32)) - 1ull))] = (uint32_t)(s * 64 + lane + 32);
         __syncthreads();
     }
 }
 
 // ---------------------------------------------------------------------------------------
-// n_f and m_f of a compacted frontier (Beamer's direction policy inputs): warp per word.
-__global__ void __launch_bounds__(256) k_frontier_stats(GraphView g, const uint64_t *__restrict__ bits,
-                                                        const uint32_t *__restrict__ offsets, DevStats *st) {
-    const uint32_t count = (uint32_t)st->count;
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+// Direction-policy inputs n_f (popcount) and m_f (sum of frontier degrees).  m_f only steers
+// the Beamer heuristic, so it is read from the graph's 8-bit log-coded degree array (16 MB for
+// 2^24 vertices, L2 resident; <= 1/16 relative error per vertex) instead of row_ptr (134 MB).
+// One thread per layer-1 word, no offsets indirection: bits + 64 code bytes per non-zero word.
+__device__ __forceinline__ uint32_t deg8_decode(uint32_t c) {
+    if (c < 32u) return c;
+    const uint32_t e = ((c - 32u) >> 3) + 5u, m = (c - 32u) & 7u;
+    return ((8u + m) << (e - 3u)) + (1u << (e - 4u));
+}
+
+__global__ void __launch_bounds__(256) k_frontier_stats(const uint64_t *__restrict__ bits, int64_t nw1,
+                                                        const uint8_t *__restrict__ deg8, DevStats *st) {
     unsigned long long nf = 0, mf = 0;
-    for (int64_t i = gw; i < count; i += nwarps) {
-        const int64_t w = offsets[i];
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nw1; w += stride) {
         const uint64_t x = bits[w];
-        int64_t sa, ea, sb, eb;
-        word_bounds(g, w, x, sa, ea, sb, eb);
-        mf += (unsigned long long)((ea - sa) + (eb - sb));
-        if (lane_id() == 0) nf += __popcll(x);
+        if (!x) continue;
+        nf += __popcll(x);
+        const uint64_t *q = reinterpret_cast<const uint64_t *>(deg8 + w * 64);
+        uint64_t c[8];
+#pragma unroll
+        for (int k = 0; k < 8; k++) c[k] = ((x >> (8 * k)) & 0xffull) ? __ldg(q + k) : 0ull;
+#pragma unroll
+        for (int k = 0; k < 8; k++) {
+            uint32_t bm = (uint32_t)((x >> (8 * k)) & 0xffull);
+            while (bm) {
+                const int j = __ffs(bm) - 1;
+                bm &= bm - 1;
+                mf += deg8_decode((uint32_t)((c[k] >> (8 * j)) & 0xffull));
+            }
+        }
     }
+    // block reduction first: one pair of atomics per CTA (a per-warp atomic on one address
+    // serialises ~10^4 operations in L2 on a dense frontier)
+    __shared__ unsigned long long s_mf[8], s_nf[8];
     mf = warp_sum(mf);
     nf = warp_sum(nf);
-    if (lane_id() == 0 && (mf | nf)) {
-        atomicAdd(&st->mf, mf);
-        atomicAdd(&st->nf, nf);
+    if (lane_id() == 0) {
+        s_mf[threadIdx.x >> 5] = mf;
+        s_nf[threadIdx.x >> 5] = nf;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long a = 0, b = 0;
+        for (int i = 0; i < (int)(blockDim.x >> 5); i++) {
+            a += s_mf[i];
+            b += s_nf[i];
+        }
+        if (a | b) {
+            atomicAdd(&st->mf, a);
+            atomicAdd(&st->nf, b);
+        }
     }
 }
 
@@ -180,7 +207,25 @@ __global__ void k_max_u8(const uint8_t *w, int64_t nnz, unsigned int *out) {
 __global__ void k_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src) {
     bits[src >> 6] = 1ull << (src & 63);
     summ[src >> 12] = 1ull << ((src >> 6) & 63);
-    if (visited) visited[src >> 6] = 1ull << (src & 63);
+    if (visited) visited[src >> 6] |= 1ull << (src & 63);
+}
+
+// bit v set iff deg(v) == 0: isolated vertices can never be reached, so BFS starts with them
+// marked visited and the pull step never scans them (1/3 of a Kronecker graph's ids).
+__global__ void k_isolated(const uint8_t *__restrict__ deg8, int64_t n, int64_t nw1, uint64_t *__restrict__ iso) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nw1; w += stride) {
+        const uint64_t *q = reinterpret_cast<const uint64_t *>(deg8 + w * 64);
+        uint64_t m = 0;
+        for (int k = 0; k < 8; k++) {
+            const uint64_t c = q[k];
+            for (int j = 0; j < 8; j++)
+                if (((c >> (8 * j)) & 0xffull) == 0ull) m |= 1ull << (8 * k + j);
+        }
+        const int64_t rem = n - w * 64;
+        if (rem < 64) m &= (1ull << rem) - 1ull;
+        iso[w] = m;
+    }
 }
 
 template <typename T>
@@ -196,47 +241,83 @@ static int grid_for(int64_t items, int threads, int max_blocks) {
 }
 
 void launch_fill_all(uint64_t *bits, uint64_t *summ, int64_t n, int64_t nw1, int64_t nw2, cudaStream_t s) {
+    note_launch();
     k_fill_all<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(bits, summ, n, nw1, nw2);
 }
 void launch_insert(uint64_t *bits, uint64_t *summ, const int32_t *v, int64_t k, int64_t n, cudaStream_t s) {
-    if (k > 0) k_insert<<<grid_for(k, 256, 148 * 8), 256, 0, s>>>(bits, summ, v, k, n);
+    if (k > 0) { note_launch(); k_insert<<<grid_for(k, 256, 148 * 8), 256, 0, s>>>(bits, summ, v, k, n); }
 }
 void launch_setop(uint64_t *dst, const uint64_t *src, int64_t nw1, int op, cudaStream_t s) {
+    note_launch();
     k_setop<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(dst, src, nw1, op);
 }
 void launch_rebuild_summary(const uint64_t *bits, uint64_t *summ, int64_t nw1, int64_t nw2, cudaStream_t s) {
+    note_launch();
     k_rebuild_summary<<<grid_for(nw2 * 32, 256, 148 * 8), 256, 0, s>>>(bits, summ, nw1, nw2);
 }
 void launch_compact(const uint64_t *summ, int64_t nw2, uint32_t *offsets, DevStats *st, cudaStream_t s) {
-    k_compact<<<grid_for(nw2, COMPACT_THREADS, 148 * 2), COMPACT_THREADS, 0, s>>>(summ, nw2, offsets, st);
+    note_launch();
+    k_compact<<<grid_for(nw2, COMPACT_WARPS, 148 * 2), COMPACT_THREADS, 0, s>>>(summ, nw2, offsets, st);
 }
-void launch_frontier_stats(const GraphView &g, const uint64_t *bits, const uint32_t *offsets, DevStats *st,
-                           int64_t max_words, cudaStream_t s) {
-    k_frontier_stats<<<grid_for(max_words * 32, 256, 148 * 8), 256, 0, s>>>(g, bits, offsets, st);
+void launch_frontier_stats(const GraphView &g, const uint64_t *bits, DevStats *st, cudaStream_t s) {
+    note_launch();
+    k_frontier_stats<<<grid_for(g.nw1, 256, 148 * 8), 256, 0, s>>>(bits, g.nw1, g.deg8, st);
+}
+// 8-bit log code of each vertex degree (exact below 32, 3 mantissa bits above); padded to 64 B
+// per layer-1 word so k_frontier_stats can read whole words.
+__global__ void k_deg8(const int64_t *__restrict__ rp, int64_t n, int64_t npad, uint8_t *__restrict__ deg8) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < npad; v += stride) {
+        uint32_t c = 0;
+        if (v < n) {
+            const int64_t d = rp[v + 1] - rp[v];
+            if (d < 32) {
+                c = (uint32_t)d;
+            } else {
+                const uint32_t e = 63u - (uint32_t)__clzll((unsigned long long)d);
+                c = 32u + (e - 5u) * 8u + (uint32_t)((d >> (e - 3u)) & 7);
+                if (c > 255u) c = 255u;
+            }
+        }
+        deg8[v] = (uint8_t)c;
+    }
+}
+void launch_isolated(const uint8_t *deg8, int64_t n, int64_t nw1, uint64_t *iso, cudaStream_t s) {
+    note_launch();
+    k_isolated<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(deg8, n, nw1, iso);
+}
+void launch_deg8(const int64_t *rp, int64_t n, int64_t npad, uint8_t *deg8, cudaStream_t s) {
+    note_launch();
+    k_deg8<<<grid_for(npad, 256, 148 * 8), 256, 0, s>>>(rp, n, npad, deg8);
 }
 void launch_popcount(const uint64_t *bits, int64_t nw1, unsigned long long *out, cudaStream_t s) {
+    note_launch();
     k_popcount<<<grid_for(nw1, 256, 148 * 4), 256, 0, s>>>(bits, nw1, out);
 }
 void launch_or_listed(const uint64_t *bits, const uint32_t *offsets, const DevStats *st, uint64_t *dst,
                       int64_t max_words, cudaStream_t s) {
+    note_launch();
     k_or_listed<<<grid_for(max_words, 256, 148 * 8), 256, 0, s>>>(bits, offsets, st, dst);
 }
 void launch_or_all(const uint64_t *bits, int64_t nw1, uint64_t *dst, cudaStream_t s) {
+    note_launch();
     k_or_all<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(bits, nw1, dst);
 }
-void launch_set_u32(uint32_t *p, int64_t i, uint32_t v, cudaStream_t s) { k_set_one<uint32_t><<<1, 1, 0, s>>>(p, i, v); }
-void launch_set_i32(int32_t *p, int64_t i, int32_t v, cudaStream_t s) { k_set_one<int32_t><<<1, 1, 0, s>>>(p, i, v); }
-void launch_set_f64(double *p, int64_t i, double v, cudaStream_t s) { k_set_one<double><<<1, 1, 0, s>>>(p, i, v); }
+void launch_set_u32(uint32_t *p, int64_t i, uint32_t v, cudaStream_t s) { note_launch(); k_set_one<uint32_t><<<1, 1, 0, s>>>(p, i, v); }
+void launch_set_i32(int32_t *p, int64_t i, int32_t v, cudaStream_t s) { note_launch(); k_set_one<int32_t><<<1, 1, 0, s>>>(p, i, v); }
+void launch_set_f64(double *p, int64_t i, double v, cudaStream_t s) { note_launch(); k_set_one<double><<<1, 1, 0, s>>>(p, i, v); }
 
 void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, cudaStream_t s) {
+    note_launch();
     k_seed<<<1, 1, 0, s>>>(bits, summ, visited, src);
 }
-void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { k_iota_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(p, n); }
+void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(p, n); }
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s) {
+    note_launch();
     k_validate_csr<<<grid_for(g.nnz > g.n ? g.nnz : g.n, 256, 148 * 8), 256, 0, s>>>(g, bad);
 }
 void launch_max_weight(const uint8_t *w, int64_t nnz, unsigned int *out, cudaStream_t s) {
-    if (nnz > 0) k_max_u8<<<grid_for(nnz, 256, 148 * 8), 256, 0, s>>>(w, nnz, out);
+    if (nnz > 0) { note_launch(); k_max_u8<<<grid_for(nnz, 256, 148 * 8), 256, 0, s>>>(w, nnz, out); }
 }
 
 }  // namespace sg

@@ -8,14 +8,18 @@ namespace sg {
 
 struct PushParams;
 
+// host-side count of kernel launches issued by the library (bench evidence: gpu_launches)
+void note_launch();
+
 // frontier.cu
 void launch_fill_all(uint64_t *bits, uint64_t *summ, int64_t n, int64_t nw1, int64_t nw2, cudaStream_t s);
 void launch_insert(uint64_t *bits, uint64_t *summ, const int32_t *v, int64_t k, int64_t n, cudaStream_t s);
 void launch_setop(uint64_t *dst, const uint64_t *src, int64_t nw1, int op, cudaStream_t s);
 void launch_rebuild_summary(const uint64_t *bits, uint64_t *summ, int64_t nw1, int64_t nw2, cudaStream_t s);
 void launch_compact(const uint64_t *summ, int64_t nw2, uint32_t *offsets, DevStats *st, cudaStream_t s);
-void launch_frontier_stats(const GraphView &g, const uint64_t *bits, const uint32_t *offsets, DevStats *st,
-                           int64_t max_words, cudaStream_t s);
+void launch_frontier_stats(const GraphView &g, const uint64_t *bits, DevStats *st, cudaStream_t s);
+void launch_isolated(const uint8_t *deg8, int64_t n, int64_t nw1, uint64_t *iso, cudaStream_t s);
+void launch_deg8(const int64_t *rp, int64_t n, int64_t npad, uint8_t *deg8, cudaStream_t s);
 void launch_popcount(const uint64_t *bits, int64_t nw1, unsigned long long *out, cudaStream_t s);
 void launch_or_listed(const uint64_t *bits, const uint32_t *offsets, const DevStats *st, uint64_t *dst,
                       int64_t max_words, cudaStream_t s);

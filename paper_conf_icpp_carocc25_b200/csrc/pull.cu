@@ -3,8 +3,10 @@
 //
 // Every unvisited vertex v scans N(v) (symmetric CSR = its in-neighbours, reading C8) and
 // stops at the first u that is in the input frontier (one bit test on the 2LB layer 1).
-// One warp owns one 64-bit word of the visited bitmap, so the new frontier word, the visited
-// word and level[] are written without atomics; only the summary bit is an atomicOr.
+// One warp owns one 64-bit word of the visited bitmap (lane l: vertices 64w+l and 64w+32+l),
+// so the new frontier word, the visited word and level[] are written without atomics; only
+// the summary bit is an atomicOr.  The two vertices of a lane are scanned in lock-step (two
+// independent load chains in flight per lane): the step is latency-bound, not bandwidth-bound.
 // Output identical to a push step from the same state (tested).
 #include "common.cuh"
 #include "kernels.h"
@@ -12,33 +14,15 @@
 namespace sg {
 
 constexpr int PULL_THREADS = 256;
+#ifndef SG_PULL_ARCS
+#define SG_PULL_ARCS 2
+#endif
+#ifndef SG_PULL_MINB
+#define SG_PULL_MINB 6
+#endif
+constexpr int PULL_ARCS = SG_PULL_ARCS;   // arcs per vertex per iteration
 
-// scan N(u) = col[s..e) four arcs at a time (4 independent loads + 4 bit probes in flight)
-__device__ __forceinline__ bool pull_scan(const GraphView &g, const uint64_t *__restrict__ in_bits, int64_t s,
-                                          int64_t e, unsigned long long &arcs) {
-    for (int64_t i = s; i < e; i += 4) {
-        int32_t c[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) c[k] = (i + k < e) ? __ldg(g.col + i + k) : -1;
-        uint64_t x[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) x[k] = c[k] >= 0 ? __ldg(in_bits + (c[k] >> 6)) : 0ull;
-        bool hit = false;
-        int used = 0;
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            if (!hit && c[k] >= 0) {
-                used++;
-                hit = (x[k] >> (c[k] & 63)) & 1ull;
-            }
-        }
-        arcs += used;
-        if (hit) return true;
-    }
-    return false;
-}
-
-__global__ void __launch_bounds__(PULL_THREADS)
+__global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited,
            uint64_t *__restrict__ out_bits, uint64_t *__restrict__ out_summ, uint32_t *__restrict__ level,
            uint32_t next, DevStats *st) {
@@ -53,14 +37,46 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
         const uint64_t valid = rem >= 64 ? ~0ull : ((1ull << rem) - 1ull);
         const uint64_t unv = ~vis & valid;
         if (!unv) continue;
-        int64_t sa, ea, sb, eb;
-        word_bounds(g, w, unv, sa, ea, sb, eb);
-        const bool fa = (ea > sa) && pull_scan(g, in_bits, sa, ea, arcs);
-        const bool fb = (eb > sb) && pull_scan(g, in_bits, sb, eb, arcs);
-        const uint32_t ba = __ballot_sync(0xffffffffu, fa), bb = __ballot_sync(0xffffffffu, fb);
+        int64_t s[2], e[2];
+        word_bounds(g, w, unv, s[0], e[0], s[1], e[1]);
+        bool found[2] = {false, false};
+        // lock-step scan of both vertices' lists until each hits a frontier neighbour
+        while (s[0] < e[0] || s[1] < e[1]) {
+            int32_t c[2][PULL_ARCS];
+#pragma unroll
+            for (int k = 0; k < 2; k++)
+#pragma unroll
+                for (int j = 0; j < PULL_ARCS; j++) c[k][j] = (s[k] + j < e[k]) ? __ldg(g.col + s[k] + j) : -1;
+            uint64_t x[2][PULL_ARCS];
+#pragma unroll
+            for (int k = 0; k < 2; k++)
+#pragma unroll
+                for (int j = 0; j < PULL_ARCS; j++) x[k][j] = c[k][j] >= 0 ? __ldg(in_bits + (c[k][j] >> 6)) : 0ull;
+#pragma unroll
+            for (int k = 0; k < 2; k++) {
+                if (s[k] >= e[k]) continue;
+                int used = 0;
+                bool hit = false;
+#pragma unroll
+                for (int j = 0; j < PULL_ARCS; j++) {
+                    if (!hit && c[k][j] >= 0) {
+                        used++;
+                        hit = (x[k][j] >> (c[k][j] & 63)) & 1ull;
+                    }
+                }
+                arcs += used;
+                if (hit) {
+                    found[k] = true;
+                    s[k] = e[k];
+                } else {
+                    s[k] += PULL_ARCS;
+                }
+            }
+        }
+        const uint32_t ba = __ballot_sync(0xffffffffu, found[0]), bb = __ballot_sync(0xffffffffu, found[1]);
         const uint64_t nb = (uint64_t)ba | ((uint64_t)bb << 32);
-        if (fa) level[w * 64 + lane] = next;
-        if (fb) level[w * 64 + 32 + lane] = next;
+        if (found[0]) level[w * 64 + lane] = next;
+        if (found[1]) level[w * 64 + 32 + lane] = next;
         if (nb && lane == 0) {
             out_bits[w] = nb;
             visited[w] = vis | nb;
@@ -80,8 +96,9 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
                      uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s) {
     int64_t blocks = (g.nw1 * 32 + PULL_THREADS - 1) / PULL_THREADS;
-    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks > 148 * SG_PULL_MINB) blocks = 148 * SG_PULL_MINB;
     if (blocks < 1) blocks = 1;
+    note_launch();
     k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, out_bits, out_summ, level, next, st);
 }
 

@@ -27,11 +27,13 @@ static void launch_push(const PushLaunch &L, const F &f, cudaStream_t s) {
         attr_done = true;
     }
     const PushParams p = make_params(L);
+    note_launch();
     k_push_words<F><<<L.grid_words, PUSH_THREADS, 0, s>>>(p, f);
+    note_launch();
     k_push_heavy<F><<<L.grid_heavy, HEAVY_THREADS, HEAVY_SMEM, s>>>(p, f);
 }
 
-int push_max_grid_words() { return 148 * 6; }
+int push_max_grid_words() { return 148 * 4; }   // 64 regs x 256 threads: 4 CTAs per SM resident
 int push_max_grid_heavy() { return 148 * 3; }
 
 void launch_push_bfs(const PushLaunch &L, const BfsArgs &a, cudaStream_t s) {

@@ -209,19 +209,19 @@ __device__ __forceinline__ unsigned long long push_word(const PushParams &p, con
 template <class F>
 __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) {
     __shared__ PushWarpSmem<F> s_warp[PUSH_WARPS];
-    __shared__ uint32_t s_batch;
     __shared__ unsigned long long s_arcs[PUSH_WARPS];
     const uint32_t count = (uint32_t)p.st->count;
     const int wid = threadIdx.x >> 5;
     unsigned long long arcs = 0;
+    // each warp grabs `batch` words (the coarsening factor) with one atomic; no CTA barrier in
+    // the loop, so a warp never waits for a slower sibling's batch
     for (;;) {
-        if (threadIdx.x == 0) s_batch = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)p.batch);
-        __syncthreads();
-        const uint32_t b0 = s_batch;
-        __syncthreads();
+        uint32_t b0 = 0;
+        if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)p.batch);
+        b0 = __shfl_sync(0xffffffffu, b0, 0);
         if (b0 >= count) break;
         const uint32_t b1 = min(b0 + (uint32_t)p.batch, count);
-        for (uint32_t i = b0 + wid; i < b1; i += PUSH_WARPS) arcs += push_word(p, f, p.offsets[i], s_warp[wid]);
+        for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid]);
     }
     arcs = warp_sum(arcs);
     if (lane_id() == 0) s_arcs[wid] = arcs;
