@@ -73,7 +73,9 @@ typedef struct {
     int64_t max_iters;        /* superstep cap (0 = n + 1); exceeding it returns SG_ERR_STATE */
     int32_t heavy_degree;     /* push tiers: degree > heavy_degree goes to the CTA/grid tier (0 = default) */
     int32_t small_degree;     /* degree <= small_degree uses the thread-granular packed tier (0 = default, <0 = none) */
-    int32_t reserved[8];
+    int32_t host_loop;        /* run_bfs: 1 = host-driven superstep loop (one control read per level);
+                                 0 = one CUDA graph with device-side control (default) */
+    int32_t reserved[7];
 } sg_opts;
 
 typedef struct {

@@ -93,6 +93,13 @@ struct Workspace {
     double *sigma = nullptr;
     uint32_t *level = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    // CUDA-graph driven BFS (ctrl.cu): instantiated once per (level buffer, tiers)
+    BfsCtrl *ctrl = nullptr, *h_ctrl = nullptr;
+    cudaGraph_t bfs_graph = nullptr;
+    cudaGraphExec_t bfs_exec = nullptr;
+    uint32_t *bfs_level = nullptr;
+    int32_t bfs_heavy = 0, bfs_small = 0;
+    cudaStream_t cap_stream = nullptr;
 };
 
 struct sg_graph {
@@ -181,6 +188,11 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->delta);
     cudaFree(ws->sigma);
     cudaFree(ws->level);
+    if (ws->bfs_exec) cudaGraphExecDestroy(ws->bfs_exec);
+    if (ws->bfs_graph) cudaGraphDestroy(ws->bfs_graph);
+    if (ws->cap_stream) cudaStreamDestroy(ws->cap_stream);
+    cudaFree(ws->ctrl);
+    cudaFreeHost(ws->h_ctrl);
     if (ws->ev0) cudaEventDestroy(ws->ev0);
     if (ws->ev1) cudaEventDestroy(ws->ev1);
     for (cudaEvent_t e : ws->prof.pool) cudaEventDestroy(e);
@@ -558,6 +570,157 @@ SG_API int advance(const sg_graph *gc, const sg_frontier *in, sg_frontier *out, 
     return SG_OK;
 }
 
+}  // extern "C"
+
+// ---- CUDA-graph driven BFS (no host round trip per superstep; ctrl.cu) -------------------
+static int capture_begin(cudaStream_t cs, cudaGraph_t graph, const std::vector<cudaGraphNode_t> &deps) {
+    CK(cudaStreamBeginCaptureToGraph(cs, graph, deps.empty() ? nullptr : deps.data(), nullptr, deps.size(),
+                                     cudaStreamCaptureModeRelaxed));
+    return SG_OK;
+}
+static int capture_end(cudaStream_t cs, std::vector<cudaGraphNode_t> &leaves) {
+    cudaStreamCaptureStatus cst;
+    const cudaGraphNode_t *d = nullptr;
+    size_t nd = 0;
+    CK(cudaStreamGetCaptureInfo(cs, &cst, nullptr, nullptr, &d, &nd));
+    leaves.assign(d, d + nd);
+    cudaGraph_t gout;
+    CK(cudaStreamEndCapture(cs, &gout));
+    return SG_OK;
+}
+// add a conditional node (IF / WHILE) after `deps`; returns its body graph
+static int add_cond(cudaGraph_t graph, const std::vector<cudaGraphNode_t> &deps, cudaGraphConditionalHandle h,
+                    cudaGraphConditionalNodeType type, cudaGraphNode_t *node, cudaGraph_t *body) {
+    cudaGraphNodeParams p = {};
+    p.type = cudaGraphNodeTypeConditional;
+    p.conditional.handle = h;
+    p.conditional.type = type;
+    p.conditional.size = 1;
+    CK(cudaGraphAddNode(node, graph, deps.empty() ? nullptr : deps.data(), deps.size(), &p));
+    *body = p.conditional.phGraph_out[0];
+    return SG_OK;
+}
+
+static int build_bfs_graph(sg_graph *g, uint32_t *level, Tiers t) {
+    Workspace *ws = g->ws;
+    const GraphView &G = g->v;
+    if (ws->bfs_exec) cudaGraphExecDestroy(ws->bfs_exec);
+    if (ws->bfs_graph) cudaGraphDestroy(ws->bfs_graph);
+    ws->bfs_exec = nullptr;
+    ws->bfs_graph = nullptr;
+    if (!ws->cap_stream) CK(cudaStreamCreateWithFlags(&ws->cap_stream, cudaStreamNonBlocking));
+    if (!ws->ctrl) {
+        CK(cudaMalloc(&ws->ctrl, sizeof(BfsCtrl)));
+        CK(cudaMallocHost(&ws->h_ctrl, sizeof(BfsCtrl)));
+    }
+    cudaStream_t cs = ws->cap_stream;
+    cudaGraph_t root;
+    CK(cudaGraphCreate(&root, 0));
+    ws->bfs_graph = root;
+    cudaGraphConditionalHandle h_loop, h_push[2], h_pull[2];
+    CK(cudaGraphConditionalHandleCreate(&h_loop, root, 0, cudaGraphCondAssignDefault));
+    for (int i = 0; i < 2; i++) {
+        CK(cudaGraphConditionalHandleCreate(&h_push[i], root, 0, cudaGraphCondAssignDefault));
+        CK(cudaGraphConditionalHandleCreate(&h_pull[i], root, 0, cudaGraphCondAssignDefault));
+    }
+    sg_frontier *F[2] = {&ws->fr[0], &ws->fr[1]};
+    std::vector<cudaGraphNode_t> leaves;
+    // prologue: level = INF, frontiers cleared, visited = isolated, seed src, compact + decide
+    TRY(capture_begin(cs, root, {}));
+    CK(cudaMemsetAsync(level, 0xFF, sizeof(uint32_t) * (size_t)G.n, cs));
+    for (int i = 0; i < 2; i++) {
+        CK(cudaMemsetAsync(F[i]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
+        CK(cudaMemsetAsync(F[i]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
+    }
+    CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), cs));
+    CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
+    launch_bfs_seed(ws->ctrl, level, F[0]->bits, F[0]->summ, ws->visited, cs);
+    launch_compact(F[0]->summ, G.nw2, F[0]->offsets, F[0]->st, cs);
+    launch_frontier_stats(G, F[0]->bits, F[0]->st, cs);
+    launch_bfs_decide(ws->ctrl, F[0]->st, nullptr, h_loop, h_push[0], h_pull[0], 1, cs);
+    TRY(capture_end(cs, leaves));
+    cudaGraphNode_t wnode;
+    cudaGraph_t body;
+    TRY(add_cond(root, leaves, h_loop, cudaGraphCondTypeWhile, &wnode, &body));
+    // body: superstep A->B then B->A
+    std::vector<cudaGraphNode_t> deps;
+    for (int half = 0; half < 2; half++) {
+        sg_frontier *in = F[half], *out = F[half ^ 1];
+        cudaGraphNode_t n_push, n_pull;
+        cudaGraph_t b_push, b_pull;
+        TRY(add_cond(body, deps, h_push[half], cudaGraphCondTypeIf, &n_push, &b_push));
+        TRY(add_cond(body, deps, h_pull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
+        PushLaunch L = push_launch(g, in, t, -1);
+        L.batch = 0;   // coarsening factor computed on the device from the count
+        BfsArgs a{ws->visited, level, 0u, out->bits, out->summ, &ws->ctrl->next};
+        TRY(capture_begin(cs, b_push, {}));
+        launch_push_bfs(L, a, cs);
+        TRY(capture_end(cs, leaves));
+        TRY(capture_begin(cs, b_pull, {}));
+        launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, level, 0u, in->st, cs, &ws->ctrl->next);
+        TRY(capture_end(cs, leaves));
+        TRY(capture_begin(cs, body, {n_push, n_pull}));
+        launch_clear_listed(in->bits, in->summ, in->offsets, in->st, G.nw1, G.nw2, out->st, cs);
+        launch_compact(out->summ, G.nw2, out->offsets, out->st, cs);
+        launch_frontier_stats(G, out->bits, out->st, cs);
+        launch_bfs_decide(ws->ctrl, out->st, in->st, h_loop, h_push[half ^ 1], h_pull[half ^ 1], 0, cs);
+        TRY(capture_end(cs, deps));
+    }
+    CK(cudaGraphInstantiate(&ws->bfs_exec, root, 0));
+    ws->bfs_level = level;
+    ws->bfs_heavy = t.heavy;
+    ws->bfs_small = t.small;
+    return SG_OK;
+}
+
+static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opts &o, Tiers t, int64_t max_iters,
+                         sg_stats *stats) {
+    Workspace *ws = g->ws;
+    cudaStream_t s = stream_of(&o);
+    if (!ws->bfs_exec || ws->bfs_level != level || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small)
+        TRY(build_bfs_graph(g, level, t));
+    BfsCtrl &c = *ws->h_ctrl;
+    memset(&c, 0, sizeof c);
+    c.mu = g->v.nnz;
+    c.n = g->v.n;
+    c.max_iters = max_iters;
+    c.alpha = o.alpha;
+    c.beta = o.beta;
+    c.src = src;
+    c.pull = o.direction == SG_DIR_PULL;
+    c.auto_dir = o.direction == SG_DIR_AUTO;
+    c.reached = 1;
+    CK(cudaEventRecord(ws->ev0, s));
+    CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, sizeof(BfsCtrl), cudaMemcpyHostToDevice, s));
+    CK(cudaGraphLaunch(ws->bfs_exec, s));
+    CK(cudaMemcpyAsync(ws->h_ctrl, ws->ctrl, sizeof(BfsCtrl), cudaMemcpyDeviceToHost, s));
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
+    {
+        // kernels the graph executed: prologue (seed, compact, stats, decide) + per WHILE body
+        // (2 x clear, compact, stats, decide) + the taken IF bodies (push = 2 kernels, pull = 1)
+        const long long bodies = (long long)(c.iters + 1) / 2;
+        const long long k = 4 + 8 * bodies + 2 * (long long)c.push_steps + (long long)c.pull_steps;
+        for (long long i = 0; i < k; i++) note_launch();
+    }
+    if (stats) {
+        stats->iterations = (int64_t)c.iters;
+        stats->push_steps = (int64_t)c.push_steps;
+        stats->pull_steps = (int64_t)c.pull_steps;
+        stats->arcs_pushed = (int64_t)c.arcs_pushed;
+        stats->arcs_pulled = (int64_t)c.arcs_pulled;
+        stats->reached = (int64_t)c.reached;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
+extern "C" {
+
 // ---- BFS (Listing 1 + Beamer direction optimisation) --------------------------------------
 SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_opts *opts, sg_stats *stats) {
     t_err.clear();
@@ -575,6 +738,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
+    if (!ws->prof.on && !o.host_loop) return run_bfs_graph(g, src, level, o, t, max_iters, stats);
     CK(cudaEventRecord(ws->ev0, s));
     CK(cudaMemsetAsync(level, 0xFF, sizeof(uint32_t) * (size_t)G.n, s));
     launch_set_u32(level, src, 0u, s);

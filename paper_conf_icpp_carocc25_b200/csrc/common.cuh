@@ -33,6 +33,21 @@ struct DevStats {
     unsigned long long pad;
 };
 
+// Device-resident state of a graph-driven BFS (written by k_bfs_decide, read back once per run).
+struct BfsCtrl {
+    unsigned long long iters, push_steps, pull_steps, arcs_pushed, arcs_pulled, reached;
+    long long mu;            // sum of degrees of unvisited vertices (Beamer m_u, estimate)
+    long long nf_prev;
+    long long n, max_iters;
+    double alpha, beta;
+    int32_t src;
+    uint32_t next;           // level value written by the superstep being launched
+    uint32_t pull;           // direction of the superstep being launched
+    uint32_t auto_dir;
+    uint32_t overflow;       // iteration cap hit
+    uint32_t pad;
+};
+
 // One CTA/grid-tier work unit: a contiguous piece of one vertex's adjacency list.
 struct HeavyItem {
     int64_t begin;   // first arc index

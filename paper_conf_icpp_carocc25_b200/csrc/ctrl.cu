@@ -1,0 +1,106 @@
+// ctrl.cu — device-side superstep control for the CUDA-graph driven loops.
+//
+// Listing 1's host loop (P:172 `while (!in_frontier.empty())`, swap + clear at P:182-184) costs
+// one device->host round trip per superstep.  Here the whole BFS is one CUDA graph: a WHILE node
+// whose body runs two supersteps (A->B, B->A, so kernel arguments stay static), each superstep an
+// IF(push) / IF(pull) pair followed by clear + compaction + statistics + k_bfs_decide, which
+// applies the direction policy on the device and sets the conditional handles
+// (cudaGraphSetConditional).  Results are identical to the host loop (tested).
+#include "common.cuh"
+#include "kernels.h"
+
+namespace sg {
+
+__device__ __forceinline__ void set_cond(unsigned long long h, unsigned v) {
+    if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, v);
+}
+
+// Decide the next superstep from the freshly compacted frontier's control block `st`.
+// `prev` (nullable) is the control block of the frontier just advanced: its arcs counter is
+// folded into the per-direction totals.
+__global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
+                             unsigned long long h_push, unsigned long long h_pull, int first) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    if (prev) {
+        if (c->pull) c->arcs_pulled += prev->arcs;
+        else c->arcs_pushed += prev->arcs;
+    }
+    const unsigned long long count = st->count;
+    bool go = count > 0;
+    if (go && c->iters >= (unsigned long long)c->max_iters) {
+        c->overflow = 1;
+        go = false;
+    }
+    if (go) {
+        const long long nf = (long long)st->nf, mf = (long long)st->mf;
+        if (!first) c->reached += (unsigned long long)nf;
+        c->mu -= mf;
+        if (c->auto_dir) {   // Beamer (R2)
+            if (!c->pull && nf > c->nf_prev && (double)mf > (double)c->mu / c->alpha) c->pull = 1;
+            else if (c->pull && nf < c->nf_prev && (double)nf < (double)c->n / c->beta) c->pull = 0;
+        }
+        c->nf_prev = nf;
+        c->next = first ? 1u : c->next + 1u;
+        if (c->pull) c->pull_steps++;
+        else c->push_steps++;
+        c->iters++;
+    }
+    set_cond(h_push, go && !c->pull);
+    set_cond(h_pull, go && c->pull);
+    set_cond(h_loop, go);
+}
+
+// BFS prologue on the device: level[src] = 0, in = {src}, visited |= {src} (src from ctrl).
+__global__ void k_bfs_seed(const BfsCtrl *c, uint32_t *level, uint64_t *bits, uint64_t *summ, uint64_t *visited) {
+    const int32_t src = c->src;
+    level[src] = 0u;
+    bits[src >> 6] = 1ull << (src & 63);
+    summ[src >> 12] = 1ull << ((src >> 6) & 63);
+    visited[src >> 6] |= 1ull << (src & 63);
+}
+
+// Clear a frontier after it was advanced (only its listed non-zero words + its summary) and
+// zero the control block of the frontier about to be compacted.
+__global__ void k_clear_listed(uint64_t *__restrict__ bits, uint64_t *__restrict__ summ,
+                               const uint32_t *__restrict__ offsets, const DevStats *st, int64_t nw2,
+                               DevStats *zero_st) {
+    const uint32_t count = (uint32_t)st->count;
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = t; i < count; i += stride) bits[offsets[i]] = 0ull;
+    for (int64_t s = t; s < nw2; s += stride) summ[s] = 0ull;
+    if (zero_st && t < (int64_t)(sizeof(DevStats) / 8)) reinterpret_cast<unsigned long long *>(zero_st)[t] = 0ull;
+}
+
+__global__ void k_zero_u64(unsigned long long *p, int64_t n) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += stride) p[i] = 0ull;
+}
+
+void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
+                       unsigned long long h_push, unsigned long long h_pull, int first, cudaStream_t s) {
+    note_launch();
+    k_bfs_decide<<<1, 32, 0, s>>>(c, st, prev, h_loop, h_push, h_pull, first);
+}
+void launch_bfs_seed(const BfsCtrl *c, uint32_t *level, uint64_t *bits, uint64_t *summ, uint64_t *visited,
+                     cudaStream_t s) {
+    note_launch();
+    k_bfs_seed<<<1, 1, 0, s>>>(c, level, bits, summ, visited);
+}
+void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
+                         int64_t nw2, DevStats *zero_st, cudaStream_t s) {
+    int64_t blocks = (nw1 + 255) / 256;
+    if (blocks > 148 * 4) blocks = 148 * 4;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_clear_listed<<<(int)blocks, 256, 0, s>>>(bits, summ, offsets, st, nw2, zero_st);
+}
+void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s) {
+    int64_t blocks = (n + 255) / 256;
+    if (blocks > 148 * 4) blocks = 148 * 4;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_zero_u64<<<(int)blocks, 256, 0, s>>>(p, n);
+}
+
+}  // namespace sg

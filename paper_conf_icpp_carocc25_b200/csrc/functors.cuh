@@ -28,6 +28,7 @@ struct FnBfs {
     uint64_t *visited;
     uint32_t *level;
     uint32_t next;
+    const uint32_t *next_ptr;   // device-driven loop: level value read at flip time (else `next`)
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t) const { return 0u; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return ld_word(visited + (v >> 6)); }
@@ -35,7 +36,7 @@ struct FnBfs {
         const uint64_t m = 1ull << (v & 63);
         if (pr & m) return;
         if (atomic_or_u64(visited + (v >> 6), m) & m) return;
-        level[v] = next;
+        level[v] = next_ptr ? *next_ptr : next;
         out.insert(v);
     }
 };

@@ -45,7 +45,7 @@ struct PushLaunch {
     int grid_words;     // CTAs for k_push_words
     int grid_heavy;     // CTAs for k_push_heavy
 };
-struct BfsArgs { uint64_t *visited; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; };
+struct BfsArgs { uint64_t *visited; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; const uint32_t *next_ptr = nullptr; };
 struct SsspArgs { uint32_t *dist; uint64_t *out_bits, *out_summ; };
 struct CcArgs { int32_t *label; uint64_t *out_bits, *out_summ; };
 struct BcArgs { const uint64_t *visited; double *sigma; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; };
@@ -58,7 +58,17 @@ int push_max_grid_heavy();
 
 // pull.cu — bottom-up BFS step (direction-optimising, Beamer)
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
-                     uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s);
+                     uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
+                     const uint32_t *next_ptr = nullptr);
+
+// ctrl.cu — device-side superstep control (CUDA-graph driven loops)
+void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
+                       unsigned long long h_push, unsigned long long h_pull, int first, cudaStream_t s);
+void launch_bfs_seed(const BfsCtrl *c, uint32_t *level, uint64_t *bits, uint64_t *summ, uint64_t *visited,
+                     cudaStream_t s);
+void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
+                         int64_t nw2, DevStats *zero_st, cudaStream_t s);
+void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s);
 
 // bc.cu — Brandes helpers
 void launch_bc_level_max(const double *sigma, const uint64_t *bits, const uint32_t *offsets, const DevStats *st,

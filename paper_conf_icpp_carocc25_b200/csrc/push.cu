@@ -41,6 +41,7 @@ void launch_push_bfs(const PushLaunch &L, const BfsArgs &a, cudaStream_t s) {
     f.visited = a.visited;
     f.level = a.level;
     f.next = a.next;
+    f.next_ptr = a.next_ptr;
     f.out = OutSink{a.out_bits, a.out_summ};
     launch_push(L, f, s);
 }

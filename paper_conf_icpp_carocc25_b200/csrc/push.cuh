@@ -215,12 +215,17 @@ __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) 
     unsigned long long arcs = 0;
     // each warp grabs `batch` words (the coarsening factor) with one atomic; no CTA barrier in
     // the loop, so a warp never waits for a slower sibling's batch
+    uint32_t batch = (uint32_t)p.batch;
+    if (batch == 0) {   // device-driven loop: coarsening factor from the device-side count
+        batch = count / (gridDim.x * PUSH_WARPS * 4u);
+        batch = batch < 1u ? 1u : (batch > 8u ? 8u : batch);
+    }
     for (;;) {
         uint32_t b0 = 0;
-        if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)p.batch);
+        if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)batch);
         b0 = __shfl_sync(0xffffffffu, b0, 0);
         if (b0 >= count) break;
-        const uint32_t b1 = min(b0 + (uint32_t)p.batch, count);
+        const uint32_t b1 = min(b0 + batch, count);
         for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid]);
     }
     arcs = warp_sum(arcs);

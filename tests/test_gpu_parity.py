@@ -89,12 +89,44 @@ def _dir(sg, d):
     return {"push": sg.SG_DIR_PUSH, "pull": sg.SG_DIR_PULL, "auto": sg.SG_DIR_AUTO}[d]
 
 
+@pytest.mark.parametrize("host_loop", [False, True])
 @pytest.mark.parametrize("direction", DIRS)
-def test_bfs_config1(sg, direction):
+def test_bfs_config1(sg, direction, host_loop):
     g = gen.rmat(10, 16)
     G = load(sg, g)
-    lv, st = sg.run_bfs(G, 0, direction=_dir(sg, direction))
+    lv, st = sg.run_bfs(G, 0, direction=_dir(sg, direction), host_loop=host_loop)
     assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, 0))
+    assert st.iterations == int(oracle.bfs(g, 0)[oracle.bfs(g, 0) != INF].max()) + 1
+
+
+def test_bfs_graph_and_host_loop_agree_on_stats(sg):
+    """The CUDA-graph driven loop (device-side direction policy) and the host loop take the same
+    direction decisions, so levels and per-direction step counts agree."""
+    g = gen.rmat(15, 16, permute=True)
+    G = load(sg, g)
+    for s in gen.sources(g, 4):
+        a, sa = sg.run_bfs(G, int(s))
+        b, sb = sg.run_bfs(G, int(s), host_loop=True)
+        assert np.array_equal(sg.as_u32(a), sg.as_u32(b))
+        assert (sa.iterations, sa.push_steps, sa.pull_steps) == (sb.iterations, sb.push_steps, sb.pull_steps)
+        assert sa.reached == sb.reached == int((sg.as_u32(a) != INF).sum())
+
+
+def test_bfs_graph_reuse_across_sources_and_buffers(sg):
+    import torch
+    g = gen.rmat(12, 16, permute=True)
+    G = load(sg, g)
+    bufs = [torch.empty(g.n, dtype=torch.int32, device="cuda") for _ in range(2)]
+    for i, s in enumerate(gen.sources(g, 6)):
+        lv, _ = sg.run_bfs(G, int(s), level=bufs[i % 2])
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s)))
+
+
+def test_bfs_iteration_cap(sg):
+    G = load(sg, gen.path(100))
+    for hl in (False, True):
+        with pytest.raises(sg.SgError):
+            sg.run_bfs(G, 0, max_iters=10, host_loop=hl)
 
 
 @pytest.mark.parametrize("opts", [dict(), dict(heavy_degree=1), dict(heavy_degree=40), dict(small_degree=-1),
