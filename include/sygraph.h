@@ -75,7 +75,9 @@ typedef struct {
     int32_t small_degree;     /* degree <= small_degree uses the thread-granular packed tier (0 = default, <0 = none) */
     int32_t host_loop;        /* run_bfs: 1 = host-driven superstep loop (one control read per level);
                                  0 = one CUDA graph with device-side control (default) */
-    int32_t reserved[7];
+    int32_t segmented;        /* BFS hub tier with the visited slice in shared memory:
+                                 0 = auto (heavy supersteps), 1 = off, 2 = always */
+    int32_t reserved[6];
 } sg_opts;
 
 typedef struct {

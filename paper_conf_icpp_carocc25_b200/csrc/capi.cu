@@ -98,7 +98,9 @@ struct Workspace {
     cudaGraph_t bfs_graph = nullptr;
     cudaGraphExec_t bfs_exec = nullptr;
     uint32_t *bfs_level = nullptr;
-    int32_t bfs_heavy = 0, bfs_small = 0;
+    int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1;
+    SegItem *seg = nullptr;        // destination-segmented hub queue (BFS)
+    uint32_t seg_cap = 0;
     cudaStream_t cap_stream = nullptr;
 };
 
@@ -109,6 +111,10 @@ struct sg_graph {
     uint8_t *w = nullptr;
     uint8_t *deg8 = nullptr;
     uint64_t *isolated = nullptr;   // bit v <=> deg(v) == 0
+    int32_t *hub_idx = nullptr;     // hub index of u (deg >= SEG_MIN) or -1
+    int32_t *hub_vertex = nullptr;
+    uint32_t *hub_off = nullptr;    // [nhubs][nseg+1] segment offsets within the hub's row
+    int64_t nhubs = 0;
     uint32_t max_w = 0;
     int device = 0;
     Workspace *ws = nullptr;
@@ -171,6 +177,12 @@ static int ensure_heavy(sg_graph *g, int32_t heavy_deg) {
     CK(cudaMalloc(&ws->heavy, sizeof(HeavyItem) * (size_t)cap64));
     ws->heavy_cap = (uint32_t)cap64;
     ws->heavy_deg = heavy_deg;
+    // segmented hub queue: sum over hubs of ceil(deg / CHUNK) <= nnz / CHUNK + nhubs
+    if (!ws->seg && g->nhubs > 0) {
+        const int64_t scap = g->v.nnz / HEAVY_CHUNK + g->nhubs + 64;
+        CK(cudaMalloc(&ws->seg, sizeof(SegItem) * (size_t)scap));
+        ws->seg_cap = (uint32_t)scap;
+    }
     return SG_OK;
 }
 
@@ -181,6 +193,7 @@ static void free_ws(Workspace *ws) {
     cudaFreeHost(ws->h_st);
     cudaFree(ws->visited);
     cudaFree(ws->heavy);
+    cudaFree(ws->seg);
     cudaFree(ws->scratch);
     cudaFreeHost(ws->h_scratch);
     cudaFree(ws->stack);
@@ -269,12 +282,17 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     CK(cudaMalloc(&g->isolated, sizeof(uint64_t) * (size_t)g->v.nw1));
     launch_isolated(g->deg8, n, g->v.nw1, g->isolated, s);
     unsigned long long *dscr = nullptr;
-    CK(cudaMalloc(&dscr, 16));
-    CK(cudaMemsetAsync(dscr, 0, 16, s));
+    CK(cudaMalloc(&dscr, 24));
+    CK(cudaMemsetAsync(dscr, 0, 24, s));
     if (flags & SG_F_VALIDATE) launch_validate_csr(g->v, dscr, s);
     if (g->w) launch_max_weight(g->w, nnz, reinterpret_cast<unsigned int *>(dscr + 1), s);
-    unsigned long long h[2] = {0, 0};
-    CK(cudaMemcpyAsync(h, dscr, 16, cudaMemcpyDeviceToHost, s));
+    // hubs of the destination-segmented BFS tier (deg >= SEG_MIN): index map + vertex list
+    const int64_t max_hubs = nnz / SEG_MIN + 1;
+    CK(cudaMalloc(&g->hub_idx, sizeof(int32_t) * (size_t)n));
+    CK(cudaMalloc(&g->hub_vertex, sizeof(int32_t) * (size_t)max_hubs));
+    launch_hub_mark(g->rp, n, g->hub_idx, g->hub_vertex, reinterpret_cast<unsigned int *>(dscr + 2), s);
+    unsigned long long h[3] = {0, 0, 0};
+    CK(cudaMemcpyAsync(h, dscr, 24, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     CK(cudaGetLastError());
     cudaFree(dscr);
@@ -282,6 +300,16 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     if (h[0]) {
         graph_free(g);
         return fail(SG_ERR_INVALID, "CSR validation failed (%llu bad entries)", h[0]);
+    }
+    g->nhubs = (int64_t)(h[2] & 0xffffffffu);
+    g->v.nseg = (int32_t)((n + SEG_V - 1) / SEG_V);
+    if (g->nhubs > 0) {
+        CK(cudaMalloc(&g->hub_off, sizeof(uint32_t) * (size_t)g->nhubs * (size_t)(g->v.nseg + 1)));
+        launch_hub_off(g->rp, g->col, g->hub_vertex, g->nhubs, g->v.nseg, g->hub_off, s);
+        CK(cudaStreamSynchronize(s));
+        CK(cudaGetLastError());
+        g->v.hub_idx = g->hub_idx;
+        g->v.hub_off = g->hub_off;
     }
     *out = g;
     return SG_OK;
@@ -295,6 +323,9 @@ SG_API int graph_free(sg_graph *g) {
     cudaFree(g->w);
     cudaFree(g->deg8);
     cudaFree(g->isolated);
+    cudaFree(g->hub_idx);
+    cudaFree(g->hub_vertex);
+    cudaFree(g->hub_off);
     delete g;
     return SG_OK;
 }
@@ -424,13 +455,18 @@ SG_API int frontier_or_into(const sg_frontier *f, uint64_t *dst, void *stream) {
 // superstep helpers
 struct Tiers {
     int32_t heavy, small;
+    int32_t seg;   // destination-segmented hub tier for BFS: 0 off, 1 auto, 2 always
 };
+// auto mode: the segmented tier pays for its per-segment slice loads only on heavy supersteps
+static const unsigned long long kSegThreshold = 32ull << 20;   // estimated frontier arcs (m_f)
+
 static Tiers tiers_from(const sg_opts *o) {
-    Tiers t{kDefaultHeavy, kDefaultSmall};
+    Tiers t{kDefaultHeavy, kDefaultSmall, 1};
     if (o && o->heavy_degree > 0) t.heavy = o->heavy_degree;
     if (o && o->small_degree > 0) t.small = o->small_degree;
     if (o && o->small_degree < 0) t.small = 0;           // no thread tier
     if (t.small > t.heavy) t.small = t.heavy;
+    if (o) t.seg = o->segmented == 1 ? 0 : (o->segmented == 2 ? 2 : 1);
     return t;
 }
 
@@ -468,6 +504,10 @@ static PushLaunch push_launch(const sg_graph *g, const sg_frontier *in, Tiers t,
         L.grid_words = (int)gw;
     }
     L.grid_heavy = push_max_grid_heavy();
+    L.seg = g->ws->seg;
+    L.seg_cap = g->ws->seg_cap;
+    L.seg_mode = g->v.hub_idx ? t.seg : 0;
+    L.seg_threshold = kSegThreshold;
     return L;
 }
 
@@ -601,7 +641,7 @@ static int add_cond(cudaGraph_t graph, const std::vector<cudaGraphNode_t> &deps,
     return SG_OK;
 }
 
-static int build_bfs_graph(sg_graph *g, uint32_t *level, Tiers t) {
+static int build_bfs_graph(sg_graph *g, Tiers t) {
     Workspace *ws = g->ws;
     const GraphView &G = g->v;
     if (ws->bfs_exec) cudaGraphExecDestroy(ws->bfs_exec);
@@ -627,14 +667,14 @@ static int build_bfs_graph(sg_graph *g, uint32_t *level, Tiers t) {
     std::vector<cudaGraphNode_t> leaves;
     // prologue: level = INF, frontiers cleared, visited = isolated, seed src, compact + decide
     TRY(capture_begin(cs, root, {}));
-    CK(cudaMemsetAsync(level, 0xFF, sizeof(uint32_t) * (size_t)G.n, cs));
+    launch_bfs_level_init(ws->ctrl, G.n, cs);
     for (int i = 0; i < 2; i++) {
         CK(cudaMemsetAsync(F[i]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
         CK(cudaMemsetAsync(F[i]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
     }
     CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), cs));
     CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
-    launch_bfs_seed(ws->ctrl, level, F[0]->bits, F[0]->summ, ws->visited, cs);
+    launch_bfs_seed(ws->ctrl, F[0]->bits, F[0]->summ, ws->visited, cs);
     launch_compact(F[0]->summ, G.nw2, F[0]->offsets, F[0]->st, cs);
     launch_frontier_stats(G, F[0]->bits, F[0]->st, cs);
     launch_bfs_decide(ws->ctrl, F[0]->st, nullptr, h_loop, h_push[0], h_pull[0], 1, cs);
@@ -652,12 +692,13 @@ static int build_bfs_graph(sg_graph *g, uint32_t *level, Tiers t) {
         TRY(add_cond(body, deps, h_pull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = 0;   // coarsening factor computed on the device from the count
-        BfsArgs a{ws->visited, level, 0u, out->bits, out->summ, &ws->ctrl->next};
+        BfsArgs a{ws->visited, nullptr, 0u, out->bits, out->summ, &ws->ctrl->next, &ws->ctrl->level};
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
         TRY(capture_end(cs, leaves));
         TRY(capture_begin(cs, b_pull, {}));
-        launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, level, 0u, in->st, cs, &ws->ctrl->next);
+        launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, nullptr, 0u, in->st, cs, &ws->ctrl->next,
+                        &ws->ctrl->level);
         TRY(capture_end(cs, leaves));
         TRY(capture_begin(cs, body, {n_push, n_pull}));
         launch_clear_listed(in->bits, in->summ, in->offsets, in->st, G.nw1, G.nw2, out->st, cs);
@@ -667,9 +708,9 @@ static int build_bfs_graph(sg_graph *g, uint32_t *level, Tiers t) {
         TRY(capture_end(cs, deps));
     }
     CK(cudaGraphInstantiate(&ws->bfs_exec, root, 0));
-    ws->bfs_level = level;
     ws->bfs_heavy = t.heavy;
     ws->bfs_small = t.small;
+    ws->bfs_seg = t.seg;
     return SG_OK;
 }
 
@@ -677,10 +718,11 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
                          sg_stats *stats) {
     Workspace *ws = g->ws;
     cudaStream_t s = stream_of(&o);
-    if (!ws->bfs_exec || ws->bfs_level != level || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small)
-        TRY(build_bfs_graph(g, level, t));
+    if (!ws->bfs_exec || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small || ws->bfs_seg != t.seg)
+        TRY(build_bfs_graph(g, t));
     BfsCtrl &c = *ws->h_ctrl;
     memset(&c, 0, sizeof c);
+    c.level = level;
     c.mu = g->v.nnz;
     c.n = g->v.n;
     c.max_iters = max_iters;

@@ -19,6 +19,9 @@ struct GraphView {
     const uint8_t *__restrict__ deg8;  // 8-bit log-coded degrees, nw1*64 bytes (direction policy only)
     int64_t n, nnz;
     int64_t nw1, nw2;
+    const int32_t *__restrict__ hub_idx;   // hub index of u (deg >= SEG_MIN) or -1; nullptr: no segmentation
+    const uint32_t *__restrict__ hub_off;  // [nhubs][nseg+1] neighbours of the hub with id < b*SEG_V
+    int32_t nseg;                          // ceil(n / SEG_V)
 };
 
 // Per-superstep control block, device resident; host reads it back with one 64-B copy.
@@ -29,7 +32,7 @@ struct DevStats {
     unsigned long long arcs;         // arcs inspected by the advance
     unsigned long long batch;        // push: next word batch (dynamic CTA scheduling)
     unsigned long long heavy_count;  // push: CTA/grid-tier chunks queued
-    unsigned long long changed;      // algorithm-specific flag/counter
+    unsigned long long seg_count;    // push: destination-segmented hub chunks queued (BFS)
     unsigned long long pad;
 };
 
@@ -40,6 +43,7 @@ struct BfsCtrl {
     long long nf_prev;
     long long n, max_iters;
     double alpha, beta;
+    uint32_t *level;         // output buffer of this run (kernels read the pointer: one graph serves any buffer)
     int32_t src;
     uint32_t next;           // level value written by the superstep being launched
     uint32_t pull;           // direction of the superstep being launched
@@ -56,6 +60,22 @@ struct HeavyItem {
 };
 
 constexpr int HEAVY_CHUNK = 4096;     // arcs per CTA-tier work unit (16 KB of col_idx)
+
+// Destination-segmented hub tier (BFS): the visited bitmap is processed in segments of SEG_V
+// vertices whose slice (SEG_V/8 bytes) fits one CTA's shared memory; hub rows (deg >= SEG_MIN)
+// carry per-segment offsets computed at graph load.
+constexpr int SEG_WORDS = 24576;                       // 192 KB of layer-1 words per slice
+constexpr int64_t SEG_V = (int64_t)SEG_WORDS * 64;     // 1,572,864 vertices per segment
+#ifndef SG_SEG_MIN
+#define SG_SEG_MIN 256
+#endif
+constexpr int SEG_MIN = SG_SEG_MIN;                    // hub threshold (degree)
+struct SegItem {
+    int64_t begin;   // first arc of the chunk
+    int64_t row;     // row_ptr[u] (segment offsets are relative to it)
+    int32_t len;     // arcs in the chunk (<= HEAVY_CHUNK)
+    int32_t h;       // hub index (row of the segment-offset table)
+};
 
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 

@@ -50,10 +50,10 @@ __global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *pre
     set_cond(h_loop, go);
 }
 
-// BFS prologue on the device: level[src] = 0, in = {src}, visited |= {src} (src from ctrl).
-__global__ void k_bfs_seed(const BfsCtrl *c, uint32_t *level, uint64_t *bits, uint64_t *summ, uint64_t *visited) {
+// BFS prologue on the device: level[src] = 0, in = {src}, visited |= {src} (src, level from ctrl).
+__global__ void k_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited) {
     const int32_t src = c->src;
-    level[src] = 0u;
+    c->level[src] = 0u;
     bits[src >> 6] = 1ull << (src & 63);
     summ[src >> 12] = 1ull << ((src >> 6) & 63);
     visited[src >> 6] |= 1ull << (src & 63);
@@ -82,10 +82,30 @@ void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, uns
     note_launch();
     k_bfs_decide<<<1, 32, 0, s>>>(c, st, prev, h_loop, h_push, h_pull, first);
 }
-void launch_bfs_seed(const BfsCtrl *c, uint32_t *level, uint64_t *bits, uint64_t *summ, uint64_t *visited,
-                     cudaStream_t s) {
+void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, cudaStream_t s) {
     note_launch();
-    k_bfs_seed<<<1, 1, 0, s>>>(c, level, bits, summ, visited);
+    k_bfs_seed<<<1, 1, 0, s>>>(c, bits, summ, visited);
+}
+
+// level[0..n) = UINT32_MAX with the buffer pointer taken from ctrl (16-B stores)
+__global__ void k_bfs_level_init(const BfsCtrl *c, int64_t n) {
+    uint32_t *level = c->level;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (((uintptr_t)level & 15) == 0) {
+        uint4 *l4 = reinterpret_cast<uint4 *>(level);
+        for (int64_t i = t; i < n / 4; i += stride) l4[i] = make_uint4(INF32, INF32, INF32, INF32);
+        for (int64_t i = (n / 4) * 4 + t; i < n; i += stride) level[i] = INF32;
+    } else {
+        for (int64_t i = t; i < n; i += stride) level[i] = INF32;
+    }
+}
+void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s) {
+    int64_t blocks = (n / 4 + 255) / 256;
+    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_bfs_level_init<<<(int)blocks, 256, 0, s>>>(c, n);
 }
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s) {

@@ -23,12 +23,14 @@ struct OutSink {
 // frontier}, identical to the frozen-visited reading.
 struct FnBfs {
     static constexpr bool kWeights = false;
+    static constexpr bool kSeg = true;      // hubs may take the destination-segmented tier
     using Ctx = uint32_t;
     using Probe = uint64_t;
     uint64_t *visited;
     uint32_t *level;
     uint32_t next;
     const uint32_t *next_ptr;   // device-driven loop: level value read at flip time (else `next`)
+    uint32_t *const *level_pp;  // device-driven loop: output buffer pointer read at flip time (else `level`)
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t) const { return 0u; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return ld_word(visited + (v >> 6)); }
@@ -36,7 +38,7 @@ struct FnBfs {
         const uint64_t m = 1ull << (v & 63);
         if (pr & m) return;
         if (atomic_or_u64(visited + (v >> 6), m) & m) return;
-        level[v] = next_ptr ? *next_ptr : next;
+        (level_pp ? *level_pp : level)[v] = next_ptr ? *next_ptr : next;
         out.insert(v);
     }
 };
@@ -45,6 +47,7 @@ struct FnBfs {
 // iff its distance decreased.  Updates are visible immediately (reading C12).
 struct FnSssp {
     static constexpr bool kWeights = true;
+    static constexpr bool kSeg = false;
     using Ctx = uint32_t;
     using Probe = uint32_t;
     uint32_t *dist;
@@ -63,6 +66,7 @@ struct FnSssp {
 // label decreased.  Fixed point: min id per component (reading C13).
 struct FnCc {
     static constexpr bool kWeights = false;
+    static constexpr bool kSeg = false;
     using Ctx = int32_t;
     using Probe = int32_t;
     int32_t *label;
@@ -80,6 +84,7 @@ struct FnCc {
 // output bit writes level[v] = d + 1.
 struct FnBcSigma {
     static constexpr bool kWeights = false;
+    static constexpr bool kSeg = false;
     using Ctx = double;
     using Probe = uint64_t;
     const uint64_t *visited;

@@ -41,11 +41,26 @@ struct PushLaunch {
     HeavyItem *heavy;
     uint32_t heavy_cap;
     int32_t heavy_deg, small_deg;
-    int32_t batch;      // words per CTA grab (coarsening factor x 8 warps)
+    int32_t batch;      // words per warp grab (coarsening factor; 0 = from the device-side count)
     int grid_words;     // CTAs for k_push_words
     int grid_heavy;     // CTAs for k_push_heavy
+    SegItem *seg = nullptr;          // destination-segmented hub tier (BFS only)
+    uint32_t seg_cap = 0;
+    int32_t seg_mode = 0;            // 0 off, 1 auto, 2 always
+    unsigned long long seg_threshold = 0;
 };
-struct BfsArgs { uint64_t *visited; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; const uint32_t *next_ptr = nullptr; };
+void launch_hub_mark(const int64_t *rp, int64_t n, int32_t *hub_idx, int32_t *hub_vertex, unsigned int *count,
+                     cudaStream_t s);
+void launch_hub_off(const int64_t *rp, const int32_t *col, const int32_t *hub_vertex, int64_t nh, int nseg,
+                    uint32_t *off, cudaStream_t s);
+struct BfsArgs {
+    uint64_t *visited;
+    uint32_t *level;
+    uint32_t next;
+    uint64_t *out_bits, *out_summ;
+    const uint32_t *next_ptr = nullptr;    // graph mode: read `next` / `level` from BfsCtrl
+    uint32_t *const *level_pp = nullptr;
+};
 struct SsspArgs { uint32_t *dist; uint64_t *out_bits, *out_summ; };
 struct CcArgs { int32_t *label; uint64_t *out_bits, *out_summ; };
 struct BcArgs { const uint64_t *visited; double *sigma; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; };
@@ -59,13 +74,13 @@ int push_max_grid_heavy();
 // pull.cu — bottom-up BFS step (direction-optimising, Beamer)
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
                      uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
-                     const uint32_t *next_ptr = nullptr);
+                     const uint32_t *next_ptr = nullptr, uint32_t *const *level_pp = nullptr);
 
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
                        unsigned long long h_push, unsigned long long h_pull, int first, cudaStream_t s);
-void launch_bfs_seed(const BfsCtrl *c, uint32_t *level, uint64_t *bits, uint64_t *summ, uint64_t *visited,
-                     cudaStream_t s);
+void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, cudaStream_t s);
+void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s);
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s);
 void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s);

@@ -25,8 +25,9 @@ constexpr int PULL_ARCS = SG_PULL_ARCS;   // arcs per vertex per iteration
 __global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited,
            uint64_t *__restrict__ out_bits, uint64_t *__restrict__ out_summ, uint32_t *__restrict__ level,
-           uint32_t next, DevStats *st, const uint32_t *next_ptr) {
+           uint32_t next, DevStats *st, const uint32_t *next_ptr, uint32_t *const *level_pp) {
     if (next_ptr) next = *next_ptr;
+    if (level_pp) level = *level_pp;
     __shared__ unsigned long long s_arcs[PULL_THREADS / 32];
     const int lane = lane_id();
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -96,12 +97,13 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
 
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
                      uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
-                     const uint32_t *next_ptr) {
+                     const uint32_t *next_ptr, uint32_t *const *level_pp) {
     int64_t blocks = (g.nw1 * 32 + PULL_THREADS - 1) / PULL_THREADS;
     if (blocks > 148 * SG_PULL_MINB) blocks = 148 * SG_PULL_MINB;
     if (blocks < 1) blocks = 1;
     note_launch();
-    k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, out_bits, out_summ, level, next, st, next_ptr);
+    k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, out_bits, out_summ, level, next, st, next_ptr,
+                                                    level_pp);
 }
 
 }  // namespace sg

@@ -42,7 +42,11 @@ struct PushParams {
     uint32_t heavy_cap;
     int32_t heavy_deg;
     int32_t small_deg;
-    int32_t batch;         // words per CTA grab (multiple of PUSH_WARPS)
+    int32_t batch;         // words per warp grab (0: derive from the device-side count)
+    SegItem *seg;          // destination-segmented hub queue (BFS only)
+    uint32_t seg_cap;
+    int32_t seg_mode;      // 0 off, 1 auto (when the frontier's m_f >= seg_threshold), 2 always
+    unsigned long long seg_threshold;
 };
 
 template <class F>
@@ -117,15 +121,44 @@ __device__ __forceinline__ void enqueue_heavy(const PushParams &p, int32_t u, in
     }
 }
 
+// ---- segmented hub tier enqueue (BFS) ----------------------------------------------------
+__device__ __forceinline__ void enqueue_seg(const PushParams &p, int32_t h, int64_t s, int64_t e) {
+    const int64_t d = e - s;
+    const uint32_t nch = (uint32_t)((d + HEAVY_CHUNK - 1) / HEAVY_CHUNK);
+    const unsigned long long pos = atomicAdd(&p.st->seg_count, (unsigned long long)nch);
+    for (uint32_t j = 0; j < nch; j++) {
+        if (pos + j >= p.seg_cap) break;        // cannot happen: capacity bound in DESIGN.md
+        SegItem it;
+        it.begin = s + (int64_t)j * HEAVY_CHUNK;
+        it.row = s;
+        it.len = (int32_t)min((int64_t)HEAVY_CHUNK, e - it.begin);
+        it.h = h;
+        p.seg[pos + j] = it;
+    }
+}
+
 // ---- one word on one warp ----------------------------------------------------------------
 template <class F>
 __device__ __forceinline__ unsigned long long push_word(const PushParams &p, const F &f, int64_t w,
-                                                        PushWarpSmem<F> &sm) {
+                                                        PushWarpSmem<F> &sm, bool seg_on) {
     const int lane = lane_id();
     const uint64_t x = __ldg(p.in_bits + w);
     int64_t sa, ea, sb, eb;
     word_bounds(p.g, w, x, sa, ea, sb, eb);
     const int32_t ua = (int32_t)(w * 64 + lane), ub = ua + 32;
+    const int64_t d_total = (ea - sa) + (eb - sb);
+    if constexpr (F::kSeg) {
+        if (seg_on) {   // hubs go to the destination-segmented tier (visited slice in shared memory)
+            if (ea - sa >= SEG_MIN) {
+                enqueue_seg(p, __ldg(p.g.hub_idx + ua), sa, ea);
+                sa = ea;
+            }
+            if (eb - sb >= SEG_MIN) {
+                enqueue_seg(p, __ldg(p.g.hub_idx + ub), sb, eb);
+                sb = eb;
+            }
+        }
+    }
     const int64_t da = ea - sa, db = eb - sb;
     const bool ha = da > p.heavy_deg, hb = db > p.heavy_deg;
     if (ha) enqueue_heavy(p, ua, sa, ea);
@@ -203,7 +236,7 @@ __device__ __forceinline__ unsigned long long push_word(const PushParams &p, con
         }
         __syncwarp();
     }
-    return (unsigned long long)(da + db);
+    return (unsigned long long)d_total;
 }
 
 template <class F>
@@ -220,13 +253,17 @@ __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) 
         batch = count / (gridDim.x * PUSH_WARPS * 4u);
         batch = batch < 1u ? 1u : (batch > 8u ? 8u : batch);
     }
+    bool seg_on = false;
+    if constexpr (F::kSeg)
+        seg_on = p.g.hub_idx != nullptr && p.seg != nullptr &&
+                 (p.seg_mode == 2 || (p.seg_mode == 1 && p.st->mf >= p.seg_threshold));
     for (;;) {
         uint32_t b0 = 0;
         if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)batch);
         b0 = __shfl_sync(0xffffffffu, b0, 0);
         if (b0 >= count) break;
         const uint32_t b1 = min(b0 + batch, count);
-        for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid]);
+        for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid], seg_on);
     }
     arcs = warp_sum(arcs);
     if (lane_id() == 0) s_arcs[wid] = arcs;

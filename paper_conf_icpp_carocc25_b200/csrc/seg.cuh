@@ -1,0 +1,162 @@
+// seg.cuh — destination-segmented hub tier of the BFS push advance.
+//
+// The per-arc visited probe of a push step is one random 8-B load into a 2 MB bitmap: one L1
+// wavefront and one L2 sector per arc, which caps the top-down advance far below HBM bandwidth
+// (ncu: profiles/r01_ncu_full_push_pull_level3.txt).  For hub rows (deg >= SEG_MIN) this tier
+// instead walks the destination space in segments of SEG_V vertices: each CTA (one per SM,
+// 192 KB of shared memory) copies the segment's visited slice into shared memory, streams the
+// part of every queued hub chunk that falls in the segment (per-hub segment offsets computed at
+// graph load; rows are sorted, so each part is contiguous), probes and marks bits in shared
+// memory, then flushes: for each slice word, bits it set that are not yet set globally go to
+// one global atomicOr; the CTA whose atomic flips a bit writes the level and the output
+// frontier.  Same result set as the probe path (advance semantics PAPER.md:116/123; tested).
+//
+// Per warp, 32 chunk parts are packed into one arc list (prefix sum of their lengths) and
+// streamed in 32-arc windows, 4 windows in flight per iteration: short parts (a mid hub has
+// ~deg/11 arcs per segment) do not idle lanes.
+#pragma once
+#include "common.cuh"
+#include "functors.cuh"
+#include "push.cuh"
+
+namespace sg {
+
+constexpr int SEG_THREADS = 1024;
+constexpr size_t SEG_SMEM = (size_t)SEG_WORDS * sizeof(uint64_t);
+#ifndef SG_SEG_UNROLL
+#define SG_SEG_UNROLL 4
+#endif
+#ifndef SG_SEG_LONG
+#define SG_SEG_LONG 192
+#endif
+constexpr int SEG_UNROLL = SG_SEG_UNROLL;
+constexpr uint32_t SEG_LONG = SG_SEG_LONG;   // parts at least this long are streamed with int4 loads
+
+__global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs f) {
+    extern __shared__ __align__(16) uint64_t s_vis[];
+    const unsigned long long cnt = p.st->seg_count;
+    const uint32_t nitems = (uint32_t)(cnt < p.seg_cap ? cnt : p.seg_cap);
+    if (nitems == 0) return;
+    const uint32_t i0 = (uint32_t)((uint64_t)nitems * blockIdx.x / gridDim.x);
+    const uint32_t i1 = (uint32_t)((uint64_t)nitems * (blockIdx.x + 1) / gridDim.x);
+    if (i0 == i1) return;
+    const int nseg = p.g.nseg, S1 = nseg + 1;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    constexpr int NW = SEG_THREADS / 32;
+    uint32_t *level = f.level_pp ? *f.level_pp : f.level;
+    const uint32_t next = f.next_ptr ? *f.next_ptr : f.next;
+    for (int b = 0; b < nseg; b++) {
+        const int64_t w0 = (int64_t)b * SEG_WORDS;
+        const int nw = (int)min((int64_t)SEG_WORDS, p.g.nw1 - w0);
+        for (int i = threadIdx.x; i < nw; i += SEG_THREADS) s_vis[i] = f.visited[w0 + i];
+        __syncthreads();
+        const int32_t vbase = (int32_t)(w0 * 64);
+        uint32_t *s_vis32 = reinterpret_cast<uint32_t *>(s_vis);   // 32-bit ATOMS.OR is native (64-bit is a CAS loop)
+        // items are dealt to warps with stride NW: consecutive chunks of one hub (which fall into
+        // the same segment) spread over all warps instead of piling onto one
+        for (uint32_t r = 0; i0 + r * 32 * NW + warp < i1; r++) {
+            // lane k: the part of item i0 + (r*32 + k)*NW + warp inside segment b
+            const uint32_t item = i0 + (r * 32 + lane) * NW + warp;
+            int64_t lo = 0;
+            uint32_t len = 0;
+            if (item < i1) {
+                const SegItem x = p.seg[item];
+                const uint32_t *off = p.g.hub_off + (size_t)x.h * S1;
+                int64_t a = x.row + __ldg(off + b), e = x.row + __ldg(off + b + 1);
+                a = max(a, x.begin);
+                e = min(e, x.begin + (int64_t)x.len);
+                if (e > a) {
+                    lo = a;
+                    len = (uint32_t)(e - a);
+                }
+            }
+            // long parts: the whole warp streams each with 16-B loads (no per-arc owner search)
+            uint32_t longm = __ballot_sync(0xffffffffu, len >= SEG_LONG);
+            while (longm) {
+                const int src = __ffs(longm) - 1;
+                longm &= longm - 1;
+                const int64_t s = __shfl_sync(0xffffffffu, lo, src);
+                const int64_t e = s + __shfl_sync(0xffffffffu, len, src);
+                int64_t a = (s + 3) & ~3ll;
+                const int64_t bb = a + ((e - a) & ~3ll);
+                {   // ragged head [s, a) on lanes 0..2, tail [bb, e) on lanes 4..6
+                    int64_t i = -1;
+                    if (lane < a - s) i = s + lane;
+                    else if (lane >= 4 && lane - 4 < e - bb) i = bb + (lane - 4);
+                    if (i >= 0) {
+                        const int32_t vv = __ldg(p.g.col + i) - vbase;
+                        const uint32_t m = 1u << (vv & 31);
+                        if (!(s_vis32[vv >> 5] & m)) atomicOr(s_vis32 + (vv >> 5), m);
+                    }
+                }
+                for (int64_t i = a + 4 * lane; i < bb; i += 256) {
+                    const bool two = i + 128 < bb;
+                    const int4 q0 = __ldg(reinterpret_cast<const int4 *>(p.g.col + i));
+                    int4 q1 = make_int4(vbase, vbase, vbase, vbase);
+                    if (two) q1 = __ldg(reinterpret_cast<const int4 *>(p.g.col + i + 128));
+                    const int32_t vv[8] = {q0.x - vbase, q0.y - vbase, q0.z - vbase, q0.w - vbase,
+                                           q1.x - vbase, q1.y - vbase, q1.z - vbase, q1.w - vbase};
+#pragma unroll
+                    for (int k = 0; k < 8; k++) {
+                        if (k >= 4 && !two) break;
+                        const uint32_t m = 1u << (vv[k] & 31);
+                        if (!(s_vis32[vv[k] >> 5] & m)) atomicOr(s_vis32 + (vv[k] >> 5), m);
+                    }
+                }
+            }
+            if (len >= SEG_LONG) len = 0;
+            // short parts: packed into one arc list, 32-arc windows
+            const uint32_t incl = warp_inclusive_scan(len);
+            const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+            const uint32_t pre = incl - len;
+            for (uint32_t win = 0; win < total; win += 32 * SEG_UNROLL) {
+                int32_t v[SEG_UNROLL];
+#pragma unroll
+                for (int j = 0; j < SEG_UNROLL; j++) {
+                    // owner of arc t = the last lane whose part starts at or before t (pre is
+                    // sorted over lanes; an empty lane is never the last such lane): 5-step
+                    // binary search with shuffles
+                    const uint32_t t = win + 32 * j + lane;
+                    int own = 0;
+#pragma unroll
+                    for (int step = 16; step > 0; step >>= 1) {
+                        const uint32_t pc = __shfl_sync(0xffffffffu, pre, own + step);
+                        if (pc <= t) own += step;
+                    }
+                    const int64_t lo_k = __shfl_sync(0xffffffffu, lo, own);
+                    const uint32_t pre_k = __shfl_sync(0xffffffffu, pre, own);
+                    v[j] = (t < total) ? __ldg(p.g.col + lo_k + (t - pre_k)) - vbase : -1;
+                }
+#pragma unroll
+                for (int j = 0; j < SEG_UNROLL; j++) {
+                    if (v[j] < 0) continue;
+                    const uint32_t m = 1u << (v[j] & 31);
+                    if (!(s_vis32[v[j] >> 5] & m)) atomicOr(s_vis32 + (v[j] >> 5), m);
+                }
+            }
+        }
+        __syncthreads();
+        // flush: bits this CTA set that are not set globally yet -> one atomicOr per word
+        for (int i = threadIdx.x; i < nw; i += SEG_THREADS) {
+            const int64_t w = w0 + i;
+            const uint64_t nb = s_vis[i] & ~f.visited[w];
+            if (!nb) continue;
+            const uint64_t old = atomic_or_u64(f.visited + w, nb);
+            const uint64_t flips = nb & ~old;
+            if (!flips) continue;
+            if (f.out.bits) {
+                const uint64_t oo = atomic_or_u64(f.out.bits + w, flips);
+                if (oo == 0ull) atomic_or_u64(f.out.summ + (w >> 6), 1ull << (w & 63));
+            }
+            uint64_t y = flips;
+            while (y) {
+                const int j = __ffsll((long long)y) - 1;
+                y &= y - 1;
+                level[w * 64 + j] = next;
+            }
+        }
+        __syncthreads();
+    }
+}
+
+}  // namespace sg

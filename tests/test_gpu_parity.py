@@ -139,6 +139,32 @@ def test_bfs_tier_forcing_invariant(sg, opts):
         assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (opts, s)
 
 
+@pytest.mark.parametrize("host_loop", [False, True])
+@pytest.mark.parametrize("make", [lambda: gen.rmat(14, 16, permute=True), lambda: gen.rmat(21, 8, permute=True),
+                                  lambda: gen.rmat(20, 16)])
+def test_bfs_segmented_hub_tier(sg, make, host_loop):
+    """Hubs (deg >= 256) through the destination-segmented tier (visited slice in shared memory),
+    forced on every superstep; RMAT-21 spans 3 segments of 802,816 vertices."""
+    g = make()
+    G = load(sg, g)
+    for s in list(gen.sources(g, 2)) + [int(np.argmax(g.degrees()))]:
+        for d in (sg.SG_DIR_PUSH, sg.SG_DIR_AUTO):
+            lv, _ = sg.run_bfs(G, int(s), direction=d, segmented=2, host_loop=host_loop)
+            assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (s, d)
+
+
+@pytest.mark.parametrize("deg", [255, 256, 257, 4097, 900_000])
+def test_bfs_segmented_degree_boundaries(sg, deg):
+    n = deg + 1 + 50
+    u = np.concatenate([np.zeros(deg, np.int64), np.arange(deg, n - 1)])
+    v = np.concatenate([np.arange(1, deg + 1), np.arange(deg + 1, n)])
+    g = gen.from_edges(n, u, v)
+    G = load(sg, g)
+    for s in (0, 1, n - 1):
+        lv, _ = sg.run_bfs(G, s, direction=sg.SG_DIR_PUSH, segmented=2)
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, s)), (deg, s)
+
+
 @pytest.mark.parametrize("make", [lambda: gen.path(5000), lambda: gen.cycle(4097), lambda: gen.grid(97, 131),
                                   lambda: gen.hypercube(16), lambda: gen.complete(300), lambda: gen.star(70_000),
                                   lambda: gen.lattice(300, 400, 0.6)])
