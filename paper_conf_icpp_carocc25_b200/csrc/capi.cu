@@ -101,6 +101,10 @@ struct Workspace {
     int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1;
     SegItem *seg = nullptr;        // destination-segmented hub queue (BFS)
     uint32_t seg_cap = 0;
+    // source-batched BC (bcb.cu)
+    BcbLaunch bcb{};
+    bool bcb_ready = false;
+    BcbCtrl *h_bcb = nullptr;
     cudaStream_t cap_stream = nullptr;
 };
 
@@ -203,6 +207,20 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->level);
     if (ws->bfs_exec) cudaGraphExecDestroy(ws->bfs_exec);
     if (ws->bfs_graph) cudaGraphDestroy(ws->bfs_graph);
+    {
+        BcbLaunch &B = ws->bcb;
+        cudaFree(B.F);
+        cudaFree(B.V);
+        cudaFree(B.M);
+        cudaFree(B.s);
+        cudaFree(B.delta);
+        cudaFree(B.lv);
+        cudaFree(B.lm);
+        cudaFree(B.loff);
+        cudaFree(B.maxb);
+        cudaFree(B.c);
+        cudaFreeHost(ws->h_bcb);
+    }
     if (ws->cap_stream) cudaStreamDestroy(ws->cap_stream);
     cudaFree(ws->ctrl);
     cudaFreeHost(ws->h_ctrl);
@@ -988,6 +1006,75 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     return SG_OK;
 }
 
+}  // extern "C"
+
+// ---- source-batched BC (bcb.cu): 32 sources per CUDA-graph launch -------------------------
+static int bcb_alloc(sg_graph *g) {
+    Workspace *ws = g->ws;
+    BcbLaunch &B = ws->bcb;
+    const int64_t n = g->v.n;
+    B.g = g->v;
+    B.cap = (int32_t)(n + 1 < (1 << 20) ? n + 1 : (1 << 20));
+    B.lcap = n * 32;   // each (vertex, source) pair is in at most one level entry
+    CK(cudaMalloc(&B.F, sizeof(uint32_t) * (size_t)n * 3));
+    CK(cudaMalloc(&B.V, sizeof(uint32_t) * (size_t)n));
+    CK(cudaMalloc(&B.M, sizeof(uint32_t) * (size_t)n * 2));
+    CK(cudaMalloc(&B.s, sizeof(double) * (size_t)n * 32));
+    CK(cudaMalloc(&B.delta, sizeof(double) * (size_t)n * 32));
+    CK(cudaMalloc(&B.lv, sizeof(int32_t) * (size_t)B.lcap));
+    CK(cudaMalloc(&B.lm, sizeof(uint32_t) * (size_t)B.lcap));
+    CK(cudaMalloc(&B.loff, sizeof(unsigned long long) * (size_t)(B.cap + 2)));
+    CK(cudaMalloc(&B.maxb, sizeof(unsigned long long) * (size_t)(B.cap + 1) * 32));
+    CK(cudaMalloc(&B.c, sizeof(BcbCtrl)));
+    CK(cudaMallocHost(&ws->h_bcb, sizeof(BcbCtrl)));
+    CK(cudaMemset(B.F, 0, sizeof(uint32_t) * (size_t)n * 3));
+    CK(cudaMemset(B.V, 0, sizeof(uint32_t) * (size_t)n));
+    CK(cudaMemset(B.M, 0, sizeof(uint32_t) * (size_t)n * 2));
+    CK(cudaMemset(B.maxb, 0, sizeof(unsigned long long) * (size_t)(B.cap + 1) * 32));
+    ws->bcb_ready = true;
+    return SG_OK;
+}
+
+// returns SG_ERR_OOM (caller falls back to the per-source path) if the batch buffers do not fit
+static int run_bc_batched(sg_graph *g, const int32_t *sources, int32_t k, double *bc, cudaStream_t s,
+                          sg_stats *stats) {
+    Workspace *ws = g->ws;
+    if (!ws->bcb_ready) {
+        const int r = bcb_alloc(g);
+        if (r != SG_OK) return r;
+    }
+    ws->bcb.bc = bc;
+    CK(cudaEventRecord(ws->ev0, s));
+    CK(cudaMemsetAsync(bc, 0, sizeof(double) * (size_t)g->v.n, s));
+    int64_t levels = 0;
+    for (int32_t b0 = 0; b0 < k; b0 += 32) {
+        BcbCtrl &c = *ws->h_bcb;
+        memset(&c, 0, sizeof c);
+        c.nsrc = k - b0 < 32 ? k - b0 : 32;
+        for (int j = 0; j < c.nsrc; j++) c.src[j] = sources[b0 + j];
+        CK(cudaMemcpyAsync(ws->bcb.c, &c, sizeof(BcbCtrl), cudaMemcpyHostToDevice, s));
+        CK(bcb_run_batch(ws->bcb, s));
+        CK(cudaMemcpyAsync(&c, ws->bcb.c, sizeof(BcbCtrl), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (c.overflow) return fail(SG_ERR_UNSUPPORTED, "batched BC: level/list capacity exceeded");
+        levels += c.depth;
+    }
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->iterations = 2 * levels;
+        stats->push_steps = levels;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
+extern "C" {
+
 // ---- BC (Brandes forward sigma + backward delta) -----------------------------------
 SG_API int run_bc(const sg_graph *gc, const int32_t *sources, int32_t k, double *bc, const sg_opts *opts,
                   sg_stats *stats) {
@@ -1004,6 +1091,12 @@ SG_API int run_bc(const sg_graph *gc, const int32_t *sources, int32_t k, double 
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
+    if (!o.host_loop && k > 0) {   // default: source-batched (f1); falls back when memory is short
+        const int r = run_bc_batched(g, sources, k, bc, s, stats);
+        if (r != SG_ERR_OOM) return r;
+        cudaGetLastError();
+        t_err.clear();
+    }
     if (!ws->sigma) {
         CK(cudaMalloc(&ws->sigma, sizeof(double) * (size_t)G.n));
         CK(cudaMalloc(&ws->delta, sizeof(double) * (size_t)G.n));

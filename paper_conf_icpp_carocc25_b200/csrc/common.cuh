@@ -52,6 +52,18 @@ struct BfsCtrl {
     uint32_t pad;
 };
 
+// Device-resident control of one source-batched BC batch (bcb.cu).
+struct BcbCtrl {
+    int32_t src[32];
+    int32_t nsrc;
+    int32_t d;                 // current level
+    int32_t par;               // frontier-mask parity
+    int32_t depth;             // number of levels
+    unsigned long long ltop;   // entries appended to the level lists
+    int32_t overflow;          // level / list capacity exceeded
+    int32_t pad;
+};
+
 // One CTA/grid-tier work unit: a contiguous piece of one vertex's adjacency list.
 struct HeavyItem {
     int64_t begin;   // first arc index

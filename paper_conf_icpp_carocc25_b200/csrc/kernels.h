@@ -85,6 +85,22 @@ void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets
                          int64_t nw2, DevStats *zero_st, cudaStream_t s);
 void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s);
 
+// bcb.cu — source-batched BC (32 sources per batch): init, cooperative forward and backward
+// kernels (grid-wide barriers between supersteps), reset
+struct BcbLaunch {
+    GraphView g;
+    uint32_t *F, *V, *M;
+    double *s, *delta;
+    int32_t *lv;
+    uint32_t *lm;
+    unsigned long long *loff, *maxb;
+    BcbCtrl *c;
+    int32_t cap;
+    int64_t lcap;
+    double *bc;
+};
+cudaError_t bcb_run_batch(const BcbLaunch &L, cudaStream_t s);
+
 // bc.cu — Brandes helpers
 void launch_bc_level_max(const double *sigma, const uint64_t *bits, const uint32_t *offsets, const DevStats *st,
                          int64_t max_words, unsigned long long *max_bits, cudaStream_t s);

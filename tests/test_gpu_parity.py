@@ -344,12 +344,24 @@ def test_cc_tiers(sg):
 @pytest.mark.parametrize("make,k", [(lambda: gen.random_simple(60, 0.08, 3), 60), (lambda: gen.path(300), 10),
                                     (lambda: gen.hypercube(10), 5), (lambda: gen.rmat(12, 16, permute=True), 8),
                                     (lambda: gen.lattice(80, 120, 0.6, seed=2), 6)])
-def test_bc(sg, make, k):
+@pytest.mark.parametrize("per_source", [False, True])
+def test_bc(sg, make, k, per_source):
+    """Default = source-batched (32 sources per graph launch); per_source = one BFS pair per source."""
     g = make()
     G = load(sg, g)
     srcs = gen.sources(g, k) if k < g.n else np.arange(g.n, dtype=np.int32)
-    bc, _ = sg.run_bc(G, srcs)
+    bc, _ = sg.run_bc(G, srcs, host_loop=per_source)
     assert bc_close(bc.cpu().numpy(), oracle.bc(g, srcs))
+
+
+def test_bc_batches_of_32_with_ragged_tail_and_duplicates(sg):
+    g = gen.lattice(60, 70, 0.7, seed=4)
+    G = load(sg, g)
+    srcs = np.concatenate([gen.sources(g, 70, stream=6), gen.sources(g, 3, stream=6)])   # 73 = 32+32+9, dups
+    bc, st = sg.run_bc(G, srcs)
+    assert bc_close(bc.cpu().numpy(), oracle.bc(g, srcs))
+    bc2, _ = sg.run_bc(G, srcs, host_loop=True)
+    assert bc_close(bc.cpu().numpy(), bc2.cpu().numpy(), 1e-12)
 
 
 def test_bc_sigma_beyond_fp64_range(sg):
