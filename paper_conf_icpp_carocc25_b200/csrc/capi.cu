@@ -476,7 +476,10 @@ struct Tiers {
     int32_t seg;   // destination-segmented hub tier for BFS: 0 off, 1 auto, 2 always
 };
 // auto mode: the segmented tier pays for its per-segment slice loads only on heavy supersteps
-static const unsigned long long kSegThreshold = 32ull << 20;   // estimated frontier arcs (m_f)
+#ifndef SG_SEG_THRESHOLD_M
+#define SG_SEG_THRESHOLD_M 32
+#endif
+static const unsigned long long kSegThreshold = (unsigned long long)SG_SEG_THRESHOLD_M << 20;   // est. frontier arcs
 
 static Tiers tiers_from(const sg_opts *o) {
     Tiers t{kDefaultHeavy, kDefaultSmall, 1};

@@ -2,10 +2,12 @@
 // weight) -> bool "whether dst should be added to the frontier"; algorithms P:161 §3.4).
 //
 // Split into ctx(src) (loaded once per source vertex), probe(dst) (the one random load per
-// arc; issued for several arcs before any decision so the loads overlap) and act(...)
-// (decision + atomics + insertion into the output 2LB).  The compute step of Listing 1
-// (dist[v] = iter + 1) is fused into act: the thread whose atomic inserts v
-// writes its value (the paper keeps it separate; on B200 the fused store saves a pass).
+// arc; issued for several arcs before any decision so the loads overlap) and act_batch<K>(...)
+// (decision + atomics + insertion into the output 2LB for K arcs at once: every atomic of the
+// batch is issued before any result is consumed, so a thread has K atomics in flight instead
+// of K round trips in series).  The compute step of Listing 1 (dist[v] = iter + 1,
+// P:178-181) is fused: the thread whose atomic inserts v writes its value (the paper keeps it
+// separate; on B200 the fused store saves a pass).
 #pragma once
 #include "common.cuh"
 
@@ -17,10 +19,30 @@ struct OutSink {
     __device__ __forceinline__ bool insert(int32_t v) const { return bits ? insert_2lb(bits, summ, v) : true; }
 };
 
+// Insert the flagged vertices into the output 2LB: all layer-1 atomics first, then the summary
+// bits of words that were empty.  flipped[k] = this call set v[k]'s bit.
+template <int K>
+__device__ __forceinline__ void insert_batch(const OutSink &out, const int32_t (&v)[K], const bool (&f)[K],
+                                             bool (&flipped)[K]) {
+    if (!out.bits) {
+#pragma unroll
+        for (int k = 0; k < K; k++) flipped[k] = f[k];
+        return;
+    }
+    unsigned long long old[K];
+#pragma unroll
+    for (int k = 0; k < K; k++) old[k] = f[k] ? atomic_or_u64(out.bits + (v[k] >> 6), 1ull << (v[k] & 63)) : ~0ull;
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        flipped[k] = f[k] && !((old[k] >> (v[k] & 63)) & 1ull);
+        if (f[k] && old[k] == 0ull) atomic_or_u64(out.summ + (v[k] >> 12), 1ull << ((v[k] >> 6) & 63));
+    }
+}
+
 // BFS (Listing 1 l.9-13 + l.14-17).  `visited` is updated live: the first thread whose
 // atomicOr sets v's visited bit owns v, writes level[v] and inserts v.  A stale probe only
 // costs one extra atomic.  Result = {v unvisited before the step with a neighbour in the
-// frontier}, identical to the frozen-visited reading.
+// frontier}, identical to the frozen-visited reading (R1).
 struct FnBfs {
     static constexpr bool kWeights = false;
     static constexpr bool kSeg = true;      // hubs may take the destination-segmented tier
@@ -34,12 +56,28 @@ struct FnBfs {
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t) const { return 0u; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return ld_word(visited + (v >> 6)); }
-    __device__ __forceinline__ void act(Ctx, int32_t v, uint32_t, Probe pr) const {
-        const uint64_t m = 1ull << (v & 63);
-        if (pr & m) return;
-        if (atomic_or_u64(visited + (v >> 6), m) & m) return;
-        (level_pp ? *level_pp : level)[v] = next_ptr ? *next_ptr : next;
-        out.insert(v);
+    template <int K>
+    __device__ __forceinline__ void act_batch(const Ctx (&)[K], const int32_t (&v)[K], const uint32_t (&)[K],
+                                              const Probe (&pr)[K], const bool (&ok)[K]) const {
+        bool cand[K], flip[K], done[K];
+        unsigned long long old[K];
+        bool any = false;
+#pragma unroll
+        for (int k = 0; k < K; k++) cand[k] = ok[k] && !((pr[k] >> (v[k] & 63)) & 1ull);
+#pragma unroll
+        for (int k = 0; k < K; k++) old[k] = cand[k] ? atomic_or_u64(visited + (v[k] >> 6), 1ull << (v[k] & 63)) : ~0ull;
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            flip[k] = cand[k] && !((old[k] >> (v[k] & 63)) & 1ull);
+            any |= flip[k];
+        }
+        if (!any) return;
+        uint32_t *lv = level_pp ? *level_pp : level;
+        const uint32_t nx = next_ptr ? *next_ptr : next;
+#pragma unroll
+        for (int k = 0; k < K; k++)
+            if (flip[k]) lv[v[k]] = nx;
+        insert_batch(out, v, flip, done);
     }
 };
 
@@ -54,11 +92,21 @@ struct FnSssp {
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return *(volatile uint32_t *)(dist + u); }
     __device__ __forceinline__ Probe probe(int32_t v) const { return dist[v]; }
-    __device__ __forceinline__ void act(Ctx du, int32_t v, uint32_t w, Probe pr) const {
-        if (du == INF32) return;
-        const uint32_t nd = du + w;
-        if (nd >= pr) return;
-        if (atomicMin(dist + v, nd) > nd) out.insert(v);
+    template <int K>
+    __device__ __forceinline__ void act_batch(const Ctx (&du)[K], const int32_t (&v)[K], const uint32_t (&w)[K],
+                                              const Probe (&pr)[K], const bool (&ok)[K]) const {
+        uint32_t nd[K], old[K];
+        bool cand[K], imp[K], done[K];
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            nd[k] = du[k] + w[k];
+            cand[k] = ok[k] && du[k] != INF32 && nd[k] < pr[k];
+        }
+#pragma unroll
+        for (int k = 0; k < K; k++) old[k] = cand[k] ? atomicMin(dist + v[k], nd[k]) : 0u;
+#pragma unroll
+        for (int k = 0; k < K; k++) imp[k] = cand[k] && old[k] > nd[k];
+        insert_batch(out, v, imp, done);
     }
 };
 
@@ -73,9 +121,18 @@ struct FnCc {
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return *(volatile int32_t *)(label + u); }
     __device__ __forceinline__ Probe probe(int32_t v) const { return label[v]; }
-    __device__ __forceinline__ void act(Ctx lu, int32_t v, uint32_t, Probe pr) const {
-        if (lu >= pr) return;
-        if (atomicMin(label + v, lu) > lu) out.insert(v);
+    template <int K>
+    __device__ __forceinline__ void act_batch(const Ctx (&lu)[K], const int32_t (&v)[K], const uint32_t (&)[K],
+                                              const Probe (&pr)[K], const bool (&ok)[K]) const {
+        int32_t old[K];
+        bool cand[K], imp[K], done[K];
+#pragma unroll
+        for (int k = 0; k < K; k++) cand[k] = ok[k] && lu[k] < pr[k];
+#pragma unroll
+        for (int k = 0; k < K; k++) old[k] = cand[k] ? atomicMin(label + v[k], lu[k]) : 0;
+#pragma unroll
+        for (int k = 0; k < K; k++) imp[k] = cand[k] && old[k] > lu[k];
+        insert_batch(out, v, imp, done);
     }
 };
 
@@ -94,10 +151,19 @@ struct FnBcSigma {
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return sigma[u]; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return __ldg(visited + (v >> 6)); }
-    __device__ __forceinline__ void act(Ctx su, int32_t v, uint32_t, Probe pr) const {
-        if (pr & (1ull << (v & 63))) return;
-        atomicAdd(sigma + v, su);
-        if (out.insert(v)) level[v] = next;
+    template <int K>
+    __device__ __forceinline__ void act_batch(const Ctx (&su)[K], const int32_t (&v)[K], const uint32_t (&)[K],
+                                              const Probe (&pr)[K], const bool (&ok)[K]) const {
+        bool cand[K], flip[K];
+#pragma unroll
+        for (int k = 0; k < K; k++) cand[k] = ok[k] && !((pr[k] >> (v[k] & 63)) & 1ull);
+#pragma unroll
+        for (int k = 0; k < K; k++)
+            if (cand[k]) atomicAdd(sigma + v[k], su[k]);
+        insert_batch(out, v, cand, flip);
+#pragma unroll
+        for (int k = 0; k < K; k++)
+            if (flip[k]) level[v[k]] = next;
     }
 };
 

@@ -75,9 +75,12 @@ __device__ __forceinline__ void warp_expand(const GraphView &g, const F &f, int6
         if (lane < a - s) i = s + lane;
         else if (lane >= 4 && lane - 4 < e - b) i = b + (lane - 4);
         if (i >= 0) {
-            const int32_t v = __ldg(g.col + i);
-            const uint32_t w = load_w<F>(g, i);
-            f.act(c, v, w, f.probe(v));
+            const int32_t v[1] = {__ldg(g.col + i)};
+            const uint32_t w[1] = {load_w<F>(g, i)};
+            const typename F::Probe pr[1] = {f.probe(v[0])};
+            const typename F::Ctx cc[1] = {c};
+            const bool ok[1] = {true};
+            f.act_batch(cc, v, w, pr, ok);
         }
     }
     for (int64_t i = a + 4 * lane; i < b; i += 256) {
@@ -90,19 +93,18 @@ __device__ __forceinline__ void warp_expand(const GraphView &g, const F &f, int6
             w0 = __ldg(reinterpret_cast<const uint32_t *>(g.w + i));
             if (two) w1 = __ldg(reinterpret_cast<const uint32_t *>(g.w + i + 128));
         }
-        typename F::Probe p0 = f.probe(v0.x), p1 = f.probe(v0.y), p2 = f.probe(v0.z), p3 = f.probe(v0.w);
-        typename F::Probe q0{}, q1{}, q2{}, q3{};
-        if (two) { q0 = f.probe(v1.x); q1 = f.probe(v1.y); q2 = f.probe(v1.z); q3 = f.probe(v1.w); }
-        f.act(c, v0.x, w0 & 0xff, p0);
-        f.act(c, v0.y, (w0 >> 8) & 0xff, p1);
-        f.act(c, v0.z, (w0 >> 16) & 0xff, p2);
-        f.act(c, v0.w, w0 >> 24, p3);
-        if (two) {
-            f.act(c, v1.x, w1 & 0xff, q0);
-            f.act(c, v1.y, (w1 >> 8) & 0xff, q1);
-            f.act(c, v1.z, (w1 >> 16) & 0xff, q2);
-            f.act(c, v1.w, w1 >> 24, q3);
+        const int32_t v[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+        const uint32_t w[8] = {w0 & 0xff, (w0 >> 8) & 0xff, (w0 >> 16) & 0xff, w0 >> 24,
+                               w1 & 0xff, (w1 >> 8) & 0xff, (w1 >> 16) & 0xff, w1 >> 24};
+        const bool ok[8] = {true, true, true, true, two, two, two, two};
+        typename F::Probe pr[8];
+        typename F::Ctx cc[8];
+#pragma unroll
+        for (int k = 0; k < 8; k++) {
+            pr[k] = ok[k] ? f.probe(v[k]) : typename F::Probe{};
+            cc[k] = c;
         }
+        f.act_batch(cc, v, w, pr, ok);
     }
 }
 
@@ -212,26 +214,26 @@ __device__ __forceinline__ unsigned long long push_word(const PushParams &p, con
             const int k1 = kb + __popcll(mask & ((2ull << (lane + 32)) - 1ull));
             const uint32_t e0 = base + lane, e1 = base + 32 + lane;
             const bool ok0 = e0 < total, ok1 = e1 < total;
-            int32_t v0 = 0, v1 = 0;
-            uint32_t w0 = 0, w1 = 0;
-            typename F::Ctx c0{}, c1{};
+            int32_t v[2] = {0, 0};
+            uint32_t w[2] = {0u, 0u};
+            typename F::Ctx cc[2] = {};
+            const bool ok[2] = {ok0, ok1};
             if (ok0) {
                 const int64_t i = sm.start[k0] + (e0 - sm.pre[k0]);
-                v0 = __ldg(p.g.col + i);
-                w0 = load_w<F>(p.g, i);
-                c0 = sm.ctx[k0];
+                v[0] = __ldg(p.g.col + i);
+                w[0] = load_w<F>(p.g, i);
+                cc[0] = sm.ctx[k0];
             }
             if (ok1) {
                 const int64_t i = sm.start[k1] + (e1 - sm.pre[k1]);
-                v1 = __ldg(p.g.col + i);
-                w1 = load_w<F>(p.g, i);
-                c1 = sm.ctx[k1];
+                v[1] = __ldg(p.g.col + i);
+                w[1] = load_w<F>(p.g, i);
+                cc[1] = sm.ctx[k1];
             }
-            typename F::Probe p0{}, p1{};
-            if (ok0) p0 = f.probe(v0);
-            if (ok1) p1 = f.probe(v1);
-            if (ok0) f.act(c0, v0, w0, p0);
-            if (ok1) f.act(c1, v1, w1, p1);
+            typename F::Probe pr[2] = {};
+            if (ok0) pr[0] = f.probe(v[0]);
+            if (ok1) pr[1] = f.probe(v[1]);
+            f.act_batch(cc, v, w, pr, ok);
             kb += __popcll(mask);
         }
         __syncwarp();
@@ -336,24 +338,27 @@ __global__ void __launch_bounds__(HEAVY_THREADS) k_push_heavy(PushParams p, F f)
         const typename F::Ctx c = f.ctx(it.u);
         mbar_wait(bar + s, phase);
         const int32_t *src = buf + (size_t)s * HEAVY_BUF_INTS + (it.begin & 3);
-        for (int i = threadIdx.x; i < it.len; i += HEAVY_THREADS * 4) {
-            int32_t v[4];
-            uint32_t w[4];
-            bool ok[4];
-            typename F::Probe pr[4];
+        // all HEAVY_CHUNK / HEAVY_THREADS arcs of a thread in one batch: their probes and then
+        // their atomics are all in flight together
+        constexpr int KH = HEAVY_CHUNK / HEAVY_THREADS;
+        {
+            const int i = threadIdx.x;
+            int32_t v[KH];
+            uint32_t w[KH];
+            bool ok[KH];
+            typename F::Probe pr[KH];
+            typename F::Ctx cc[KH];
 #pragma unroll
-            for (int k = 0; k < 4; k++) {
+            for (int k = 0; k < KH; k++) {
                 const int ii = i + k * HEAVY_THREADS;
                 ok[k] = ii < it.len;
                 v[k] = ok[k] ? src[ii] : 0;
                 w[k] = ok[k] ? load_w<F>(p.g, it.begin + ii) : 0u;
+                cc[k] = c;
             }
 #pragma unroll
-            for (int k = 0; k < 4; k++)
-                if (ok[k]) pr[k] = f.probe(v[k]);
-#pragma unroll
-            for (int k = 0; k < 4; k++)
-                if (ok[k]) f.act(c, v[k], w[k], pr[k]);
+            for (int k = 0; k < KH; k++) pr[k] = ok[k] ? f.probe(v[k]) : typename F::Probe{};
+            f.act_batch(cc, v, w, pr, ok);
         }
         __syncthreads();   // buffer s fully consumed
         if (threadIdx.x == 0 && j + HEAVY_STAGES < my_n) {
