@@ -470,6 +470,45 @@ SG_API int frontier_or_into(const sg_frontier *f, uint64_t *dst, void *stream) {
 }  // extern "C"
 
 // ------------------------------------------------------------------------------------------
+// L2 residency for the array every arc probes (CC labels): a persisting access-policy window on
+// the stream for the duration of a run_* call, so the col_idx stream does not evict it (B200:
+// 126 MB L2, 82.9 MB persisting carve-out).  Measured on config 3 it is SLOWER (18.2 vs 13.0 ms:
+// the carve-out shrinks the L2 left for everything else), so it is opt-in (SG_L2PIN=1) and kept
+// for the record.  Best effort: errors ignored.
+struct L2Pin {
+    cudaStream_t s;
+    bool on = false;
+    L2Pin(const void *p, size_t bytes, cudaStream_t st) : s(st) {
+        if (!getenv("SG_L2PIN")) return;
+        int dev = 0, maxp = 0, maxw = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess) return;
+        cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
+        cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+        if (maxp <= 0 || maxw <= 0 || !p || !bytes) return;
+        size_t limit = 0;
+        cudaDeviceGetLimit(&limit, cudaLimitPersistingL2CacheSize);
+        if (limit < (size_t)maxp) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp);
+        cudaStreamAttrValue a = {};
+        a.accessPolicyWindow.base_ptr = const_cast<void *>(p);
+        a.accessPolicyWindow.num_bytes = bytes < (size_t)maxw ? bytes : (size_t)maxw;
+        const double ratio = (double)maxp / (double)a.accessPolicyWindow.num_bytes;
+        a.accessPolicyWindow.hitRatio = (float)(ratio < 1.0 ? ratio : 1.0);
+        a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        a.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        on = cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &a) == cudaSuccess;
+        cudaGetLastError();
+    }
+    ~L2Pin() {
+        if (!on) return;
+        cudaStreamAttrValue a = {};
+        a.accessPolicyWindow.num_bytes = 0;
+        cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &a);
+        cudaCtxResetPersistingL2Cache();
+        cudaGetLastError();
+    }
+};
+
+// ------------------------------------------------------------------------------------------
 // superstep helpers
 struct Tiers {
     int32_t heavy, small;
@@ -970,25 +1009,36 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
+    L2Pin pin(label, sizeof(int32_t) * (size_t)G.n, s);   // labels are probed once per arc: keep them in L2
     CK(cudaEventRecord(ws->ev0, s));
     launch_iota_i32(label, G.n, s);
     sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
     launch_fill_all(in->bits, in->summ, G.n, G.nw1, G.nw2, s);    // advance::vertices
     TRY(clear_frontier(out, s));
-    TRY(compact(g, in, false, s));
+    TRY(compact(g, in, true, s));
     TRY(read_stats(ws, s));
-    int64_t iters = 0, arcs = 0;
+    int64_t iters = 0, push_steps = 0, pull_steps = 0, arcs_pushed = 0, arcs_pulled = 0;
     int in_idx = 0;
     for (;;) {
         const int64_t count = (int64_t)ws->h_st[in_idx].count;
         if (count == 0) break;
         if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
-        const PushLaunch L = push_launch(g, in, t, count);
-        launch_push_cc(L, CcArgs{label, out->bits, out->summ}, s);
+        // direction: a dense superstep (frontier arcs > nnz/4) pulls — every vertex takes the min of
+        // its neighbours' labels without atomics; a sparse one pushes from the changed vertices
+        const bool pull = o.direction == SG_DIR_PULL ||
+                          (o.direction == SG_DIR_AUTO && (double)ws->h_st[in_idx].mf * 4.0 > (double)G.nnz);
+        if (pull) {
+            launch_pull_cc(G, label, out->bits, out->summ, in->st, s);
+            pull_steps++;
+        } else {
+            const PushLaunch L = push_launch(g, in, t, count);
+            launch_push_cc(L, CcArgs{label, out->bits, out->summ}, s);
+            push_steps++;
+        }
         TRY(clear_frontier(in, s));
-        TRY(compact(g, out, false, s));
+        TRY(compact(g, out, true, s));
         TRY(read_stats(ws, s));
-        arcs += (int64_t)ws->h_st[in_idx].arcs;
+        (pull ? arcs_pulled : arcs_pushed) += (int64_t)ws->h_st[in_idx].arcs;
         std::swap(in, out);
         in_idx ^= 1;
         iters++;
@@ -1001,8 +1051,10 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     if (stats) {
         memset(stats, 0, sizeof *stats);
         stats->iterations = iters;
-        stats->push_steps = iters;
-        stats->arcs_pushed = arcs;
+        stats->push_steps = push_steps;
+        stats->pull_steps = pull_steps;
+        stats->arcs_pushed = arcs_pushed;
+        stats->arcs_pulled = arcs_pulled;
         stats->reached = G.n;
         stats->device_ms = ms;
     }

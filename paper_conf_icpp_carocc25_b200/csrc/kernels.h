@@ -76,6 +76,10 @@ void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visi
                      uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
                      const uint32_t *next_ptr = nullptr, uint32_t *const *level_pp = nullptr);
 
+// pull_cc.cu — pull label-propagation step (dense CC supersteps)
+void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,
+                    cudaStream_t s);
+
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
                        unsigned long long h_push, unsigned long long h_pull, int first, cudaStream_t s);

@@ -336,8 +336,20 @@ def test_cc_tiers(sg):
     G = load(sg, g)
     ref = oracle.cc(g)
     for opts in (dict(heavy_degree=1), dict(small_degree=-1), dict(small_degree=100000, heavy_degree=100000)):
-        lab, _ = sg.run_cc(G, **opts)
+        lab, _ = sg.run_cc(G, direction=sg.SG_DIR_PUSH, **opts)
         assert np.array_equal(lab.cpu().numpy(), ref)
+
+
+@pytest.mark.parametrize("make", [lambda: gen.gnm(200_000, 1_000_000), lambda: gen.rmat(14, 8, permute=True),
+                                  lambda: gen.lattice(200, 300, 0.55), lambda: gen.gnm(100_003, 40_000, seed=7)])
+def test_cc_directions_agree(sg, make):
+    """push-only, pull-only and auto (pull on dense supersteps) reach the same min labels."""
+    g = make()
+    G = load(sg, g)
+    ref = oracle.cc(g)
+    for d in (sg.SG_DIR_PUSH, sg.SG_DIR_PULL, sg.SG_DIR_AUTO):
+        lab, st = sg.run_cc(G, direction=d)
+        assert np.array_equal(lab.cpu().numpy(), ref), d
 
 
 # -------------------------------------------------------------------------------- BC
