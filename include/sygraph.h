@@ -122,6 +122,27 @@ SG_API int frontier_op(sg_frontier *dst, const sg_frontier *src, int op, void *s
 /* OR the layer-1 words of f into a plain bitmap `dst` (ceil(n/64) words). Async. */
 SG_API int frontier_or_into(const sg_frontier *f, uint64_t *dst, void *stream);
 
+/* ---- filter / compute (Table 2, §3.1) ---------------------------------- */
+/* The paper's Filter / Compute functors are C++ lambdas; across this ABI they are a predicate /
+ * operation code with parameters.  Predicates on vertex v (a, b are doubles):
+ *   SG_PRED_DEGREE_RANGE  a <= deg(v) < b               (array unused)
+ *   SG_PRED_U32_RANGE     a <= ((uint32*)array)[v] < b   (device array[n])
+ *   SG_PRED_I32_RANGE     a <= ((int32*)array)[v] < b
+ *   SG_PRED_F64_RANGE     a <= ((double*)array)[v] < b
+ *   SG_PRED_IN_BITMAP     bit v of the layer-1-shaped device bitmap `array`                  */
+enum { SG_PRED_DEGREE_RANGE = 0, SG_PRED_U32_RANGE = 1, SG_PRED_I32_RANGE = 2, SG_PRED_F64_RANGE = 3,
+       SG_PRED_IN_BITMAP = 4 };
+/* filter::inplace(G, F, pred) when out == NULL: removes failing elements from `in`; a word that
+ * becomes 0 resets its layer-2 bit.  filter::external(G, In, Out, pred) otherwise:
+ * passing elements are inserted into `out` (not cleared first).  Async. */
+SG_API int frontier_filter(sg_frontier *in, sg_frontier *out, int pred, const void *array, double a, double b,
+                           void *stream);
+/* compute::execute(G, F, op): for every active v:
+ *   SG_OP_SET_U32 / SG_OP_SET_I32 / SG_OP_SET_F64: array[v] = value
+ *   SG_OP_ADD_U32 / SG_OP_ADD_F64:                 array[v] += value      (device array[n]). Async. */
+enum { SG_OP_SET_U32 = 0, SG_OP_SET_I32 = 1, SG_OP_SET_F64 = 2, SG_OP_ADD_U32 = 3, SG_OP_ADD_F64 = 4 };
+SG_API int compute_execute(const sg_frontier *f, int op, void *array, double value, void *stream);
+
 /* ---- advance (Table 2; §4.2-4.3) ----------------------------------- */
 /* One push advance superstep: compacts the summary layer of `in` into the offsets buffer
  * (P:255), then expands every active vertex's adjacency with the degree-tiered load balance,

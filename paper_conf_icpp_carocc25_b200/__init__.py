@@ -74,7 +74,10 @@ K_NAMES = ["compact", "stats", "advance_push", "advance_pull", "bc"]
 EXPORTS = ["graph_load_csr", "graph_free", "graph_info", "frontier_init", "frontier_free", "frontier_insert",
            "frontier_fill_all", "frontier_clear", "frontier_count", "frontier_view", "frontier_op",
            "frontier_or_into", "advance", "run_bfs", "run_sssp", "run_cc", "run_bc", "sg_opts_default",
-           "sg_last_error", "sg_version", "sg_profile", "sg_profile_read", "sg_launch_count"]
+           "sg_last_error", "sg_version", "sg_profile", "sg_profile_read", "sg_launch_count", "frontier_filter",
+           "compute_execute"]
+SG_PRED_DEGREE_RANGE, SG_PRED_U32_RANGE, SG_PRED_I32_RANGE, SG_PRED_F64_RANGE, SG_PRED_IN_BITMAP = 0, 1, 2, 3, 4
+SG_OP_SET_U32, SG_OP_SET_I32, SG_OP_SET_F64, SG_OP_ADD_U32, SG_OP_ADD_F64 = 0, 1, 2, 3, 4
 
 _lib = None
 
@@ -113,6 +116,8 @@ def load():
         "sg_profile": (c_int, [vp, c_int]),
         "sg_profile_read": (c_int, [vp, ctypes.POINTER(SgKprof)]),
         "sg_launch_count": (i64, []),
+        "frontier_filter": (c_int, [vp, vp, c_int, vp, ctypes.c_double, ctypes.c_double, vp]),
+        "compute_execute": (c_int, [vp, c_int, vp, ctypes.c_double, vp]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -263,6 +268,19 @@ def frontier_view(f: Frontier):
 
 def frontier_op(dst: Frontier, src: Frontier, op: int, stream=None):
     _check(load().frontier_op(dst.handle, src.handle, op, _stream_ptr(stream)))
+
+
+def frontier_filter(fin: Frontier, fout: Frontier | None, pred: int, array=None, a: float = 0.0, b: float = 0.0,
+                    stream=None):
+    """filter::inplace (fout None) / filter::external (Table 2) with a SG_PRED_* predicate."""
+    _check(load().frontier_filter(fin.handle, fout.handle if fout is not None else None, pred,
+                                  array.data_ptr() if array is not None else None, float(a), float(b),
+                                  _stream_ptr(stream)))
+
+
+def compute_execute(f: Frontier, op: int, array, value: float, stream=None):
+    """compute::execute (Table 2): SG_OP_* applied to array[v] for every active v."""
+    _check(load().compute_execute(f.handle, op, array.data_ptr(), float(value), _stream_ptr(stream)))
 
 
 def frontier_or_into(f: Frontier, dst, stream=None):

@@ -460,6 +460,29 @@ SG_API int frontier_op(sg_frontier *dst, const sg_frontier *src, int op, void *s
     return SG_OK;
 }
 
+SG_API int frontier_filter(sg_frontier *in, sg_frontier *out, int pred, const void *array, double a, double b,
+                           void *stream) {
+    t_err.clear();
+    if (!in || pred < SG_PRED_DEGREE_RANGE || pred > SG_PRED_IN_BITMAP) return fail(SG_ERR_INVALID, "bad filter arguments");
+    if (pred != SG_PRED_DEGREE_RANGE && !array) return fail(SG_ERR_INVALID, "predicate needs an array");
+    if (out && out->g->v.n != in->g->v.n) return fail(SG_ERR_INVALID, "frontiers of different graphs");
+    const GraphView &g = in->g->v;
+    if (out && out != in)
+        launch_filter(g, in->bits, out->bits, out->summ, pred, array, a, b, 0, (cudaStream_t)stream);
+    else
+        launch_filter(g, in->bits, in->bits, in->summ, pred, array, a, b, 1, (cudaStream_t)stream);
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
+SG_API int compute_execute(const sg_frontier *f, int op, void *array, double value, void *stream) {
+    t_err.clear();
+    if (!f || !array || op < SG_OP_SET_U32 || op > SG_OP_ADD_F64) return fail(SG_ERR_INVALID, "bad compute arguments");
+    launch_compute(f->g->v, f->bits, op, array, value, (cudaStream_t)stream);
+    CK(cudaGetLastError());
+    return SG_OK;
+}
+
 SG_API int frontier_or_into(const sg_frontier *f, uint64_t *dst, void *stream) {
     if (!f || !dst) return fail(SG_ERR_INVALID, "NULL argument");
     launch_or_all(f->bits, f->g->v.nw1, dst, (cudaStream_t)stream);

@@ -76,6 +76,11 @@ void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visi
                      uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
                      const uint32_t *next_ptr = nullptr, uint32_t *const *level_pp = nullptr);
 
+// filter.cu — filter::inplace / external, compute::execute (Table 2)
+void launch_filter(const GraphView &g, const uint64_t *in_bits, uint64_t *out_bits, uint64_t *out_summ, int pred,
+                   const void *array, double a, double b, int inplace, cudaStream_t s);
+void launch_compute(const GraphView &g, const uint64_t *bits, int op, void *array, double value, cudaStream_t s);
+
 // pull_cc.cu — pull label-propagation step (dense CC supersteps)
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,
                     cudaStream_t s);
