@@ -77,7 +77,10 @@ typedef struct {
                                  0 = one CUDA graph with device-side control (default) */
     int32_t segmented;        /* BFS hub tier with the visited slice in shared memory:
                                  0 = auto (heavy supersteps), 1 = off, 2 = always */
-    int32_t reserved[6];
+    int32_t one_layer;        /* ablation (Fig. 7): 1 = push visits every layer-1 word (plain bitmap,
+                                 no summary-layer compaction); host-driven loop only */
+    int32_t coarsening;       /* push: layer-1 words per warp grab (CF); 0 = auto */
+    int32_t reserved[4];
 } sg_opts;
 
 typedef struct {

@@ -82,6 +82,7 @@ struct Workspace {
     DevStats *st = nullptr;        // 2 contiguous control blocks (fr[0].st, fr[1].st)
     DevStats *h_st = nullptr;      // pinned host mirror
     uint64_t *visited = nullptr;   // nw1 words
+    uint32_t *all_offsets = nullptr;   // one-layer ablation: identity word list
     HeavyItem *heavy = nullptr;
     uint32_t heavy_cap = 0;
     int32_t heavy_deg = 0;
@@ -98,7 +99,7 @@ struct Workspace {
     cudaGraph_t bfs_graph = nullptr;
     cudaGraphExec_t bfs_exec = nullptr;
     uint32_t *bfs_level = nullptr;
-    int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1;
+    int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1, bfs_cf = -1;
     SegItem *seg = nullptr;        // destination-segmented hub queue (BFS)
     uint32_t seg_cap = 0;
     // source-batched BC (bcb.cu)
@@ -154,9 +155,9 @@ static int ensure_ws(sg_graph *g) {
     if (g->ws) return SG_OK;
     Workspace *ws = new Workspace();
     g->ws = ws;
-    CK(cudaMalloc(&ws->st, 2 * sizeof(DevStats)));
-    CK(cudaMemset(ws->st, 0, 2 * sizeof(DevStats)));
-    CK(cudaMallocHost(&ws->h_st, 2 * sizeof(DevStats)));
+    CK(cudaMalloc(&ws->st, 3 * sizeof(DevStats)));   // fr[0], fr[1], one-layer ablation list
+    CK(cudaMemset(ws->st, 0, 3 * sizeof(DevStats)));
+    CK(cudaMallocHost(&ws->h_st, 3 * sizeof(DevStats)));
     for (int i = 0; i < 2; i++) {
         TRY(alloc_frontier_bufs(&ws->fr[i], g, false));
         ws->fr[i].st = ws->st + i;
@@ -198,6 +199,7 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->visited);
     cudaFree(ws->heavy);
     cudaFree(ws->seg);
+    cudaFree(ws->all_offsets);
     cudaFree(ws->scratch);
     cudaFreeHost(ws->h_scratch);
     cudaFree(ws->stack);
@@ -536,6 +538,7 @@ struct L2Pin {
 struct Tiers {
     int32_t heavy, small;
     int32_t seg;   // destination-segmented hub tier for BFS: 0 off, 1 auto, 2 always
+    int32_t cf;    // words per warp grab (coarsening factor); 0 = auto
 };
 // auto mode: the segmented tier pays for its per-segment slice loads only on heavy supersteps
 #ifndef SG_SEG_THRESHOLD_M
@@ -544,7 +547,8 @@ struct Tiers {
 static const unsigned long long kSegThreshold = (unsigned long long)SG_SEG_THRESHOLD_M << 20;   // est. frontier arcs
 
 static Tiers tiers_from(const sg_opts *o) {
-    Tiers t{kDefaultHeavy, kDefaultSmall, 1};
+    Tiers t{kDefaultHeavy, kDefaultSmall, 1, 0};
+    if (o && o->coarsening > 0) t.cf = o->coarsening > 64 ? 64 : o->coarsening;
     if (o && o->heavy_degree > 0) t.heavy = o->heavy_degree;
     if (o && o->small_degree > 0) t.small = o->small_degree;
     if (o && o->small_degree < 0) t.small = 0;           // no thread tier
@@ -586,6 +590,13 @@ static PushLaunch push_launch(const sg_graph *g, const sg_frontier *in, Tiers t,
         if (gw > maxg) gw = maxg;
         L.grid_words = (int)gw;
     }
+    if (t.cf > 0) {
+        L.batch = t.cf;
+        if (count_hint >= 0) {
+            int64_t gw = (count_hint + 8 * L.batch - 1) / (8 * L.batch);
+            L.grid_words = (int)(gw < 1 ? 1 : (gw > maxg ? maxg : gw));
+        }
+    }
     L.grid_heavy = push_max_grid_heavy();
     L.seg = g->ws->seg;
     L.seg_cap = g->ws->seg_cap;
@@ -595,7 +606,7 @@ static PushLaunch push_launch(const sg_graph *g, const sg_frontier *in, Tiers t,
 }
 
 static int read_stats(Workspace *ws, cudaStream_t s) {
-    CK(cudaMemcpyAsync(ws->h_st, ws->st, 2 * sizeof(DevStats), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(ws->h_st, ws->st, 3 * sizeof(DevStats), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     CK(cudaGetLastError());
     return SG_OK;
@@ -774,7 +785,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         TRY(add_cond(body, deps, h_push[half], cudaGraphCondTypeIf, &n_push, &b_push));
         TRY(add_cond(body, deps, h_pull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
         PushLaunch L = push_launch(g, in, t, -1);
-        L.batch = 0;   // coarsening factor computed on the device from the count
+        L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
         BfsArgs a{ws->visited, nullptr, 0u, out->bits, out->summ, &ws->ctrl->next, &ws->ctrl->level};
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
@@ -794,6 +805,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     ws->bfs_heavy = t.heavy;
     ws->bfs_small = t.small;
     ws->bfs_seg = t.seg;
+    ws->bfs_cf = t.cf;
     return SG_OK;
 }
 
@@ -801,7 +813,8 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
                          sg_stats *stats) {
     Workspace *ws = g->ws;
     cudaStream_t s = stream_of(&o);
-    if (!ws->bfs_exec || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small || ws->bfs_seg != t.seg)
+    if (!ws->bfs_exec || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small || ws->bfs_seg != t.seg ||
+        ws->bfs_cf != t.cf)
         TRY(build_bfs_graph(g, t));
     BfsCtrl &c = *ws->h_ctrl;
     memset(&c, 0, sizeof c);
@@ -863,7 +876,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
-    if (!ws->prof.on && !o.host_loop) return run_bfs_graph(g, src, level, o, t, max_iters, stats);
+    if (!ws->prof.on && !o.host_loop && !o.one_layer) return run_bfs_graph(g, src, level, o, t, max_iters, stats);
     CK(cudaEventRecord(ws->ev0, s));
     CK(cudaMemsetAsync(level, 0xFF, sizeof(uint32_t) * (size_t)G.n, s));
     launch_set_u32(level, src, 0u, s);
@@ -903,7 +916,13 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
             launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, level, d + 1, in->st, s);
             pull_steps++;
         } else {
-            const PushLaunch L = push_launch(g, in, t, count);
+            PushLaunch L = push_launch(g, in, t, o.one_layer ? G.nw1 : count);
+            if (o.one_layer) {   // Fig. 7 ablation: no summary layer, every word is visited
+                if (!ws->all_offsets) CK(cudaMalloc(&ws->all_offsets, sizeof(uint32_t) * (size_t)G.nw1));
+                launch_list_all(ws->all_offsets, ws->st + 2, in->st, G.nw1, s);
+                L.offsets = ws->all_offsets;
+                L.st = ws->st + 2;
+            }
             launch_push_bfs(L, BfsArgs{ws->visited, level, d + 1, out->bits, out->summ}, s);
             push_steps++;
         }
@@ -931,7 +950,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
             prof_bytes(ws, pc, 8.0 * (double)G.nw2 + 12.0 * c_out + 16.0 * n_new);
         }
         if (pull) arcs_pulled += (int64_t)ws->h_st[in_idx].arcs;
-        else arcs_pushed += (int64_t)ws->h_st[in_idx].arcs;
+        else arcs_pushed += (int64_t)ws->h_st[o.one_layer ? 2 : in_idx].arcs;
         if (trace)
             fprintf(stderr, "[sygraph bfs] level %u %s in: words %lld n_f %lld m_f~%lld | arcs %llu | out: n_f %llu\n", d,
                     pull ? "pull" : "push", (long long)count, (long long)nf, (long long)mf,

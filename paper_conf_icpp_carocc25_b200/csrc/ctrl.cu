@@ -72,6 +72,26 @@ __global__ void k_clear_listed(uint64_t *__restrict__ bits, uint64_t *__restrict
     if (zero_st && t < (int64_t)(sizeof(DevStats) / 8)) reinterpret_cast<unsigned long long *>(zero_st)[t] = 0ull;
 }
 
+// One-layer ablation: the offsets list names every layer-1 word (count = nw1), the control
+// block's other fields are reset and m_f is copied from the compacted frontier.
+__global__ void k_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *st_src, int64_t nw1) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    for (int64_t w = t; w < nw1; w += stride) offsets[w] = (uint32_t)w;
+    if (t == 0) {
+        st_all->count = (unsigned long long)nw1;
+        st_all->nf = st_src->nf;
+        st_all->mf = st_src->mf;
+        st_all->arcs = st_all->batch = st_all->heavy_count = st_all->seg_count = st_all->pad = 0ull;
+    }
+}
+void launch_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *st_src, int64_t nw1, cudaStream_t s) {
+    int64_t blocks = (nw1 + 255) / 256;
+    if (blocks > 148 * 8) blocks = 148 * 8;
+    note_launch();
+    k_list_all<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(offsets, st_all, st_src, nw1);
+}
+
 __global__ void k_zero_u64(unsigned long long *p, int64_t n) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += stride) p[i] = 0ull;

@@ -93,6 +93,7 @@ void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s);
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s);
 void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s);
+void launch_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *st_src, int64_t nw1, cudaStream_t s);
 
 // bcb.cu — source-batched BC (32 sources per batch): init, cooperative forward and backward
 // kernels (grid-wide barriers between supersteps), reset

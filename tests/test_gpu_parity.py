@@ -139,6 +139,18 @@ def test_bfs_tier_forcing_invariant(sg, opts):
         assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (opts, s)
 
 
+@pytest.mark.parametrize("kw", [dict(one_layer=True), dict(one_layer=True, coarsening=1, small_degree=-1),
+                                dict(coarsening=7), dict(coarsening=1, heavy_degree=1 << 30)])
+def test_bfs_ablation_knobs_do_not_change_results(sg, kw):
+    """Fig. 7 ablation switches (plain one-layer bitmap, coarsening factor) keep levels exact."""
+    g = gen.rmat(15, 12)
+    G = load(sg, g)
+    for s in gen.sources(g, 3):
+        for d in (sg.SG_DIR_PUSH, sg.SG_DIR_AUTO):
+            lv, _ = sg.run_bfs(G, int(s), direction=d, host_loop=True, **kw)
+            assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (kw, d)
+
+
 @pytest.mark.parametrize("host_loop", [False, True])
 @pytest.mark.parametrize("make", [lambda: gen.rmat(14, 16, permute=True), lambda: gen.rmat(21, 8, permute=True),
                                   lambda: gen.rmat(20, 16)])
