@@ -80,7 +80,9 @@ typedef struct {
     int32_t one_layer;        /* ablation (Fig. 7): 1 = push visits every layer-1 word (plain bitmap,
                                  no summary-layer compaction); host-driven loop only */
     int32_t coarsening;       /* push: layer-1 words per warp grab (CF); 0 = auto */
-    int32_t reserved[4];
+    int32_t sssp_delta;       /* run_sssp: 0 = frontier Bellman-Ford (the paper); D > 0 = near-far
+                                 delta-stepping with bucket width D (P:161 refs [23,34]) */
+    int32_t reserved[3];
 } sg_opts;
 
 typedef struct {

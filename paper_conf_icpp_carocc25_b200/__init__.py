@@ -34,7 +34,8 @@ class SgOpts(ctypes.Structure):
     _fields_ = [("stream", ctypes.c_void_p), ("direction", ctypes.c_int), ("alpha", ctypes.c_double),
                 ("beta", ctypes.c_double), ("max_iters", ctypes.c_int64), ("heavy_degree", ctypes.c_int32),
                 ("small_degree", ctypes.c_int32), ("host_loop", ctypes.c_int32), ("segmented", ctypes.c_int32),
-                ("one_layer", ctypes.c_int32), ("coarsening", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
+                ("one_layer", ctypes.c_int32), ("coarsening", ctypes.c_int32), ("sssp_delta", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 3)]
 
 
 class SgStats(ctypes.Structure):
@@ -154,7 +155,7 @@ def _ptr_mem(a):
 
 
 def opts(stream=None, direction=SG_DIR_AUTO, alpha=14.0, beta=24.0, max_iters=0, heavy_degree=0, small_degree=0,
-         host_loop=False, segmented=0, one_layer=False, coarsening=0):
+         host_loop=False, segmented=0, one_layer=False, coarsening=0, sssp_delta=0):
     """segmented: BFS hub tier with the visited slice in shared memory (0 auto, 1 off, 2 always);
     one_layer: ablation without the summary layer; coarsening: words per warp grab (0 auto)."""
     o = SgOpts()
@@ -162,7 +163,7 @@ def opts(stream=None, direction=SG_DIR_AUTO, alpha=14.0, beta=24.0, max_iters=0,
     o.stream = _stream_ptr(stream)
     o.direction, o.alpha, o.beta, o.max_iters = direction, alpha, beta, max_iters
     o.heavy_degree, o.small_degree, o.host_loop = heavy_degree, small_degree, int(host_loop)
-    o.segmented, o.one_layer, o.coarsening = segmented, int(one_layer), coarsening
+    o.segmented, o.one_layer, o.coarsening, o.sssp_delta = segmented, int(one_layer), coarsening, sssp_delta
     return o
 
 

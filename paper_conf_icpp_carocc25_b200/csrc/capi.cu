@@ -83,6 +83,7 @@ struct Workspace {
     DevStats *h_st = nullptr;      // pinned host mirror
     uint64_t *visited = nullptr;   // nw1 words
     uint32_t *all_offsets = nullptr;   // one-layer ablation: identity word list
+    sg_frontier *far = nullptr;        // delta-stepping SSSP: far pile
     HeavyItem *heavy = nullptr;
     uint32_t heavy_cap = 0;
     int32_t heavy_deg = 0;
@@ -200,6 +201,10 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->heavy);
     cudaFree(ws->seg);
     cudaFree(ws->all_offsets);
+    if (ws->far) {
+        free_frontier_bufs(ws->far);
+        delete ws->far;
+    }
     cudaFree(ws->scratch);
     cudaFreeHost(ws->h_scratch);
     cudaFree(ws->stack);
@@ -1007,7 +1012,47 @@ SG_API int run_sssp(const sg_graph *gc, int32_t src, uint32_t *dist, const sg_op
     TRY(read_stats(ws, s));
     int64_t iters = 0, arcs = 0;
     int in_idx = 0;
-    for (;;) {
+    if (o.sssp_delta > 0) {
+        // near-far delta-stepping (the paper uses plain Bellman-Ford): only the
+        // vertices with dist < T (near) are advanced; improved vertices at >= T wait in `far`; when
+        // near empties, T jumps to the bucket of far's minimum and those vertices move to near.
+        if (!ws->far) {
+            ws->far = new sg_frontier();
+            TRY(alloc_frontier_bufs(ws->far, g, true));
+        }
+        sg_frontier *near = in, *far = ws->far;
+        TRY(clear_frontier(far, s));
+        const double D = (double)o.sssp_delta;
+        double T = D;
+        unsigned int *d_min = reinterpret_cast<unsigned int *>(ws->scratch);
+        for (;;) {
+            while (ws->h_st[0].count) {
+                if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
+                const PushLaunch L = push_launch(g, near, t, (int64_t)ws->h_st[0].count);
+                launch_push_sssp(L, SsspArgs{dist, out->bits, out->summ}, s);
+                TRY(clear_frontier(near, s));
+                launch_filter(G, out->bits, near->bits, near->summ, SG_PRED_U32_RANGE, dist, 0.0, T, 0, s);
+                launch_filter(G, out->bits, far->bits, far->summ, SG_PRED_U32_RANGE, dist, T, 4294967296.0, 0, s);
+                TRY(clear_frontier(out, s));
+                TRY(compact(g, near, false, s));
+                TRY(read_stats(ws, s));
+                iters++;
+            }
+            CK(cudaMemsetAsync(d_min, 0xFF, sizeof(unsigned int), s));
+            launch_min_over_bits(G, far->bits, dist, d_min, s);
+            unsigned int hmin = 0;
+            CK(cudaMemcpyAsync(&hmin, d_min, sizeof hmin, cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            if (hmin == INF32) break;
+            T = (std::floor((double)hmin / D) + 1.0) * D;
+            launch_filter(G, far->bits, near->bits, near->summ, SG_PRED_U32_RANGE, dist, 0.0, T, 0, s);
+            launch_filter(G, far->bits, far->bits, far->summ, SG_PRED_U32_RANGE, dist, T, 4294967296.0, 1, s);
+            TRY(compact(g, near, false, s));
+            TRY(read_stats(ws, s));
+        }
+        arcs = -1;   // not accumulated in this mode
+    }
+    for (; o.sssp_delta <= 0;) {
         const int64_t count = (int64_t)ws->h_st[in_idx].count;
         if (count == 0) break;
         if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);

@@ -94,6 +94,24 @@ __global__ void k_compute(GraphView g, const uint64_t *__restrict__ bits, OpArgs
     }
 }
 
+// min over the active vertices of a uint32 array (delta-stepping: far pile's smallest distance)
+__global__ void k_min_over_bits(GraphView g, const uint64_t *__restrict__ bits, const uint32_t *__restrict__ a,
+                                unsigned int *out) {
+    unsigned int m = 0xFFFFFFFFu;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < g.nw1; w += stride) {
+        uint64_t y = bits[w];
+        while (y) {
+            const int b = __ffsll((long long)y) - 1;
+            y &= y - 1;
+            m = min(m, a[w * 64 + b]);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = min(m, __shfl_xor_sync(0xffffffffu, m, o));
+    if (lane_id() == 0 && m != 0xFFFFFFFFu) atomicMin(out, m);
+}
+
 static int grid_for(int64_t items) {
     int64_t b = (items + 255) / 256;
     if (b > 148 * 8) b = 148 * 8;
@@ -105,6 +123,12 @@ void launch_filter(const GraphView &g, const uint64_t *in_bits, uint64_t *out_bi
     PredArgs p{pred, array, a, b};
     note_launch();
     k_filter<<<grid_for(g.nw1), 256, 0, s>>>(g, in_bits, out_bits, out_summ, p, inplace);
+}
+
+void launch_min_over_bits(const GraphView &g, const uint64_t *bits, const uint32_t *a, unsigned int *out,
+                          cudaStream_t s) {
+    note_launch();
+    k_min_over_bits<<<grid_for(g.nw1), 256, 0, s>>>(g, bits, a, out);
 }
 
 void launch_compute(const GraphView &g, const uint64_t *bits, int op, void *array, double value, cudaStream_t s) {

@@ -80,6 +80,8 @@ void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visi
 void launch_filter(const GraphView &g, const uint64_t *in_bits, uint64_t *out_bits, uint64_t *out_summ, int pred,
                    const void *array, double a, double b, int inplace, cudaStream_t s);
 void launch_compute(const GraphView &g, const uint64_t *bits, int op, void *array, double value, cudaStream_t s);
+void launch_min_over_bits(const GraphView &g, const uint64_t *bits, const uint32_t *a, unsigned int *out,
+                          cudaStream_t s);
 
 // pull_cc.cu — pull label-propagation step (dense CC supersteps)
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,

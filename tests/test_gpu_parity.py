@@ -326,6 +326,18 @@ def test_sssp_lattice_and_unit_weights(sg):
     assert np.array_equal(sg.as_u32(d), oracle.bfs(g2, 0))
 
 
+@pytest.mark.parametrize("delta", [1, 7, 64, 100_000])
+@pytest.mark.parametrize("make", [lambda: gen.with_weights(gen.rmat(14, 16, permute=True), seed=3),
+                                  lambda: gen.with_weights(gen.lattice(150, 200, 0.7), seed=5)])
+def test_sssp_delta_stepping(sg, make, delta):
+    """Near-far delta-stepping (f4) reaches the same distances as Dijkstra for any bucket width."""
+    g = make()
+    G = load(sg, g)
+    for s in gen.sources(g, 2, stream=6):
+        d, st = sg.run_sssp(G, int(s), sssp_delta=delta)
+        assert np.array_equal(sg.as_u32(d), oracle.sssp(g, int(s))), (delta, s)
+
+
 def test_sssp_requires_weights(sg):
     G = load(sg, gen.path(10))
     with pytest.raises(sg.SgError):
