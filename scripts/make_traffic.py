@@ -1,0 +1,54 @@
+"""profiles/traffic.json from an ncu launch list with DRAM metrics of ONE BFS (host-driven loop):
+
+    ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
+        --csv --log-file launches.csv python scripts/profile_one_bfs.py auto
+    python scripts/make_traffic.py launches.csv > profiles/traffic.json
+
+Per bench roofline class: mean DRAM bytes (read + write) per advance launch, where one push
+advance = k_push_words + k_push_heavy (+ k_push_seg) and one pull advance = k_pull_bfs."""
+import collections
+import csv
+import json
+import sys
+
+
+def main(path):
+    lines = open(path).read().splitlines()
+    start = [i for i, l in enumerate(lines) if l.startswith('"ID"')][0]
+    rows = list(csv.reader(lines[start:]))
+    hdr = rows[0]
+    ki, mi, vi, ii = hdr.index("Kernel Name"), hdr.index("Metric Name"), hdr.index("Metric Value"), hdr.index("ID")
+    launches = collections.OrderedDict()
+    for r in rows[1:]:
+        key = (int(r[ii]), r[ki].split("(")[0].replace("void ", ""))
+        launches.setdefault(key, {})[r[mi]] = float(r[vi].replace(",", ""))
+    # keep the last BFS: from the last k_seed on
+    items = list(launches.items())
+    last_seed = max(i for i, ((_, k), _) in enumerate(items) if "k_seed" in k)
+    items = items[last_seed:]
+    push, pull, cur = [], [], None
+    for (_, k), m in items:
+        b = m.get("dram__bytes_read.sum", 0.0) + m.get("dram__bytes_write.sum", 0.0)
+        t = m.get("gpu__time_duration.sum", 0.0)
+        if "k_push_words" in k:
+            cur = [b, t]
+            push.append(cur)
+        elif ("k_push_heavy" in k or "k_push_seg" in k) and cur is not None:
+            cur[0] += b
+            cur[1] += t
+        elif "k_pull_bfs" in k:
+            pull.append([b, t])
+            cur = None
+    out = {
+        "source": f"ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum ({path}); "
+                  "one DO BFS on config 4, cold-cache serialised launches",
+        "advance_push": {"dram_bytes_per_launch": sum(b for b, _ in push) / max(len(push), 1), "launches": len(push),
+                         "ncu_ms_total": sum(t for _, t in push) / 1e6},
+        "advance_pull": {"dram_bytes_per_launch": sum(b for b, _ in pull) / max(len(pull), 1), "launches": len(pull),
+                         "ncu_ms_total": sum(t for _, t in pull) / 1e6},
+    }
+    print(json.dumps(out, indent=1))
+
+
+if __name__ == "__main__":
+    main(sys.argv[1])

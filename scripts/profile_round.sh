@@ -1,0 +1,18 @@
+#!/bin/bash
+# Round profiling pass (run under gpurun): ncu launch lists + full captures of the dominant kernels,
+# summarised into profiles/ by the commands at the bottom (run locally after the merge).
+set -u
+R=${1:-r01}
+mkdir -p gpurun_out
+# 1) launch list of the bench command itself (time only; shares, not absolutes)
+ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${R}_launches_bench.csv \
+    python bench.py --steps 2 --warmup 1 --e2e-steps 0 --no-cpu-baseline > gpurun_out/${R}_ncu_bench.log 2>&1
+# 2) one DO BFS (host-driven loop) with DRAM bytes per launch -> traffic.json
+ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
+    --log-file gpurun_out/${R}_launches_do_dram.csv python scripts/profile_one_bfs.py auto > /dev/null 2>&1
+# 3) full captures: both pull launches (DO), the heavy push level (push-only: words + seg)
+ncu --set full --clock-control none --import-source on -k regex:k_pull_bfs -c 2 \
+    -o gpurun_out/${R}_full_pull python scripts/profile_one_bfs.py auto > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:"k_push_(words|seg)" -s 6 -c 2 \
+    -o gpurun_out/${R}_full_push_l3 python scripts/profile_one_bfs.py push > /dev/null 2>&1
+echo done
