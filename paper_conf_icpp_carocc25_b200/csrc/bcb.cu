@@ -39,12 +39,14 @@ constexpr int BCB_B = 32;   // sources per batch
 #define SG_BCB_PER_SM 1
 #endif
 constexpr int BCB_THREADS = SG_BCB_THREADS;   // few large CTAs: a grid barrier over 148 CTAs is cheap
+constexpr int QUAD = 4;                       // threads per level entry (arcs strided by QUAD)
 
 struct BcbView {
     GraphView g;
     uint32_t *F;          // [3][n] frontier masks (rotating)
     uint32_t *V;          // [n] visited masks
     uint32_t *M;          // [2][n] backward: masks of level d+1
+    uint64_t *VB, *VS;    // vertex-level 2LB of the level being built (layer 1 / layer 2)
     double *s;            // [n][32] scaled sigma
     double *delta;        // [n][32]
     int32_t *lv;          // list vertices (all levels, concatenated)
@@ -64,6 +66,11 @@ __device__ __forceinline__ int exp_of(double x) {   // floor(log2 x) for a posit
 }
 template <typename T>
 __device__ __forceinline__ T vload(const T *p) { return *reinterpret_cast<const volatile T *>(p); }
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 
 // L_0: masks of the batch's sources (duplicates merge into one entry)
 __global__ void k_bcb_init(BcbView b) {
@@ -100,52 +107,29 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
     const int64_t n = b.g.n;
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+    unsigned long long t_mark = gtimer();
     for (;;) {
         const int d = vload(&c->d);
         uint32_t *Fc = b.F + (int64_t)(d % 3) * n;            // masks of L_d
         uint32_t *Fn = b.F + (int64_t)((d + 1) % 3) * n;      // masks of L_{d+1} (being built)
         uint32_t *Fo = b.F + (int64_t)((d + 2) % 3) * n;      // masks of L_{d-1} (to clear)
-        // ---- A: expand L_d; clear L_{d-1}'s masks
+        // ---- A: expand L_d into the next level's masks and a vertex-level 2LB; clear L_{d-1}
         {
+            // QUAD threads per entry (thread k: arcs k, k+QUAD, ...): short dependent chains; all
+            // updates are idempotent ORs issued without waiting for a result (RED)
             const unsigned long long a = vload(&b.loff[d]), e = vload(&b.loff[d + 1]);
-            // warp-uniform loop bounds so list appends can be aggregated: one atomicAdd on the
-            // list tail per warp and neighbour step (a per-vertex atomic on one address
-            // serialises ~10^5 operations per level in L2)
-            const int lane = lane_id();
-            for (unsigned long long i0 = a + (tid & ~31ll); i0 < e; i0 += nthr) {
-                const unsigned long long i = i0 + lane;
-                int32_t v = 0;
-                uint32_t m = 0;
-                int64_t r0 = 0, r1 = 0;
-                if (i < e) {
-                    v = b.lv[i];
-                    m = b.lm[i];
-                    r0 = __ldg(b.g.rp + v);
-                    r1 = __ldg(b.g.rp + v + 1);
-                }
-                int64_t dmax = r1 - r0;
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) {
-                    const int64_t y = __shfl_xor_sync(0xffffffffu, dmax, o);
-                    dmax = y > dmax ? y : dmax;
-                }
-                for (int64_t k = 0; k < dmax; k++) {
-                    bool app = false;
-                    int32_t w = 0;
-                    if (r0 + k < r1) {
-                        w = __ldg(b.g.col + r0 + k);
-                        const uint32_t nm = m & ~vload(b.V + w);
-                        if (nm) app = atomicOr(Fn + w, nm) == 0u;
-                    }
-                    const uint32_t am = __ballot_sync(0xffffffffu, app);
-                    if (am) {
-                        unsigned long long base = 0;
-                        if (lane == __ffs(am) - 1) base = atomicAdd(&c->ltop, (unsigned long long)__popc(am));
-                        base = __shfl_sync(0xffffffffu, base, __ffs(am) - 1);
-                        if (app) {
-                            const unsigned long long pos = base + __popc(am & ((1u << lane) - 1u));
-                            if (pos < (unsigned long long)b.lcap) b.lv[pos] = w;
-                        }
+            const int k = (int)(tid & (QUAD - 1));
+            for (unsigned long long i = a + tid / QUAD; i < e; i += nthr / QUAD) {
+                const int32_t v = b.lv[i];
+                const uint32_t m = b.lm[i];
+                const int64_t r1 = __ldg(b.g.rp + v + 1);
+                for (int64_t r = __ldg(b.g.rp + v) + k; r < r1; r += QUAD) {
+                    const int32_t w = __ldg(b.g.col + r);
+                    const uint32_t nm = m & ~vload(b.V + w);
+                    if (nm) {
+                        atomicOr(Fn + w, nm);
+                        atomic_or_u64(b.VB + (w >> 6), 1ull << (w & 63));
+                        atomic_or_u64(b.VS + (w >> 12), 1ull << ((w >> 6) & 63));
                     }
                 }
             }
@@ -156,6 +140,46 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
         }
         if (threadIdx.x < BCB_B) s_maxe[threadIdx.x] = -1000000;
         grid.sync();
+        if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[0] += t1 - t_mark; t_mark = t1; }
+        // ---- A2: the new level's entries in ascending vertex order (summary-layer compaction:
+        // warp per summary word, lane l owns layer-1 words 64s+2l, 64s+2l+1), clearing the 2LB;
+        // id order gives the sigma / delta passes spatial locality on sigma rows and masks
+        {
+            const int lane = lane_id();
+            const int64_t gw = tid >> 5, nwarps = nthr >> 5;
+            for (int64_t sw = gw; sw < b.g.nw2; sw += nwarps) {
+                const uint64_t x = vload(b.VS + sw);
+                if (!x) continue;
+                const int64_t w0 = sw * 64 + 2 * lane;
+                uint64_t y0 = 0, y1 = 0;
+                if ((x >> (2 * lane)) & 1ull) y0 = vload(b.VB + w0);
+                if ((x >> (2 * lane + 1)) & 1ull) y1 = vload(b.VB + w0 + 1);
+                const uint32_t cnt = __popcll(y0) + __popcll(y1);
+                const uint32_t incl = warp_inclusive_scan(cnt);
+                const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
+                unsigned long long base = 0;
+                if (lane == 0) base = atomicAdd(&c->ltop, (unsigned long long)tot);
+                base = __shfl_sync(0xffffffffu, base, 0) + (incl - cnt);
+                for (int q = 0; q < 2; q++) {
+                    uint64_t y = q ? y1 : y0;
+                    const int64_t w = w0 + q;
+                    if (y) b.VB[w] = 0ull;
+                    while (y) {
+                        const int bit = __ffsll((long long)y) - 1;
+                        y &= y - 1;
+                        const int32_t v = (int32_t)(w * 64 + bit);
+                        if (base < (unsigned long long)b.lcap) {
+                            b.lv[base] = v;
+                            b.lm[base] = vload(Fn + v);
+                        }
+                        base++;
+                    }
+                }
+                if (lane == 0) b.VS[sw] = 0ull;
+            }
+        }
+        grid.sync();
+        if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[1] += t1 - t_mark; t_mark = t1; }
         // ---- B: sigma of the new level (thread per entry, loop over its sources); control step
         const unsigned long long top0 = vload(&c->ltop);
         const bool over = top0 > (unsigned long long)b.lcap || d + 2 > b.cap;
@@ -164,25 +188,41 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
             const unsigned long long e = over ? a : top0;
             if (threadIdx.x < BCB_B) s_kexp[threadIdx.x] = kexp(vload(&b.maxb[(int64_t)d * BCB_B + threadIdx.x]));
             __syncthreads();
-            for (unsigned long long i = a + tid; i < e; i += nthr) {
-                const int32_t w = b.lv[i];
-                const uint32_t m = vload(Fn + w);
-                const int64_t r0 = __ldg(b.g.rp + w), r1 = __ldg(b.g.rp + w + 1);
-                uint32_t mm = m;
-                while (mm) {
-                    const int j = __ffs(mm) - 1;
-                    mm &= mm - 1;
-                    double acc = 0.0;
-                    for (int64_t r = r0; r < r1; r++) {
-                        const int32_t v = __ldg(b.g.col + r);
-                        if ((vload(Fc + v) >> j) & 1u) acc += b.s[(int64_t)v * BCB_B + j];
-                    }
-                    const double sv = ldexp(acc, -s_kexp[j]);
-                    b.s[(int64_t)w * BCB_B + j] = sv;
-                    atomicMax(&s_maxe[j], exp_of(sv));
+            // QUAD threads per entry: thread k sums arcs k, k+QUAD, ...; quad shuffle reduction in a
+            // fixed order (deterministic)
+            const int k = (int)(tid & (QUAD - 1));
+            // warp-uniform trip count (the loop body uses warp shuffles / votes)
+            const unsigned long long ncap = ((e - a) * QUAD + 31) / 32 * 32;
+            for (unsigned long long ii = tid; ii < ncap; ii += nthr) {
+                const unsigned long long i = a + ii / QUAD;
+                const bool valid = i < e;
+                const int32_t w = valid ? b.lv[i] : 0;
+                const uint32_t m = valid ? b.lm[i] : 0u;
+                int64_t r0 = 0, r1 = 0;
+                if (valid) {
+                    r0 = __ldg(b.g.rp + w);
+                    r1 = __ldg(b.g.rp + w + 1);
                 }
-                b.lm[i] = m;
-                b.V[w] |= m;
+                uint32_t mm = m;
+                while (__any_sync(0xffffffffu, mm != 0u)) {
+                    const int j = mm ? __ffs(mm) - 1 : 0;
+                    double acc = 0.0;
+                    if (mm) {
+                        for (int64_t r = r0 + k; r < r1; r += QUAD) {
+                            const int32_t v = __ldg(b.g.col + r);
+                            if ((vload(Fc + v) >> j) & 1u) acc += b.s[(int64_t)v * BCB_B + j];
+                        }
+                    }
+                    acc += __shfl_xor_sync(0xffffffffu, acc, 1);
+                    acc += __shfl_xor_sync(0xffffffffu, acc, 2);
+                    if (mm && k == 0) {
+                        const double sv = ldexp(acc, -s_kexp[j]);
+                        b.s[(int64_t)w * BCB_B + j] = sv;
+                        atomicMax(&s_maxe[j], exp_of(sv));
+                    }
+                    if (mm) mm &= mm - 1;
+                }
+                if (valid && k == 0) b.V[w] |= m;
             }
             __syncthreads();
             if (threadIdx.x < BCB_B && s_maxe[threadIdx.x] > -100000)
@@ -202,6 +242,7 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
             c->par = more ? 1 : 0;               // loop flag
         }
         grid.sync();
+        if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[2] += t1 - t_mark; t_mark = t1; }
         if (!vload(&c->par)) break;
     }
 }
@@ -215,6 +256,7 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     if (threadIdx.x < BCB_B) s_src[threadIdx.x] = threadIdx.x < c->nsrc ? c->src[threadIdx.x] : -1;
     __syncthreads();
+    unsigned long long t_mark = gtimer();
     // the deepest level has no successors: delta = 0 there, written by its own pass
     for (int d = vload(&c->depth) - 1; d >= 1; d--) {
         uint32_t *Mn = b.M + (int64_t)((d + 1) & 1) * n;   // masks of L_{d+1}
@@ -224,32 +266,47 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
             for (unsigned long long i = a + tid; i < e; i += nthr) Mn[b.lv[i]] = b.lm[i];
         }
         grid.sync();
+        if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[3] += t1 - t_mark; t_mark = t1; }
         {
             const unsigned long long a = b.loff[d], e = b.loff[d + 1];
             if (threadIdx.x < BCB_B) s_kexp[threadIdx.x] = kexp(b.maxb[(int64_t)d * BCB_B + threadIdx.x]);
             __syncthreads();
-            for (unsigned long long i = a + tid; i < e; i += nthr) {
-                const int32_t v = b.lv[i];
-                const uint32_t m = b.lm[i];
-                const int64_t r0 = __ldg(b.g.rp + v), r1 = __ldg(b.g.rp + v + 1);
+            const int k = (int)(tid & (QUAD - 1));
+            const unsigned long long ncap = ((e - a) * QUAD + 31) / 32 * 32;   // warp-uniform trip count
+            for (unsigned long long ii = tid; ii < ncap; ii += nthr) {
+                const unsigned long long i = a + ii / QUAD;
+                const bool valid = i < e;
+                const int32_t v = valid ? b.lv[i] : 0;
+                const uint32_t m = valid ? b.lm[i] : 0u;
+                int64_t r0 = 0, r1 = 0;
+                if (valid) {
+                    r0 = __ldg(b.g.rp + v);
+                    r1 = __ldg(b.g.rp + v + 1);
+                }
                 double contrib = 0.0;
                 uint32_t mm = m;
-                while (mm) {   // sources in ascending order: deterministic sum
-                    const int j = __ffs(mm) - 1;
-                    mm &= mm - 1;
+                while (__any_sync(0xffffffffu, mm != 0u)) {   // sources ascending: deterministic
+                    const int j = mm ? __ffs(mm) - 1 : 0;
                     double acc = 0.0;
-                    for (int64_t r = r0; r < r1; r++) {
-                        const int32_t w = __ldg(b.g.col + r);
-                        if ((vload(Mn + w) >> j) & 1u) {
-                            const int64_t q = (int64_t)w * BCB_B + j;
-                            acc += (1.0 + b.delta[q]) / b.s[q];
+                    if (mm) {
+                        for (int64_t r = r0 + k; r < r1; r += QUAD) {
+                            const int32_t w = __ldg(b.g.col + r);
+                            if ((vload(Mn + w) >> j) & 1u) {
+                                const int64_t q = (int64_t)w * BCB_B + j;
+                                acc += (1.0 + b.delta[q]) / b.s[q];
+                            }
                         }
                     }
-                    const double dv = ldexp(b.s[(int64_t)v * BCB_B + j] * acc, -s_kexp[j]);
-                    b.delta[(int64_t)v * BCB_B + j] = dv;
-                    if (v != s_src[j]) contrib += dv;
+                    acc += __shfl_xor_sync(0xffffffffu, acc, 1);
+                    acc += __shfl_xor_sync(0xffffffffu, acc, 2);
+                    if (mm && k == 0) {
+                        const double dv = ldexp(b.s[(int64_t)v * BCB_B + j] * acc, -s_kexp[j]);
+                        b.delta[(int64_t)v * BCB_B + j] = dv;
+                        if (v != s_src[j]) contrib += dv;
+                    }
+                    if (mm) mm &= mm - 1;
                 }
-                if (m) b.bc[v] += contrib;
+                if (valid && k == 0 && m) b.bc[v] += contrib;
             }
             if (d + 2 <= vload(&c->depth)) {
                 const unsigned long long a2 = b.loff[d + 2], e2 = b.loff[d + 3];
@@ -257,6 +314,7 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
             }
         }
         grid.sync();
+        if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[4] += t1 - t_mark; t_mark = t1; }
     }
 }
 
@@ -287,6 +345,8 @@ static BcbView view_of(const BcbLaunch &L) {
     b.F = L.F;
     b.V = L.V;
     b.M = L.M;
+    b.VB = L.VB;
+    b.VS = L.VS;
     b.s = L.s;
     b.delta = L.delta;
     b.lv = L.lv;

@@ -219,6 +219,8 @@ static void free_ws(Workspace *ws) {
         cudaFree(B.F);
         cudaFree(B.V);
         cudaFree(B.M);
+        cudaFree(B.VB);
+        cudaFree(B.VS);
         cudaFree(B.s);
         cudaFree(B.delta);
         cudaFree(B.lv);
@@ -1169,6 +1171,10 @@ static int bcb_alloc(sg_graph *g) {
     CK(cudaMalloc(&B.maxb, sizeof(unsigned long long) * (size_t)(B.cap + 1) * 32));
     CK(cudaMalloc(&B.c, sizeof(BcbCtrl)));
     CK(cudaMallocHost(&ws->h_bcb, sizeof(BcbCtrl)));
+    CK(cudaMalloc(&B.VB, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMalloc(&B.VS, sizeof(uint64_t) * (size_t)g->v.nw2));
+    CK(cudaMemset(B.VB, 0, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMemset(B.VS, 0, sizeof(uint64_t) * (size_t)g->v.nw2));
     CK(cudaMemset(B.F, 0, sizeof(uint32_t) * (size_t)n * 3));
     CK(cudaMemset(B.V, 0, sizeof(uint32_t) * (size_t)n));
     CK(cudaMemset(B.M, 0, sizeof(uint32_t) * (size_t)n * 2));
@@ -1200,6 +1206,10 @@ static int run_bc_batched(sg_graph *g, const int32_t *sources, int32_t k, double
         CK(cudaStreamSynchronize(s));
         if (c.overflow) return fail(SG_ERR_UNSUPPORTED, "batched BC: level/list capacity exceeded");
         levels += c.depth;
+        if (getenv("SG_TRACE"))
+            fprintf(stderr, "[sygraph bc] batch %d: %d levels, phase ms fwdA %.2f fwdA2 %.2f fwdB %.2f bwdA %.2f bwdB %.2f\n",
+                    b0 / 32, c.depth, c.t_ns[0] / 1e6, c.t_ns[1] / 1e6, c.t_ns[2] / 1e6, c.t_ns[3] / 1e6,
+                    c.t_ns[4] / 1e6);
     }
     CK(cudaEventRecord(ws->ev1, s));
     CK(cudaEventSynchronize(ws->ev1));

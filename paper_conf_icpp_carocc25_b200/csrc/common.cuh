@@ -62,6 +62,7 @@ struct BcbCtrl {
     unsigned long long ltop;   // entries appended to the level lists
     int32_t overflow;          // level / list capacity exceeded
     int32_t pad;
+    unsigned long long t_ns[6];   // per-phase time (globaltimer, CTA 0 view): fwd A, A2, B; bwd A, B
 };
 
 // One CTA/grid-tier work unit: a contiguous piece of one vertex's adjacency list.

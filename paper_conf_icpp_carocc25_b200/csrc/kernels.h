@@ -102,6 +102,7 @@ void launch_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *st_src
 struct BcbLaunch {
     GraphView g;
     uint32_t *F, *V, *M;
+    uint64_t *VB, *VS;
     double *s, *delta;
     int32_t *lv;
     uint32_t *lm;
