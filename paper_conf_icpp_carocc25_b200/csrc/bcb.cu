@@ -8,9 +8,11 @@
 // separated by grid-wide barriers (two per level) instead of kernel launches.
 //
 // Forward level d -> d+1:
-//   A  expand: for (v, m) in L_d, w in N(v): nm = m & ~V[w]; if nm: F_{d+1}[w] |= nm (first
-//      setter appends w to L_{d+1});  clear F_{d-1} for the entries of L_{d-1}    | grid sync
-//   B  sigma (warp per new entry, lane j): if j in F_{d+1}[w]:
+//   A  expand (QUAD threads per entry): for (v, m) in L_d, w in N(v): nm = m & ~V[w]; if nm:
+//      F_{d+1}[w] |= nm and w is set in a vertex-level 2LB (VB / VS);  clear F_{d-1} | grid sync
+//   A2 extract L_{d+1} from the 2LB in ascending vertex order (summary compaction), clear it
+//                                                                                  | grid sync
+//   B  sigma (QUAD threads per new entry, loop over its sources j): if j in F_{d+1}[w]:
 //        s[w][j] = 2^-k_j(d) * sum_{v in N(w), j in F_d[v]} s[v][j];  V[w] |= F_{d+1}[w]
 //      per-source max of the level -> k_j(d+1) = floor(log2 max); control step   | grid sync
 //   (three frontier-mask buffers rotate: F_{d-1} is cleared while F_d / F_{d+1} are live)
@@ -144,22 +146,33 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
         // ---- A2: the new level's entries in ascending vertex order (summary-layer compaction:
         // warp per summary word, lane l owns layer-1 words 64s+2l, 64s+2l+1), clearing the 2LB;
         // id order gives the sigma / delta passes spatial locality on sigma rows and masks
+        // (one list reservation per CTA and round: a same-address atomic per summary word
+        // serialises thousands of requests per level)
         {
-            const int lane = lane_id();
-            const int64_t gw = tid >> 5, nwarps = nthr >> 5;
-            for (int64_t sw = gw; sw < b.g.nw2; sw += nwarps) {
-                const uint64_t x = vload(b.VS + sw);
-                if (!x) continue;
+            __shared__ uint32_t s_wofs[BCB_THREADS / 32];
+            __shared__ unsigned long long s_base;
+            const int lane = lane_id(), wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
+            for (int64_t sw0 = (int64_t)blockIdx.x * nwb; sw0 < b.g.nw2; sw0 += (int64_t)gridDim.x * nwb) {
+                const int64_t sw = sw0 + wib;
+                const uint64_t x = sw < b.g.nw2 ? vload(b.VS + sw) : 0ull;
                 const int64_t w0 = sw * 64 + 2 * lane;
                 uint64_t y0 = 0, y1 = 0;
                 if ((x >> (2 * lane)) & 1ull) y0 = vload(b.VB + w0);
                 if ((x >> (2 * lane + 1)) & 1ull) y1 = vload(b.VB + w0 + 1);
                 const uint32_t cnt = __popcll(y0) + __popcll(y1);
                 const uint32_t incl = warp_inclusive_scan(cnt);
-                const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
-                unsigned long long base = 0;
-                if (lane == 0) base = atomicAdd(&c->ltop, (unsigned long long)tot);
-                base = __shfl_sync(0xffffffffu, base, 0) + (incl - cnt);
+                if (lane == 31) s_wofs[wib] = incl;
+                __syncthreads();
+                if (wib == 0) {
+                    const uint32_t t = lane < nwb ? s_wofs[lane] : 0u;
+                    const uint32_t ti = warp_inclusive_scan(t);
+                    if (lane < nwb) s_wofs[lane] = ti - t;
+                    if (lane == 31) s_base = ti ? atomicAdd(&c->ltop, (unsigned long long)ti) : 0ull;
+                }
+                __syncthreads();
+                unsigned long long base = s_base + s_wofs[wib] + (incl - cnt);
+                __syncthreads();   // s_wofs / s_base are rewritten next round
+                if (!x) continue;
                 for (int q = 0; q < 2; q++) {
                     uint64_t y = q ? y1 : y0;
                     const int64_t w = w0 + q;
@@ -168,10 +181,9 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
                         const int bit = __ffsll((long long)y) - 1;
                         y &= y - 1;
                         const int32_t v = (int32_t)(w * 64 + bit);
-                        if (base < (unsigned long long)b.lcap) {
-                            b.lv[base] = v;
-                            b.lm[base] = vload(Fn + v);
-                        }
+                        // stores only (a load whose result is stored would stall every bit);
+                        // the mask lm is filled by phase B, which reads F_{d+1}[w] anyway
+                        if (base < (unsigned long long)b.lcap) b.lv[base] = v;
                         base++;
                     }
                 }
@@ -197,18 +209,29 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
                 const unsigned long long i = a + ii / QUAD;
                 const bool valid = i < e;
                 const int32_t w = valid ? b.lv[i] : 0;
-                const uint32_t m = valid ? b.lm[i] : 0u;
+                uint32_t m = 0u;
                 int64_t r0 = 0, r1 = 0;
                 if (valid) {
+                    m = vload(Fn + w);
                     r0 = __ldg(b.g.rp + w);
                     r1 = __ldg(b.g.rp + w + 1);
+                    if (k == 0) b.lm[i] = m;
                 }
+                // the thread's first two arcs and their frontier masks are loaded once, outside
+                // the loop over sources (each source then costs one dependent load of sigma)
+                const int64_t ra = r0 + k;
+                const int32_t v0 = ra < r1 ? __ldg(b.g.col + ra) : 0;
+                const int32_t v1 = ra + QUAD < r1 ? __ldg(b.g.col + ra + QUAD) : 0;
+                const uint32_t f0 = ra < r1 ? vload(Fc + v0) & m : 0u;
+                const uint32_t f1 = ra + QUAD < r1 ? vload(Fc + v1) & m : 0u;
                 uint32_t mm = m;
                 while (__any_sync(0xffffffffu, mm != 0u)) {
                     const int j = mm ? __ffs(mm) - 1 : 0;
                     double acc = 0.0;
                     if (mm) {
-                        for (int64_t r = r0 + k; r < r1; r += QUAD) {
+                        if ((f0 >> j) & 1u) acc += b.s[(int64_t)v0 * BCB_B + j];
+                        if ((f1 >> j) & 1u) acc += b.s[(int64_t)v1 * BCB_B + j];
+                        for (int64_t r = ra + 2 * QUAD; r < r1; r += QUAD) {
                             const int32_t v = __ldg(b.g.col + r);
                             if ((vload(Fc + v) >> j) & 1u) acc += b.s[(int64_t)v * BCB_B + j];
                         }
@@ -283,13 +306,28 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
                     r0 = __ldg(b.g.rp + v);
                     r1 = __ldg(b.g.rp + v + 1);
                 }
+                // first two arcs of the thread and their successor masks hoisted out of the
+                // loop over sources (as in the forward sigma pass)
+                const int64_t ra = r0 + k;
+                const int32_t w0 = ra < r1 ? __ldg(b.g.col + ra) : 0;
+                const int32_t w1 = ra + QUAD < r1 ? __ldg(b.g.col + ra + QUAD) : 0;
+                const uint32_t g0 = ra < r1 ? vload(Mn + w0) & m : 0u;
+                const uint32_t g1 = ra + QUAD < r1 ? vload(Mn + w1) & m : 0u;
                 double contrib = 0.0;
                 uint32_t mm = m;
                 while (__any_sync(0xffffffffu, mm != 0u)) {   // sources ascending: deterministic
                     const int j = mm ? __ffs(mm) - 1 : 0;
                     double acc = 0.0;
                     if (mm) {
-                        for (int64_t r = r0 + k; r < r1; r += QUAD) {
+                        if ((g0 >> j) & 1u) {
+                            const int64_t q = (int64_t)w0 * BCB_B + j;
+                            acc += (1.0 + b.delta[q]) / b.s[q];
+                        }
+                        if ((g1 >> j) & 1u) {
+                            const int64_t q = (int64_t)w1 * BCB_B + j;
+                            acc += (1.0 + b.delta[q]) / b.s[q];
+                        }
+                        for (int64_t r = ra + 2 * QUAD; r < r1; r += QUAD) {
                             const int32_t w = __ldg(b.g.col + r);
                             if ((vload(Mn + w) >> j) & 1u) {
                                 const int64_t q = (int64_t)w * BCB_B + j;

@@ -1207,8 +1207,8 @@ static int run_bc_batched(sg_graph *g, const int32_t *sources, int32_t k, double
         if (c.overflow) return fail(SG_ERR_UNSUPPORTED, "batched BC: level/list capacity exceeded");
         levels += c.depth;
         if (getenv("SG_TRACE"))
-            fprintf(stderr, "[sygraph bc] batch %d: %d levels, phase ms fwdA %.2f fwdA2 %.2f fwdB %.2f bwdA %.2f bwdB %.2f\n",
-                    b0 / 32, c.depth, c.t_ns[0] / 1e6, c.t_ns[1] / 1e6, c.t_ns[2] / 1e6, c.t_ns[3] / 1e6,
+            fprintf(stderr, "[sygraph bc] batch %d: %d levels, %llu entries, phase ms fwdA %.2f fwdA2 %.2f fwdB %.2f bwdA %.2f bwdB %.2f\n",
+                    b0 / 32, c.depth, c.ltop, c.t_ns[0] / 1e6, c.t_ns[1] / 1e6, c.t_ns[2] / 1e6, c.t_ns[3] / 1e6,
                     c.t_ns[4] / 1e6);
     }
     CK(cudaEventRecord(ws->ev1, s));
