@@ -41,7 +41,10 @@ constexpr int BCB_B = 32;   // sources per batch
 #define SG_BCB_PER_SM 1
 #endif
 constexpr int BCB_THREADS = SG_BCB_THREADS;   // few large CTAs: a grid barrier over 148 CTAs is cheap
-constexpr int QUAD = 4;                       // threads per level entry (arcs strided by QUAD)
+#ifndef SG_BCB_QUAD
+#define SG_BCB_QUAD 2
+#endif
+constexpr int QUAD = SG_BCB_QUAD;             // threads per level entry (arcs strided by QUAD)
 
 struct BcbView {
     GraphView g;
@@ -72,6 +75,15 @@ __device__ __forceinline__ unsigned long long gtimer() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
+}
+
+// F_{d+1}[w] |= nm and w into the level's vertex 2LB (fire-and-forget ORs)
+__device__ __forceinline__ void bcb_mark(const BcbView &b, uint32_t *Fn, int32_t w, uint32_t nm) {
+    if (nm) {
+        atomicOr(Fn + w, nm);
+        atomic_or_u64(b.VB + (w >> 6), 1ull << (w & 63));
+        atomic_or_u64(b.VS + (w >> 12), 1ull << ((w >> 6) & 63));
+    }
 }
 
 // L_0: masks of the batch's sources (duplicates merge into one entry)
@@ -105,13 +117,24 @@ __global__ void k_bcb_init(BcbView b) {
 __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
     cg::grid_group grid = cg::this_grid();
     __shared__ int s_maxe[BCB_B], s_kexp[BCB_B];
+    // control words are read by one thread per CTA and broadcast through shared memory (151K
+    // threads loading one address would queue ~5K requests on one L2 slice per phase)
+    __shared__ unsigned long long s_ctl[6];
     BcbCtrl *c = b.c;
     const int64_t n = b.g.n;
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     unsigned long long t_mark = gtimer();
     for (;;) {
-        const int d = vload(&c->d);
+        if (threadIdx.x == 0) {
+            const int dd = vload(&c->d);
+            s_ctl[0] = (unsigned long long)dd;
+            s_ctl[1] = vload(&b.loff[dd]);
+            s_ctl[2] = vload(&b.loff[dd + 1]);
+            s_ctl[3] = dd >= 1 ? vload(&b.loff[dd - 1]) : 0ull;
+        }
+        __syncthreads();
+        const int d = (int)s_ctl[0];
         uint32_t *Fc = b.F + (int64_t)(d % 3) * n;            // masks of L_d
         uint32_t *Fn = b.F + (int64_t)((d + 1) % 3) * n;      // masks of L_{d+1} (being built)
         uint32_t *Fo = b.F + (int64_t)((d + 2) % 3) * n;      // masks of L_{d-1} (to clear)
@@ -119,24 +142,27 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
         {
             // QUAD threads per entry (thread k: arcs k, k+QUAD, ...): short dependent chains; all
             // updates are idempotent ORs issued without waiting for a result (RED)
-            const unsigned long long a = vload(&b.loff[d]), e = vload(&b.loff[d + 1]);
+            const unsigned long long a = s_ctl[1], e = s_ctl[2];
             const int k = (int)(tid & (QUAD - 1));
             for (unsigned long long i = a + tid / QUAD; i < e; i += nthr / QUAD) {
                 const int32_t v = b.lv[i];
                 const uint32_t m = b.lm[i];
                 const int64_t r1 = __ldg(b.g.rp + v + 1);
-                for (int64_t r = __ldg(b.g.rp + v) + k; r < r1; r += QUAD) {
+                const int64_t ra = __ldg(b.g.rp + v) + k;
+                // the thread's first two arcs are loaded side by side (two independent chains)
+                const int32_t w0 = ra < r1 ? __ldg(b.g.col + ra) : 0;
+                const int32_t w1 = ra + QUAD < r1 ? __ldg(b.g.col + ra + QUAD) : 0;
+                const uint32_t n0 = ra < r1 ? m & ~vload(b.V + w0) : 0u;
+                const uint32_t n1 = ra + QUAD < r1 ? m & ~vload(b.V + w1) : 0u;
+                bcb_mark(b, Fn, w0, n0);
+                bcb_mark(b, Fn, w1, n1);
+                for (int64_t r = ra + 2 * QUAD; r < r1; r += QUAD) {
                     const int32_t w = __ldg(b.g.col + r);
-                    const uint32_t nm = m & ~vload(b.V + w);
-                    if (nm) {
-                        atomicOr(Fn + w, nm);
-                        atomic_or_u64(b.VB + (w >> 6), 1ull << (w & 63));
-                        atomic_or_u64(b.VS + (w >> 12), 1ull << ((w >> 6) & 63));
-                    }
+                    bcb_mark(b, Fn, w, m & ~vload(b.V + w));
                 }
             }
             if (d >= 1) {
-                const unsigned long long a0 = vload(&b.loff[d - 1]), e0 = vload(&b.loff[d]);
+                const unsigned long long a0 = s_ctl[3], e0 = s_ctl[1];
                 for (unsigned long long i = a0 + tid; i < e0; i += nthr) Fo[b.lv[i]] = 0u;
             }
         }
@@ -193,13 +219,14 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
         grid.sync();
         if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[1] += t1 - t_mark; t_mark = t1; }
         // ---- B: sigma of the new level (thread per entry, loop over its sources); control step
-        const unsigned long long top0 = vload(&c->ltop);
+        if (threadIdx.x == 0) s_ctl[4] = vload(&c->ltop);
+        if (threadIdx.x < BCB_B) s_kexp[threadIdx.x] = kexp(vload(&b.maxb[(int64_t)d * BCB_B + threadIdx.x]));
+        __syncthreads();
+        const unsigned long long top0 = s_ctl[4];
         const bool over = top0 > (unsigned long long)b.lcap || d + 2 > b.cap;
         {
-            const unsigned long long a = vload(&b.loff[d + 1]);
+            const unsigned long long a = s_ctl[2];
             const unsigned long long e = over ? a : top0;
-            if (threadIdx.x < BCB_B) s_kexp[threadIdx.x] = kexp(vload(&b.maxb[(int64_t)d * BCB_B + threadIdx.x]));
-            __syncthreads();
             // QUAD threads per entry: thread k sums arcs k, k+QUAD, ...; quad shuffle reduction in a
             // fixed order (deterministic)
             const int k = (int)(tid & (QUAD - 1));
@@ -236,8 +263,8 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
                             if ((vload(Fc + v) >> j) & 1u) acc += b.s[(int64_t)v * BCB_B + j];
                         }
                     }
-                    acc += __shfl_xor_sync(0xffffffffu, acc, 1);
-                    acc += __shfl_xor_sync(0xffffffffu, acc, 2);
+#pragma unroll
+                    for (int o = 1; o < QUAD; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
                     if (mm && k == 0) {
                         const double sv = ldexp(acc, -s_kexp[j]);
                         b.s[(int64_t)w * BCB_B + j] = sv;
@@ -253,7 +280,7 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
                           (unsigned long long)(s_maxe[threadIdx.x] + EXP_BIAS));
         }
         if (tid == 0) {
-            const bool more = !over && top0 > b.loff[d + 1];
+            const bool more = !over && top0 > s_ctl[2];
             if (over) c->overflow = 1;
             if (more) {
                 c->d = d + 1;
@@ -266,7 +293,9 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
         }
         grid.sync();
         if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[2] += t1 - t_mark; t_mark = t1; }
-        if (!vload(&c->par)) break;
+        if (threadIdx.x == 0) s_ctl[5] = vload(&c->par);
+        __syncthreads();
+        if (!s_ctl[5]) break;
     }
 }
 
@@ -275,23 +304,33 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
     BcbCtrl *c = b.c;
     const int64_t n = b.g.n;
     __shared__ int s_kexp[BCB_B], s_src[BCB_B];
+    __shared__ unsigned long long s_off[5];   // loff[d .. d+3], depth (one reader per CTA)
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     if (threadIdx.x < BCB_B) s_src[threadIdx.x] = threadIdx.x < c->nsrc ? c->src[threadIdx.x] : -1;
+    if (threadIdx.x == 0) s_off[4] = (unsigned long long)vload(&c->depth);
     __syncthreads();
+    const int depth = (int)s_off[4];
     unsigned long long t_mark = gtimer();
     // the deepest level has no successors: delta = 0 there, written by its own pass
-    for (int d = vload(&c->depth) - 1; d >= 1; d--) {
+    for (int d = depth - 1; d >= 1; d--) {
+        if (threadIdx.x == 0) {
+            s_off[0] = b.loff[d];
+            s_off[1] = b.loff[d + 1];
+            s_off[2] = b.loff[d + 2];
+            s_off[3] = d + 2 <= depth ? b.loff[d + 3] : 0ull;
+        }
+        __syncthreads();
         uint32_t *Mn = b.M + (int64_t)((d + 1) & 1) * n;   // masks of L_{d+1}
         uint32_t *Mo = b.M + (int64_t)(d & 1) * n;         // held L_{d+2}: cleared below
         {
-            const unsigned long long a = b.loff[d + 1], e = b.loff[d + 2];
+            const unsigned long long a = s_off[1], e = s_off[2];
             for (unsigned long long i = a + tid; i < e; i += nthr) Mn[b.lv[i]] = b.lm[i];
         }
         grid.sync();
         if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[3] += t1 - t_mark; t_mark = t1; }
         {
-            const unsigned long long a = b.loff[d], e = b.loff[d + 1];
+            const unsigned long long a = s_off[0], e = s_off[1];
             if (threadIdx.x < BCB_B) s_kexp[threadIdx.x] = kexp(b.maxb[(int64_t)d * BCB_B + threadIdx.x]);
             __syncthreads();
             const int k = (int)(tid & (QUAD - 1));
@@ -335,8 +374,8 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
                             }
                         }
                     }
-                    acc += __shfl_xor_sync(0xffffffffu, acc, 1);
-                    acc += __shfl_xor_sync(0xffffffffu, acc, 2);
+#pragma unroll
+                    for (int o = 1; o < QUAD; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
                     if (mm && k == 0) {
                         const double dv = ldexp(b.s[(int64_t)v * BCB_B + j] * acc, -s_kexp[j]);
                         b.delta[(int64_t)v * BCB_B + j] = dv;
@@ -346,8 +385,8 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
                 }
                 if (valid && k == 0 && m) b.bc[v] += contrib;
             }
-            if (d + 2 <= vload(&c->depth)) {
-                const unsigned long long a2 = b.loff[d + 2], e2 = b.loff[d + 3];
+            if (d + 2 <= depth) {
+                const unsigned long long a2 = s_off[2], e2 = s_off[3];
                 for (unsigned long long i = a2 + tid; i < e2; i += nthr) Mo[b.lv[i]] = 0u;
             }
         }
@@ -363,7 +402,21 @@ __global__ void k_bcb_reset(BcbView b) {
     if (top > (unsigned long long)b.lcap) top = b.lcap;
     const int64_t n = b.g.n;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (unsigned long long i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < top; i += stride) {
+    const int64_t t0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (top > (unsigned long long)n / 2) {
+        // many entries (a vertex recurs once per source): zeroing the mask arrays whole is cheaper
+        // than scattering 6 stores per entry
+        uint32_t *arr[3] = {b.V, b.F, b.M};
+        const int64_t len[3] = {n, 3 * n, 2 * n};
+        for (int a = 0; a < 3; a++) {
+            uint32_t *p = arr[a];
+            const int64_t nv = len[a] / 4;   // cudaMalloc'd: 256-B aligned
+            for (int64_t i = t0; i < nv; i += stride) reinterpret_cast<uint4 *>(p)[i] = make_uint4(0, 0, 0, 0);
+            for (int64_t i = nv * 4 + t0; i < len[a]; i += stride) p[i] = 0u;
+        }
+        top = 0;
+    }
+    for (unsigned long long i = t0; i < top; i += stride) {
         const int32_t v = b.lv[i];
         b.V[v] = 0u;
         b.F[v] = 0u;
