@@ -7,23 +7,24 @@
 // direction (forward / backward) is ONE persistent cooperative kernel whose supersteps are
 // separated by grid-wide barriers (two per level) instead of kernel launches.
 //
-// Forward level d -> d+1:
+// Forward level d -> d+1 (k_j(d) = exponent of the max of level d's stored sigma for source j):
 //   A  expand (QUAD threads per entry): for (v, m) in L_d, w in N(v): nm = m & ~V[w]; if nm:
-//      F_{d+1}[w] |= nm and w is set in a vertex-level 2LB (VB / VS);  clear F_{d-1} | grid sync
+//      F_{d+1}[w] |= nm and w into a vertex-level 2LB (VB / VS);  clear F_{d-1}      | grid sync
 //   A2 extract L_{d+1} from the 2LB in ascending vertex order (summary compaction), clear it
 //                                                                                  | grid sync
-//   B  sigma (QUAD threads per new entry, loop over its sources j): if j in F_{d+1}[w]:
+//   B  sigma (QUAD threads per new entry, loop over its sources j; fixed-order gather):
 //        s[w][j] = 2^-k_j(d) * sum_{v in N(w), j in F_d[v]} s[v][j];  V[w] |= F_{d+1}[w]
-//      per-source max of the level -> k_j(d+1) = floor(log2 max); control step   | grid sync
+//      per-source max -> k_j(d+1); control step                                    | grid sync
 //   (three frontier-mask buffers rotate: F_{d-1} is cleared while F_d / F_{d+1} are live)
 // Stored s is sigma scaled by 2^-G_j(level) with G_j(L+1) = G_j(L) + k_j(L): exact power-of-two
-// scaling (reading C20 / R5), every level's max in [1, 2).
-// Backward level d = D-1 .. 1:
-//   A  M_{(d+1)%2}[w] = mask of w in L_{d+1}                                      | grid sync
-//   B  for (v, m) in L_d (warp; lane j in m):
-//        delta[v][j] = 2^-k_j(d) * s[v][j] * sum_{w in N(v), j in M[w]} (1 + delta[w][j]) / s[w][j]
-//      bc[v] += sum over lanes (fixed shuffle order: deterministic); clear M_{d%2} of L_{d+2}
-//                                                                                  | grid sync
+// scaling (reading C20 / R5), every level's max in [1, 2).  (Pushing sigma with fp64 atomics in
+// A instead was measured slower on config 5: 302 vs 284 ms of forward time per batch.)
+// Backward, one pass per level d = D-1 .. 1 (three rotating level-mask buffers M):
+//   for (v, m) in L_d, j in m: delta[v][j] = 2^-k_j(d) * s[v][j] * acc[v][j], where acc (the
+//   `delta` array) holds sum_{w succ} (1 + delta[w][j]) / s[w][j] pushed by the pass of d+1;
+//   bc[v] += delta[v][j] (j ascending); push (1 + delta[v][j]) / s[v][j] to predecessors u with
+//   j in M_{d-1}[u] (fp64 atomics, as the paper's functors; one barrier per level instead of
+//   the gather's two); lay out M_{d-2}, clear M_d                                  | grid sync
 #include <cooperative_groups.h>
 
 #include "common.cuh"
@@ -299,12 +300,14 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_forward(BcbView b) {
     }
 }
 
+// M_x: masks of level x (three rotating buffers)
+__device__ __forceinline__ uint32_t *bcb_M(const BcbView &b, int x) { return b.M + (int64_t)(x % 3) * b.g.n; }
+
 __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
     cg::grid_group grid = cg::this_grid();
     BcbCtrl *c = b.c;
-    const int64_t n = b.g.n;
     __shared__ int s_kexp[BCB_B], s_src[BCB_B];
-    __shared__ unsigned long long s_off[5];   // loff[d .. d+3], depth (one reader per CTA)
+    __shared__ unsigned long long s_off[5];   // loff[d], loff[d+1], loff[d-2], loff[d-1]; depth
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     if (threadIdx.x < BCB_B) s_src[threadIdx.x] = threadIdx.x < c->nsrc ? c->src[threadIdx.x] : -1;
@@ -312,90 +315,75 @@ __global__ void __launch_bounds__(BCB_THREADS) k_bcb_backward(BcbView b) {
     __syncthreads();
     const int depth = (int)s_off[4];
     unsigned long long t_mark = gtimer();
-    // the deepest level has no successors: delta = 0 there, written by its own pass
+    // pre-pass: masks of the level below the deepest
+    if (depth - 2 >= 1) {
+        uint32_t *Mp = bcb_M(b, depth - 2);
+        for (unsigned long long i = b.loff[depth - 2] + tid; i < b.loff[depth - 1]; i += nthr) Mp[b.lv[i]] = b.lm[i];
+    }
+    grid.sync();
+    if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[3] += t1 - t_mark; t_mark = t1; }
+    // level d (deepest first): delta_j(v) = 2^-k_j(d) s_j(v) acc_j(v) with acc_j(v) the sum of
+    // (1 + delta_j(w)) / s_j(w) over successors w, pushed by level d+1 (zero for the deepest);
+    // v pushes (1 + delta_j(v)) / s_j(v) to its predecessors u (j in M_{d-1}(u)); the masks of
+    // level d-2 are laid out for the next pass and those of level d cleared
     for (int d = depth - 1; d >= 1; d--) {
+        if (threadIdx.x < BCB_B) s_kexp[threadIdx.x] = kexp(b.maxb[(int64_t)d * BCB_B + threadIdx.x]);
         if (threadIdx.x == 0) {
             s_off[0] = b.loff[d];
             s_off[1] = b.loff[d + 1];
-            s_off[2] = b.loff[d + 2];
-            s_off[3] = d + 2 <= depth ? b.loff[d + 3] : 0ull;
+            s_off[2] = d >= 3 ? b.loff[d - 2] : 0ull;
+            s_off[3] = d >= 3 ? b.loff[d - 1] : 0ull;
         }
         __syncthreads();
-        uint32_t *Mn = b.M + (int64_t)((d + 1) & 1) * n;   // masks of L_{d+1}
-        uint32_t *Mo = b.M + (int64_t)(d & 1) * n;         // held L_{d+2}: cleared below
-        {
-            const unsigned long long a = s_off[1], e = s_off[2];
-            for (unsigned long long i = a + tid; i < e; i += nthr) Mn[b.lv[i]] = b.lm[i];
-        }
-        grid.sync();
-        if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[3] += t1 - t_mark; t_mark = t1; }
+        uint32_t *Mp = bcb_M(b, d - 1);   // predecessors' masks
+        uint32_t *Mc = bcb_M(b, d);       // this level's masks (read by the pass of d+1): cleared
+        uint32_t *Mq = bcb_M(b, d + 1);   // == M_{d-2}: set for the next pass
         {
             const unsigned long long a = s_off[0], e = s_off[1];
-            if (threadIdx.x < BCB_B) s_kexp[threadIdx.x] = kexp(b.maxb[(int64_t)d * BCB_B + threadIdx.x]);
-            __syncthreads();
             const int k = (int)(tid & (QUAD - 1));
-            const unsigned long long ncap = ((e - a) * QUAD + 31) / 32 * 32;   // warp-uniform trip count
-            for (unsigned long long ii = tid; ii < ncap; ii += nthr) {
-                const unsigned long long i = a + ii / QUAD;
-                const bool valid = i < e;
-                const int32_t v = valid ? b.lv[i] : 0;
-                const uint32_t m = valid ? b.lm[i] : 0u;
-                int64_t r0 = 0, r1 = 0;
-                if (valid) {
-                    r0 = __ldg(b.g.rp + v);
-                    r1 = __ldg(b.g.rp + v + 1);
-                }
-                // first two arcs of the thread and their successor masks hoisted out of the
-                // loop over sources (as in the forward sigma pass)
-                const int64_t ra = r0 + k;
-                const int32_t w0 = ra < r1 ? __ldg(b.g.col + ra) : 0;
-                const int32_t w1 = ra + QUAD < r1 ? __ldg(b.g.col + ra + QUAD) : 0;
-                const uint32_t g0 = ra < r1 ? vload(Mn + w0) & m : 0u;
-                const uint32_t g1 = ra + QUAD < r1 ? vload(Mn + w1) & m : 0u;
+            const bool push = d >= 2;     // level-0 vertices are sources: their delta is not used
+            for (unsigned long long i = a + tid / QUAD; i < e; i += nthr / QUAD) {
+                const int32_t v = b.lv[i];
+                const uint32_t m = b.lm[i];
+                const int64_t r1 = __ldg(b.g.rp + v + 1);
+                const int64_t ra = __ldg(b.g.rp + v) + k;
+                const int32_t u0 = push && ra < r1 ? __ldg(b.g.col + ra) : 0;
+                const int32_t u1 = push && ra + QUAD < r1 ? __ldg(b.g.col + ra + QUAD) : 0;
+                const uint32_t g0 = push && ra < r1 ? vload(Mp + u0) & m : 0u;
+                const uint32_t g1 = push && ra + QUAD < r1 ? vload(Mp + u1) & m : 0u;
                 double contrib = 0.0;
-                uint32_t mm = m;
-                while (__any_sync(0xffffffffu, mm != 0u)) {   // sources ascending: deterministic
-                    const int j = mm ? __ffs(mm) - 1 : 0;
-                    double acc = 0.0;
-                    if (mm) {
-                        if ((g0 >> j) & 1u) {
-                            const int64_t q = (int64_t)w0 * BCB_B + j;
-                            acc += (1.0 + b.delta[q]) / b.s[q];
-                        }
-                        if ((g1 >> j) & 1u) {
-                            const int64_t q = (int64_t)w1 * BCB_B + j;
-                            acc += (1.0 + b.delta[q]) / b.s[q];
-                        }
+                for (uint32_t mm = m; mm; mm &= mm - 1) {   // sources ascending: fixed order
+                    const int j = __ffs(mm) - 1;
+                    const int64_t q = (int64_t)v * BCB_B + j;
+                    const double sv = __ldcg(b.s + q);
+                    const double dv = ldexp(sv * __ldcg(b.delta + q), -s_kexp[j]);
+                    if (v != s_src[j]) contrib += dv;
+                    if (push) {
+                        const double t = (1.0 + dv) / sv;
+                        if ((g0 >> j) & 1u) atomicAdd(b.delta + (int64_t)u0 * BCB_B + j, t);
+                        if ((g1 >> j) & 1u) atomicAdd(b.delta + (int64_t)u1 * BCB_B + j, t);
                         for (int64_t r = ra + 2 * QUAD; r < r1; r += QUAD) {
-                            const int32_t w = __ldg(b.g.col + r);
-                            if ((vload(Mn + w) >> j) & 1u) {
-                                const int64_t q = (int64_t)w * BCB_B + j;
-                                acc += (1.0 + b.delta[q]) / b.s[q];
-                            }
+                            const int32_t u = __ldg(b.g.col + r);
+                            if ((vload(Mp + u) >> j) & 1u) atomicAdd(b.delta + (int64_t)u * BCB_B + j, t);
                         }
                     }
-#pragma unroll
-                    for (int o = 1; o < QUAD; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-                    if (mm && k == 0) {
-                        const double dv = ldexp(b.s[(int64_t)v * BCB_B + j] * acc, -s_kexp[j]);
-                        b.delta[(int64_t)v * BCB_B + j] = dv;
-                        if (v != s_src[j]) contrib += dv;
-                    }
-                    if (mm) mm &= mm - 1;
                 }
-                if (valid && k == 0 && m) b.bc[v] += contrib;
+                if (k == 0) {
+                    b.bc[v] += contrib;
+                    Mc[v] = 0u;
+                }
             }
-            if (d + 2 <= depth) {
-                const unsigned long long a2 = s_off[2], e2 = s_off[3];
-                for (unsigned long long i = a2 + tid; i < e2; i += nthr) Mo[b.lv[i]] = 0u;
-            }
+            const unsigned long long a2 = s_off[2], e2 = s_off[3];
+            for (unsigned long long i = a2 + tid; i < e2; i += nthr) Mq[b.lv[i]] = b.lm[i];
         }
         grid.sync();
         if (tid == 0) { const unsigned long long t1 = gtimer(); c->t_ns[4] += t1 - t_mark; t_mark = t1; }
     }
 }
 
-// reset the per-batch state for the next batch (entries of every level)
+// reset the per-batch masks and delta accumulators for the next batch (entries of every level;
+// whole arrays when the entries outnumber the vertices; full 32-B sectors either way: a partial
+// sector store would make L2 fetch the sector from HBM first)
 __global__ void k_bcb_reset(BcbView b) {
     BcbCtrl *c = b.c;
     unsigned long long top = c->ltop;
@@ -404,16 +392,18 @@ __global__ void k_bcb_reset(BcbView b) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t t0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (top > (unsigned long long)n / 2) {
-        // many entries (a vertex recurs once per source): zeroing the mask arrays whole is cheaper
-        // than scattering 6 stores per entry
+        // many entries (a vertex recurs once per source): zeroing the arrays whole is cheaper
+        // than scattering per entry
         uint32_t *arr[3] = {b.V, b.F, b.M};
-        const int64_t len[3] = {n, 3 * n, 2 * n};
+        const int64_t len[3] = {n, 3 * n, 3 * n};
         for (int a = 0; a < 3; a++) {
             uint32_t *p = arr[a];
             const int64_t nv = len[a] / 4;   // cudaMalloc'd: 256-B aligned
             for (int64_t i = t0; i < nv; i += stride) reinterpret_cast<uint4 *>(p)[i] = make_uint4(0, 0, 0, 0);
             for (int64_t i = nv * 4 + t0; i < len[a]; i += stride) p[i] = 0u;
         }
+        const int64_t nd = n * (BCB_B / 2);   // delta accumulators: 16 B per store
+        for (int64_t i = t0; i < nd; i += stride) reinterpret_cast<uint4 *>(b.delta)[i] = make_uint4(0, 0, 0, 0);
         top = 0;
     }
     for (unsigned long long i = t0; i < top; i += stride) {
@@ -424,6 +414,10 @@ __global__ void k_bcb_reset(BcbView b) {
         b.F[2 * n + v] = 0u;
         b.M[v] = 0u;
         b.M[n + v] = 0u;
+        b.M[2 * n + v] = 0u;
+        uint4 *row = reinterpret_cast<uint4 *>(b.delta + (int64_t)v * BCB_B);   // delta accumulators
+#pragma unroll
+        for (int q = 0; q < BCB_B / 2; q++) row[q] = make_uint4(0, 0, 0, 0);
     }
     int64_t levels = (int64_t)c->depth + 1;
     if (levels > b.cap + 1) levels = b.cap + 1;

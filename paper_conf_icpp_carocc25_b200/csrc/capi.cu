@@ -1162,7 +1162,7 @@ static int bcb_alloc(sg_graph *g) {
     B.lcap = n * 32;   // each (vertex, source) pair is in at most one level entry
     CK(cudaMalloc(&B.F, sizeof(uint32_t) * (size_t)n * 3));
     CK(cudaMalloc(&B.V, sizeof(uint32_t) * (size_t)n));
-    CK(cudaMalloc(&B.M, sizeof(uint32_t) * (size_t)n * 2));
+    CK(cudaMalloc(&B.M, sizeof(uint32_t) * (size_t)n * 3));
     CK(cudaMalloc(&B.s, sizeof(double) * (size_t)n * 32));
     CK(cudaMalloc(&B.delta, sizeof(double) * (size_t)n * 32));
     CK(cudaMalloc(&B.lv, sizeof(int32_t) * (size_t)B.lcap));
@@ -1177,7 +1177,8 @@ static int bcb_alloc(sg_graph *g) {
     CK(cudaMemset(B.VS, 0, sizeof(uint64_t) * (size_t)g->v.nw2));
     CK(cudaMemset(B.F, 0, sizeof(uint32_t) * (size_t)n * 3));
     CK(cudaMemset(B.V, 0, sizeof(uint32_t) * (size_t)n));
-    CK(cudaMemset(B.M, 0, sizeof(uint32_t) * (size_t)n * 2));
+    CK(cudaMemset(B.M, 0, sizeof(uint32_t) * (size_t)n * 3));
+    CK(cudaMemset(B.delta, 0, sizeof(double) * (size_t)n * 32));   // backward accumulators
     CK(cudaMemset(B.maxb, 0, sizeof(unsigned long long) * (size_t)(B.cap + 1) * 32));
     ws->bcb_ready = true;
     return SG_OK;
@@ -1204,7 +1205,17 @@ static int run_bc_batched(sg_graph *g, const int32_t *sources, int32_t k, double
         CK(bcb_run_batch(ws->bcb, s));
         CK(cudaMemcpyAsync(&c, ws->bcb.c, sizeof(BcbCtrl), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
-        if (c.overflow) return fail(SG_ERR_UNSUPPORTED, "batched BC: level/list capacity exceeded");
+        if (c.overflow) {
+            // entries past the list capacity were not recorded: clear every per-batch array
+            CK(cudaMemsetAsync(ws->bcb.delta, 0, sizeof(double) * (size_t)g->v.n * 32, s));
+            CK(cudaMemsetAsync(ws->bcb.F, 0, sizeof(uint32_t) * (size_t)g->v.n * 3, s));
+            CK(cudaMemsetAsync(ws->bcb.V, 0, sizeof(uint32_t) * (size_t)g->v.n, s));
+            CK(cudaMemsetAsync(ws->bcb.M, 0, sizeof(uint32_t) * (size_t)g->v.n * 3, s));
+            CK(cudaMemsetAsync(ws->bcb.VB, 0, sizeof(uint64_t) * (size_t)g->v.nw1, s));
+            CK(cudaMemsetAsync(ws->bcb.VS, 0, sizeof(uint64_t) * (size_t)g->v.nw2, s));
+            CK(cudaStreamSynchronize(s));
+            return fail(SG_ERR_UNSUPPORTED, "batched BC: level/list capacity exceeded");
+        }
         levels += c.depth;
         if (getenv("SG_TRACE"))
             fprintf(stderr, "[sygraph bc] batch %d: %d levels, %llu entries, phase ms fwdA %.2f fwdA2 %.2f fwdB %.2f bwdA %.2f bwdB %.2f\n",
