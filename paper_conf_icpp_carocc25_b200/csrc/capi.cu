@@ -116,6 +116,7 @@ struct sg_graph {
     int32_t *col = nullptr;
     uint8_t *w = nullptr;
     uint8_t *deg8 = nullptr;
+    int32_t *fnbr = nullptr;        // pull candidate per vertex
     uint64_t *isolated = nullptr;   // bit v <=> deg(v) == 0
     int32_t *hub_idx = nullptr;     // hub index of u (deg >= SEG_MIN) or -1
     int32_t *hub_vertex = nullptr;
@@ -308,6 +309,9 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     g->v.deg8 = g->deg8;
     CK(cudaMalloc(&g->isolated, sizeof(uint64_t) * (size_t)g->v.nw1));
     launch_isolated(g->deg8, n, g->v.nw1, g->isolated, s);
+    CK(cudaMalloc(&g->fnbr, sizeof(int32_t) * (size_t)(g->v.nw1 ? g->v.nw1 * 64 : 1)));   // padded: 16-B quad loads
+    launch_first_nbr(g->rp, g->col, g->deg8, n, g->v.nw1 * 64, g->fnbr, s);
+    g->v.fnbr = g->fnbr;
     unsigned long long *dscr = nullptr;
     CK(cudaMalloc(&dscr, 24));
     CK(cudaMemsetAsync(dscr, 0, 24, s));
@@ -349,6 +353,7 @@ SG_API int graph_free(sg_graph *g) {
     cudaFree(g->col);
     cudaFree(g->w);
     cudaFree(g->deg8);
+    cudaFree(g->fnbr);
     cudaFree(g->isolated);
     cudaFree(g->hub_idx);
     cudaFree(g->hub_vertex);

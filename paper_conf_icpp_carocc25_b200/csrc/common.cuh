@@ -17,6 +17,7 @@ struct GraphView {
     const int32_t *__restrict__ col;   // col_idx[nnz] (+16 B zero padding for 16-B bulk copies)
     const uint8_t *__restrict__ w;     // weights[nnz] or nullptr
     const uint8_t *__restrict__ deg8;  // 8-bit log-coded degrees, nw1*64 bytes (direction policy only)
+    const int32_t *__restrict__ fnbr;  // pull candidate: neighbour of largest degree among the first arcs, -1 if none
     int64_t n, nnz;
     int64_t nw1, nw2;
     const int32_t *__restrict__ hub_idx;   // hub index of u (deg >= SEG_MIN) or -1; nullptr: no segmentation

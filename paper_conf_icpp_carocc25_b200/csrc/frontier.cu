@@ -282,6 +282,43 @@ __global__ void k_deg8(const int64_t *__restrict__ rp, int64_t n, int64_t npad, 
         deg8[v] = (uint8_t)c;
     }
 }
+// Pull candidate of every vertex (graph load): the neighbour with the largest log-coded degree
+// among its first FNBR_SCAN arcs (first such in list order), -1 for an isolated vertex.  A
+// bottom-up BFS step tests it before the adjacency list: in a scale-free graph the large
+// frontiers that make pull steps worthwhile hold the hubs, so one dense 4-B read usually
+// replaces a row_ptr read plus a random col_idx sector.  Any choice is correct.
+constexpr int FNBR_SCAN = 64;
+__global__ void k_first_nbr(const int64_t *__restrict__ rp, const int32_t *__restrict__ col,
+                            const uint8_t *__restrict__ deg8, int64_t n, int64_t npad, int32_t *__restrict__ fn) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < npad; v += stride) {
+        if (v >= n) {
+            fn[v] = -1;
+            continue;
+        }
+        const int64_t s = rp[v];
+        int64_t e = rp[v + 1];
+        if (e > s + FNBR_SCAN) e = s + FNBR_SCAN;
+        int32_t best = -1;
+        int bd = -1;
+        for (int64_t r = s; r < e; r++) {
+            const int32_t u = __ldg(col + r);
+            if (u < 0 || (int64_t)u >= n) continue;   // unvalidated input: never index out of range
+            const int du = __ldg(deg8 + u);
+            if (du > bd) {
+                bd = du;
+                best = u;
+            }
+        }
+        fn[v] = best;
+    }
+}
+void launch_first_nbr(const int64_t *rp, const int32_t *col, const uint8_t *deg8, int64_t n, int64_t npad,
+                      int32_t *fn, cudaStream_t s) {
+    if (npad <= 0) return;
+    note_launch();
+    k_first_nbr<<<grid_for(npad, 256, 148 * 8), 256, 0, s>>>(rp, col, deg8, n, npad, fn);
+}
 void launch_isolated(const uint8_t *deg8, int64_t n, int64_t nw1, uint64_t *iso, cudaStream_t s) {
     note_launch();
     k_isolated<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(deg8, n, nw1, iso);

@@ -20,6 +20,8 @@ void launch_compact(const uint64_t *summ, int64_t nw2, uint32_t *offsets, DevSta
 void launch_frontier_stats(const GraphView &g, const uint64_t *bits, DevStats *st, cudaStream_t s);
 void launch_isolated(const uint8_t *deg8, int64_t n, int64_t nw1, uint64_t *iso, cudaStream_t s);
 void launch_deg8(const int64_t *rp, int64_t n, int64_t npad, uint8_t *deg8, cudaStream_t s);
+void launch_first_nbr(const int64_t *rp, const int32_t *col, const uint8_t *deg8, int64_t n, int64_t npad,
+                      int32_t *fn, cudaStream_t s);
 void launch_popcount(const uint64_t *bits, int64_t nw1, unsigned long long *out, cudaStream_t s);
 void launch_or_listed(const uint64_t *bits, const uint32_t *offsets, const DevStats *st, uint64_t *dst,
                       int64_t max_words, cudaStream_t s);

@@ -1,13 +1,22 @@
 // pull.cu — bottom-up (pull) BFS step for direction-optimising BFS (§3.4:
 // "it is also possible to use both push and pull techniques as per Beamer et al. [5]").
 //
-// Every unvisited vertex v scans N(v) (symmetric CSR = its in-neighbours, reading C8) and
-// stops at the first u that is in the input frontier (one bit test on the 2LB layer 1).
-// One warp owns one 64-bit word of the visited bitmap (lane l: vertices 64w+l and 64w+32+l),
-// so the new frontier word, the visited word and level[] are written without atomics; only
-// the summary bit is an atomicOr.  The two vertices of a lane are scanned in lock-step (two
-// independent load chains in flight per lane): the step is latency-bound, not bandwidth-bound.
-// Output identical to a push step from the same state (tested).
+// Every unvisited vertex v looks for a neighbour u in the input frontier (symmetric CSR: N(v)
+// = its in-neighbours, reading C8).  An unvisited vertex's visited neighbours are all in the
+// frontier (one at an earlier level would have reached v already), so any hit is a parent.
+//   1. candidate test: u = fnbr[v], the neighbour of largest degree among v's first arcs
+//      (graph load, frontier.cu): one bit test on the 2LB layer 1, no row_ptr / col_idx access.
+//      In the large scale-free frontiers where the policy pulls, the hubs are in the frontier
+//      and most vertices end here.
+//   2. a vertex whose candidate missed scans N(v) until its first frontier neighbour.
+// Mapping: one thread per quad of 4 consecutive vertices (16 threads = one 64-bit visited word),
+// no loop in the common path: the thread reads the visited word and, if one of its vertices is
+// unvisited, their 4 candidates with one 16-B load, then tests them (the only random reads, on
+// a 2 MB bitmap that stays in L2).  The 16 threads of a word OR their found bits together
+// (half-warp reduction), and one of them writes the new frontier word, the visited word and the
+// summary bit; level[] is written per found vertex.  The step is a streaming pass over the
+// visited bitmap and fnbr with enough independent threads in flight to cover the latency of
+// the dependent bit test.  Output identical to a push step from the same state.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -17,72 +26,81 @@ constexpr int PULL_THREADS = 256;
 #ifndef SG_PULL_ARCS
 #define SG_PULL_ARCS 2
 #endif
-#ifndef SG_PULL_MINB
-#define SG_PULL_MINB 6
-#endif
-constexpr int PULL_ARCS = SG_PULL_ARCS;   // arcs per vertex per iteration
+constexpr int PULL_ARCS = SG_PULL_ARCS;   // arcs in flight per step of a list scan
 
-__global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
+__global__ void __launch_bounds__(PULL_THREADS)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited,
            uint64_t *__restrict__ out_bits, uint64_t *__restrict__ out_summ, uint32_t *__restrict__ level,
            uint32_t next, DevStats *st, const uint32_t *next_ptr, uint32_t *const *level_pp) {
-    if (next_ptr) next = *next_ptr;
-    if (level_pp) level = *level_pp;
     __shared__ unsigned long long s_arcs[PULL_THREADS / 32];
     const int lane = lane_id();
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const uint32_t *in32 = reinterpret_cast<const uint32_t *>(in_bits);
+    const int64_t nq = g.nw1 * 16;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;   // multiple of 16: a word's quads stay in one half-warp
+    const uint32_t half = (lane < 16) ? 0x0000ffffu : 0xffff0000u;
     unsigned long long arcs = 0;
-    for (int64_t w = gw; w < g.nw1; w += nwarps) {
+    for (int64_t qd = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; qd < nq; qd += stride) {
+        const int64_t w = qd >> 4;
+        const int sh = (int)(qd & 15) * 4;
         const uint64_t vis = visited[w];
-        const int64_t rem = g.n - w * 64;
-        const uint64_t valid = rem >= 64 ? ~0ull : ((1ull << rem) - 1ull);
-        const uint64_t unv = ~vis & valid;
-        if (!unv) continue;
-        int64_t s[2], e[2];
-        word_bounds(g, w, unv, s[0], e[0], s[1], e[1]);
-        bool found[2] = {false, false};
-        // lock-step scan of both vertices' lists until each hits a frontier neighbour
-        while (s[0] < e[0] || s[1] < e[1]) {
-            int32_t c[2][PULL_ARCS];
+        const int64_t v0 = w * 64 + sh;
+        const int64_t rem = g.n - v0;
+        const uint32_t valid = rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
+        const uint32_t unv = (uint32_t)(~vis >> sh) & valid;
+        uint32_t found = 0;
+        if (unv) {
+            const int4 c4 = __ldg(reinterpret_cast<const int4 *>(g.fnbr + v0));
+            const int32_t c[4] = {c4.x, c4.y, c4.z, c4.w};
+            uint32_t x[4];
 #pragma unroll
-            for (int k = 0; k < 2; k++)
+            for (int k = 0; k < 4; k++) x[k] = ((unv >> k) & 1u) && c[k] >= 0 ? __ldg(in32 + (c[k] >> 5)) : 0u;
 #pragma unroll
-                for (int j = 0; j < PULL_ARCS; j++) c[k][j] = (s[k] + j < e[k]) ? __ldg(g.col + s[k] + j) : -1;
-            uint64_t x[2][PULL_ARCS];
-#pragma unroll
-            for (int k = 0; k < 2; k++)
-#pragma unroll
-                for (int j = 0; j < PULL_ARCS; j++) x[k][j] = c[k][j] >= 0 ? __ldg(in_bits + (c[k][j] >> 6)) : 0ull;
-#pragma unroll
-            for (int k = 0; k < 2; k++) {
-                if (s[k] >= e[k]) continue;
-                int used = 0;
-                bool hit = false;
-#pragma unroll
-                for (int j = 0; j < PULL_ARCS; j++) {
-                    if (!hit && c[k][j] >= 0) {
-                        used++;
-                        hit = (x[k][j] >> (c[k][j] & 63)) & 1ull;
-                    }
-                }
-                arcs += used;
-                if (hit) {
-                    found[k] = true;
-                    s[k] = e[k];
-                } else {
-                    s[k] += PULL_ARCS;
+            for (int k = 0; k < 4; k++) {
+                if (((unv >> k) & 1u) && c[k] >= 0) {
+                    arcs++;
+                    if ((x[k] >> (c[k] & 31)) & 1u) found |= 1u << k;
                 }
             }
+            // 2. list scans of the vertices whose candidate missed
+            for (uint32_t miss = unv & ~found; miss; miss &= miss - 1) {
+                const int k = __ffs(miss) - 1;
+                int64_t r = __ldg(g.rp + v0 + k);
+                const int64_t e = __ldg(g.rp + v0 + k + 1);
+                bool hit = false;
+                while (r < e && !hit) {
+                    int32_t u[PULL_ARCS];
+                    uint32_t y[PULL_ARCS];
+#pragma unroll
+                    for (int j = 0; j < PULL_ARCS; j++) u[j] = r + j < e ? __ldg(g.col + r + j) : -1;
+#pragma unroll
+                    for (int j = 0; j < PULL_ARCS; j++) y[j] = u[j] >= 0 ? __ldg(in32 + (u[j] >> 5)) : 0u;
+#pragma unroll
+                    for (int j = 0; j < PULL_ARCS; j++) {
+                        if (!hit && u[j] >= 0) {
+                            arcs++;
+                            hit = (y[j] >> (u[j] & 31)) & 1u;
+                        }
+                    }
+                    r += PULL_ARCS;
+                }
+                if (hit) found |= 1u << k;
+            }
         }
-        const uint32_t ba = __ballot_sync(0xffffffffu, found[0]), bb = __ballot_sync(0xffffffffu, found[1]);
-        const uint64_t nb = (uint64_t)ba | ((uint64_t)bb << 32);
-        if (found[0]) level[w * 64 + lane] = next;
-        if (found[1]) level[w * 64 + 32 + lane] = next;
-        if (nb && lane == 0) {
-            out_bits[w] = nb;
-            visited[w] = vis | nb;
-            atomic_or_u64(out_summ + (w >> 6), 1ull << (w & 63));
+        // the word's found bits: OR over the half-warp
+        const uint64_t mine = (uint64_t)found << sh;
+        const uint64_t nb = (uint64_t)__reduce_or_sync(half, (uint32_t)mine) |
+                            ((uint64_t)__reduce_or_sync(half, (uint32_t)(mine >> 32)) << 32);
+        if (nb) {
+            if (found) {
+                uint32_t *lvl = level_pp ? *level_pp : level;
+                const uint32_t nx = next_ptr ? *next_ptr : next;
+                for (uint32_t f = found; f; f &= f - 1) lvl[v0 + __ffs(f) - 1] = nx;
+            }
+            if ((lane & 15) == 0) {
+                out_bits[w] = nb;
+                visited[w] = vis | nb;
+                atomic_or_u64(out_summ + (w >> 6), 1ull << (w & 63));
+            }
         }
     }
     arcs = warp_sum(arcs);
@@ -98,8 +116,9 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
                      uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
                      const uint32_t *next_ptr, uint32_t *const *level_pp) {
-    int64_t blocks = (g.nw1 * 32 + PULL_THREADS - 1) / PULL_THREADS;
-    if (blocks > 148 * SG_PULL_MINB) blocks = 148 * SG_PULL_MINB;
+    // one thread per quad, no grid-stride loop up to 64 resident CTA waves
+    int64_t blocks = (g.nw1 * 16 + PULL_THREADS - 1) / PULL_THREADS;
+    if (blocks > 148 * 8 * 64) blocks = 148 * 8 * 64;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, out_bits, out_summ, level, next, st, next_ptr,
