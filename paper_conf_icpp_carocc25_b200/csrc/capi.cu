@@ -82,6 +82,7 @@ struct Workspace {
     DevStats *st = nullptr;        // 2 contiguous control blocks (fr[0].st, fr[1].st)
     DevStats *h_st = nullptr;      // pinned host mirror
     uint64_t *visited = nullptr;   // nw1 words
+    uint64_t *vis_old = nullptr;   // nw1 words: visited before the current BFS superstep (k_bfs_diff)
     uint32_t *all_offsets = nullptr;   // one-layer ablation: identity word list
     sg_frontier *far = nullptr;        // delta-stepping SSSP: far pile
     HeavyItem *heavy = nullptr;
@@ -165,6 +166,7 @@ static int ensure_ws(sg_graph *g) {
         ws->fr[i].st = ws->st + i;
     }
     CK(cudaMalloc(&ws->visited, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMalloc(&ws->vis_old, sizeof(uint64_t) * (size_t)g->v.nw1));
     CK(cudaMalloc(&ws->scratch, 8 * sizeof(unsigned long long)));
     CK(cudaMallocHost(&ws->h_scratch, 8 * sizeof(unsigned long long)));
     CK(cudaEventCreate(&ws->ev0));
@@ -199,6 +201,7 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->st);
     cudaFreeHost(ws->h_st);
     cudaFree(ws->visited);
+    cudaFree(ws->vis_old);
     cudaFree(ws->heavy);
     cudaFree(ws->seg);
     cudaFree(ws->all_offsets);
@@ -780,7 +783,8 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     }
     CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), cs));
     CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
-    launch_bfs_seed(ws->ctrl, F[0]->bits, F[0]->summ, ws->visited, cs);
+    CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
+    launch_bfs_seed(ws->ctrl, F[0]->bits, F[0]->summ, ws->visited, ws->vis_old, cs);
     launch_compact(F[0]->summ, G.nw2, F[0]->offsets, F[0]->st, cs);
     launch_frontier_stats(G, F[0]->bits, F[0]->st, cs);
     launch_bfs_decide(ws->ctrl, F[0]->st, nullptr, h_loop, h_push[0], h_pull[0], 1, cs);
@@ -798,18 +802,18 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         TRY(add_cond(body, deps, h_pull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
-        BfsArgs a{ws->visited, nullptr, 0u, out->bits, out->summ, &ws->ctrl->next, &ws->ctrl->level};
+        BfsArgs a{ws->visited, nullptr, 0u, nullptr, nullptr, &ws->ctrl->next, &ws->ctrl->level, 1u};
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
         TRY(capture_end(cs, leaves));
         TRY(capture_begin(cs, b_pull, {}));
-        launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, nullptr, 0u, in->st, cs, &ws->ctrl->next,
-                        &ws->ctrl->level);
+        launch_pull_bfs(G, in->bits, ws->visited, in->st, cs);
         TRY(capture_end(cs, leaves));
         TRY(capture_begin(cs, body, {n_push, n_pull}));
         launch_clear_listed(in->bits, in->summ, in->offsets, in->st, G.nw1, G.nw2, out->st, cs);
+        launch_bfs_diff(G, ws->visited, ws->vis_old, out->bits, out->summ, nullptr, 0u, &ws->ctrl->next,
+                        &ws->ctrl->level, out->st, cs);
         launch_compact(out->summ, G.nw2, out->offsets, out->st, cs);
-        launch_frontier_stats(G, out->bits, out->st, cs);
         launch_bfs_decide(ws->ctrl, out->st, in->st, h_loop, h_push[half ^ 1], h_pull[half ^ 1], 0, cs);
         TRY(capture_end(cs, deps));
     }
@@ -897,7 +901,8 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     TRY(clear_frontier(out, s));
     // visited starts as the isolated vertices (unreachable: level stays INF) plus src
     CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, s));
-    launch_seed(in->bits, in->summ, ws->visited, src, s);      // in = {src}, visited |= {src}
+    CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, s));
+    launch_seed(in->bits, in->summ, ws->visited, src, s, ws->vis_old);   // in = {src}, visited |= {src}
     const bool auto_dir = o.direction == SG_DIR_AUTO;
     static const bool trace = getenv("SG_TRACE") != nullptr;
     TRY(compact(g, in, true, s));
@@ -925,7 +930,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         const int64_t reached_before = reached;
         const int pr = prof_begin(ws, pull ? SG_K_PULL : SG_K_PUSH, s);
         if (pull) {
-            launch_pull_bfs(G, in->bits, ws->visited, out->bits, out->summ, level, d + 1, in->st, s);
+            launch_pull_bfs(G, in->bits, ws->visited, in->st, s);
             pull_steps++;
         } else {
             PushLaunch L = push_launch(g, in, t, o.one_layer ? G.nw1 : count);
@@ -935,31 +940,35 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
                 L.offsets = ws->all_offsets;
                 L.st = ws->st + 2;
             }
-            launch_push_bfs(L, BfsArgs{ws->visited, level, d + 1, out->bits, out->summ}, s);
+            BfsArgs a{ws->visited, level, d + 1, nullptr, nullptr};
+            a.diff = 1;
+            launch_push_bfs(L, a, s);
             push_steps++;
         }
         prof_end(ws, pr, s);
         TRY(clear_frontier(in, s));
         const int pc = prof_begin(ws, SG_K_COMPACT, s);
-        TRY(compact(g, out, true, s));
+        // output of the superstep: new = visited & ~vis_old -> out 2LB, level, n_f / m_f
+        CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
+        launch_bfs_diff(G, ws->visited, ws->vis_old, out->bits, out->summ, level, d + 1, nullptr, nullptr, out->st, s);
+        launch_compact(out->summ, G.nw2, out->offsets, out->st, s);
         prof_end(ws, pc, s);
         TRY(read_stats(ws, s));
         {
-            // algorithmic bytes of this step: col_idx 4 B/arc, row_ptr 16 B per
-            // expanded vertex, 8 B per input word, level 4 B + 8 B output word per new vertex/word
+            // algorithmic bytes of this step.  push: col_idx 4 B/arc, row_ptr 16 B
+            // per expanded vertex, 8 B per input word, 8 B per visited word updated; pull: 8 B per
+            // visited word read, 4 B per candidate / arc tested, 8 B per visited word updated;
+            // output pass (k_bfs_diff + compaction): visited and vis_old 16 B per word, level
+            // 4 B + degree code 1 B per new vertex, 16 B per output word + 4 B offset, summary
             const DevStats &ho = ws->h_st[in_idx ^ 1];
             const double n_new = (double)ho.nf, c_out = (double)ho.count;
             double bytes;
-            if (pull) {
-                const double unvisited = (double)(G.n - reached_before);
-                bytes = 4.0 * (double)ws->h_st[in_idx].arcs + 16.0 * unvisited + 8.0 * (double)G.nw1 +
-                        4.0 * n_new + 16.0 * c_out;
-            } else {
-                bytes = 4.0 * (double)ws->h_st[in_idx].arcs + 16.0 * (double)nf + 8.0 * (double)count + 4.0 * n_new +
-                        8.0 * c_out;
-            }
+            if (pull)
+                bytes = 8.0 * (double)G.nw1 + 4.0 * (double)ws->h_st[in_idx].arcs + 8.0 * c_out;
+            else
+                bytes = 4.0 * (double)ws->h_st[in_idx].arcs + 16.0 * (double)nf + 8.0 * (double)count + 8.0 * c_out;
             prof_bytes(ws, pr, bytes);
-            prof_bytes(ws, pc, 8.0 * (double)G.nw2 + 12.0 * c_out + 16.0 * n_new);
+            prof_bytes(ws, pc, 16.0 * (double)G.nw1 + 5.0 * n_new + 20.0 * c_out + 8.0 * (double)G.nw2);
         }
         if (pull) arcs_pulled += (int64_t)ws->h_st[in_idx].arcs;
         else arcs_pushed += (int64_t)ws->h_st[o.one_layer ? 2 : in_idx].arcs;

@@ -51,12 +51,13 @@ __global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *pre
 }
 
 // BFS prologue on the device: level[src] = 0, in = {src}, visited |= {src} (src, level from ctrl).
-__global__ void k_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited) {
+__global__ void k_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old) {
     const int32_t src = c->src;
     c->level[src] = 0u;
     bits[src >> 6] = 1ull << (src & 63);
     summ[src >> 12] = 1ull << ((src >> 6) & 63);
     visited[src >> 6] |= 1ull << (src & 63);
+    if (vis_old) vis_old[src >> 6] |= 1ull << (src & 63);
 }
 
 // Clear a frontier after it was advanced (only its listed non-zero words + its summary) and
@@ -102,9 +103,10 @@ void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, uns
     note_launch();
     k_bfs_decide<<<1, 32, 0, s>>>(c, st, prev, h_loop, h_push, h_pull, first);
 }
-void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, cudaStream_t s) {
+void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,
+                     cudaStream_t s) {
     note_launch();
-    k_bfs_seed<<<1, 1, 0, s>>>(c, bits, summ, visited);
+    k_bfs_seed<<<1, 1, 0, s>>>(c, bits, summ, visited, vis_old);
 }
 
 // level[0..n) = UINT32_MAX with the buffer pointer taken from ctrl (16-B stores)

@@ -204,10 +204,11 @@ __global__ void k_max_u8(const uint8_t *w, int64_t nnz, unsigned int *out) {
 }
 
 // in = {src} (both layers) and optionally visited = {src}; buffers were just cleared
-__global__ void k_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src) {
+__global__ void k_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, uint64_t *vis_old) {
     bits[src >> 6] = 1ull << (src & 63);
     summ[src >> 12] = 1ull << ((src >> 6) & 63);
     if (visited) visited[src >> 6] |= 1ull << (src & 63);
+    if (vis_old) vis_old[src >> 6] |= 1ull << (src & 63);
 }
 
 // bit v set iff deg(v) == 0: isolated vertices can never be reached, so BFS starts with them
@@ -344,9 +345,98 @@ void launch_set_u32(uint32_t *p, int64_t i, uint32_t v, cudaStream_t s) { note_l
 void launch_set_i32(int32_t *p, int64_t i, int32_t v, cudaStream_t s) { note_launch(); k_set_one<int32_t><<<1, 1, 0, s>>>(p, i, v); }
 void launch_set_f64(double *p, int64_t i, double v, cudaStream_t s) { note_launch(); k_set_one<double><<<1, 1, 0, s>>>(p, i, v); }
 
-void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, cudaStream_t s) {
+void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, cudaStream_t s,
+                 uint64_t *vis_old) {
     note_launch();
-    k_seed<<<1, 1, 0, s>>>(bits, summ, visited, src);
+    k_seed<<<1, 1, 0, s>>>(bits, summ, visited, src, vis_old);
+}
+
+// Output of a diff-mode BFS superstep (FnBfs::diff, pull.cu): the vertices first visited by
+// the step are new = visited & ~vis_old.  A warp reads 32 word pairs (one per lane, coalesced)
+// and skips the unchanged ones by ballot; the changed words are processed two at a time, one
+// per half-warp, one thread per quad of 4 vertices: the quad's level entries and degree codes,
+// the word's new bits written by the half-warp's first thread with the summary bit and vis_old.
+// n_f / m_f of the output frontier (direction policy) come out of the same pass.
+__global__ void __launch_bounds__(256) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited,
+                                                  uint64_t *__restrict__ vis_old, uint64_t *__restrict__ out_bits,
+                                                  uint64_t *__restrict__ out_summ, uint32_t *level, uint32_t next,
+                                                  const uint32_t *next_ptr, uint32_t *const *level_pp, DevStats *st) {
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int sh = (lane & 15) * 4;
+    unsigned long long nf = 0, mf = 0;
+    uint32_t *lvl = nullptr;
+    uint32_t nx = 0;
+    for (int64_t base = gw * 32; base < g.nw1; base += nwarps * 32) {
+        const int64_t wl = base + lane;
+        uint64_t nv = 0, ov = 0;
+        if (wl < g.nw1) {
+            nv = visited[wl];
+            ov = vis_old[wl];
+        }
+        uint32_t changed = __ballot_sync(0xffffffffu, nv != ov);
+        if (changed && !lvl) {
+            lvl = level_pp ? *level_pp : level;
+            nx = next_ptr ? *next_ptr : next;
+        }
+        while (changed) {
+            const int i0 = __ffs(changed) - 1;
+            changed &= changed - 1;
+            const int i1 = changed ? __ffs(changed) - 1 : -1;
+            if (i1 >= 0) changed &= changed - 1;
+            const int mi = lane < 16 ? i0 : i1;
+            const uint64_t wn = __shfl_sync(0xffffffffu, nv, mi < 0 ? 0 : mi);
+            const uint64_t wo = __shfl_sync(0xffffffffu, ov, mi < 0 ? 0 : mi);
+            if (mi < 0) continue;
+            const int64_t w = base + mi;
+            const uint64_t nb = wn & ~wo;
+            const uint32_t mine = (uint32_t)(nb >> sh) & 0xfu;
+            if (mine) {
+                const uint32_t codes = __ldg(reinterpret_cast<const uint32_t *>(g.deg8 + w * 64 + sh));
+                nf += __popc(mine);
+                for (uint32_t f = mine; f; f &= f - 1) {
+                    const int k = __ffs(f) - 1;
+                    lvl[w * 64 + sh + k] = nx;
+                    mf += deg8_decode((codes >> (8 * k)) & 0xffu);
+                }
+            }
+            if ((lane & 15) == 0) {
+                vis_old[w] = wn;
+                if (nb) {
+                    out_bits[w] = nb;
+                    atomic_or_u64(out_summ + (w >> 6), 1ull << (w & 63));
+                }
+            }
+        }
+    }
+    __shared__ unsigned long long s_mf[8], s_nf[8];
+    mf = warp_sum(mf);
+    nf = warp_sum(nf);
+    if (lane == 0) {
+        s_mf[threadIdx.x >> 5] = mf;
+        s_nf[threadIdx.x >> 5] = nf;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long a = 0, b = 0;
+        for (int i = 0; i < (int)(blockDim.x >> 5); i++) {
+            a += s_mf[i];
+            b += s_nf[i];
+        }
+        if (a | b) {
+            atomicAdd(&st->mf, a);
+            atomicAdd(&st->nf, b);
+        }
+    }
+}
+void launch_bfs_diff(const GraphView &g, const uint64_t *visited, uint64_t *vis_old, uint64_t *out_bits,
+                     uint64_t *out_summ, uint32_t *level, uint32_t next, const uint32_t *next_ptr,
+                     uint32_t *const *level_pp, DevStats *st, cudaStream_t s) {
+    note_launch();
+    k_bfs_diff<<<grid_for((g.nw1 + 31) / 32 * 32, 256, 148 * 16), 256, 0, s>>>(g, visited, vis_old, out_bits,
+                                                                             out_summ, level, next, next_ptr,
+                                                                             level_pp, st);
 }
 void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(p, n); }
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s) {

@@ -43,6 +43,9 @@ __device__ __forceinline__ void insert_batch(const OutSink &out, const int32_t (
 // atomicOr sets v's visited bit owns v, writes level[v] and inserts v.  A stale probe only
 // costs one extra atomic.  Result = {v unvisited before the step with a neighbour in the
 // frontier}, identical to the frozen-visited reading (R1).
+// diff mode (run_bfs): the arc only ORs v's visited bit, a fire-and-forget RED with no result
+// to wait for; k_bfs_diff then derives the output frontier, level[] and the frontier
+// statistics from visited & ~visited_before in one pass over the bitmap (same result set).
 struct FnBfs {
     static constexpr bool kWeights = false;
     static constexpr bool kSeg = true;      // hubs may take the destination-segmented tier
@@ -54,6 +57,7 @@ struct FnBfs {
     const uint32_t *next_ptr;   // device-driven loop: level value read at flip time (else `next`)
     uint32_t *const *level_pp;  // device-driven loop: output buffer pointer read at flip time (else `level`)
     OutSink out;
+    uint32_t diff;              // 1: mark visited only (k_bfs_diff builds the output)
     __device__ __forceinline__ Ctx ctx(int32_t) const { return 0u; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return ld_word(visited + (v >> 6)); }
     template <int K>
@@ -64,6 +68,12 @@ struct FnBfs {
         bool any = false;
 #pragma unroll
         for (int k = 0; k < K; k++) cand[k] = ok[k] && !((pr[k] >> (v[k] & 63)) & 1ull);
+        if (diff) {
+#pragma unroll
+            for (int k = 0; k < K; k++)
+                if (cand[k]) atomic_or_u64(visited + (v[k] >> 6), 1ull << (v[k] & 63));   // RED
+            return;
+        }
 #pragma unroll
         for (int k = 0; k < K; k++) old[k] = cand[k] ? atomic_or_u64(visited + (v[k] >> 6), 1ull << (v[k] & 63)) : ~0ull;
 #pragma unroll

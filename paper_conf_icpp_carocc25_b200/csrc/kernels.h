@@ -30,7 +30,8 @@ void launch_set_u32(uint32_t *p, int64_t i, uint32_t v, cudaStream_t s);
 void launch_set_i32(int32_t *p, int64_t i, int32_t v, cudaStream_t s);
 void launch_set_f64(double *p, int64_t i, double v, cudaStream_t s);
 void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s);
-void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, cudaStream_t s);
+void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, cudaStream_t s,
+                 uint64_t *vis_old = nullptr);
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s);
 void launch_max_weight(const uint8_t *w, int64_t nnz, unsigned int *out, cudaStream_t s);
 
@@ -62,6 +63,7 @@ struct BfsArgs {
     uint64_t *out_bits, *out_summ;
     const uint32_t *next_ptr = nullptr;    // graph mode: read `next` / `level` from BfsCtrl
     uint32_t *const *level_pp = nullptr;
+    uint32_t diff = 0;                     // 1: visited marks only; k_bfs_diff builds the output
 };
 struct SsspArgs { uint32_t *dist; uint64_t *out_bits, *out_summ; };
 struct CcArgs { int32_t *label; uint64_t *out_bits, *out_summ; };
@@ -73,10 +75,14 @@ void launch_push_bc(const PushLaunch &L, const BcArgs &a, cudaStream_t s);
 int push_max_grid_words();
 int push_max_grid_heavy();
 
-// pull.cu — bottom-up BFS step (direction-optimising, Beamer)
-void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
-                     uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
-                     const uint32_t *next_ptr = nullptr, uint32_t *const *level_pp = nullptr);
+// pull.cu — bottom-up BFS step (direction-optimising, Beamer): marks visited only,
+// k_bfs_diff builds the output frontier / level / statistics
+void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, cudaStream_t s);
+// frontier.cu — output of a diff-mode BFS superstep: new = visited & ~vis_old -> out 2LB,
+// level[new] = next, vis_old |= new, out->st n_f / m_f (st zeroed before)
+void launch_bfs_diff(const GraphView &g, const uint64_t *visited, uint64_t *vis_old, uint64_t *out_bits,
+                     uint64_t *out_summ, uint32_t *level, uint32_t next, const uint32_t *next_ptr,
+                     uint32_t *const *level_pp, DevStats *st, cudaStream_t s);
 
 // filter.cu — filter::inplace / external, compute::execute (Table 2)
 void launch_filter(const GraphView &g, const uint64_t *in_bits, uint64_t *out_bits, uint64_t *out_summ, int pred,
@@ -92,7 +98,8 @@ void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
                        unsigned long long h_push, unsigned long long h_pull, int first, cudaStream_t s);
-void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, cudaStream_t s);
+void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,
+                     cudaStream_t s);
 void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s);
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s);

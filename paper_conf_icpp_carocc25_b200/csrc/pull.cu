@@ -13,10 +13,11 @@
 // no loop in the common path: the thread reads the visited word and, if one of its vertices is
 // unvisited, their 4 candidates with one 16-B load, then tests them (the only random reads, on
 // a 2 MB bitmap that stays in L2).  The 16 threads of a word OR their found bits together
-// (half-warp reduction), and one of them writes the new frontier word, the visited word and the
-// summary bit; level[] is written per found vertex.  The step is a streaming pass over the
-// visited bitmap and fnbr with enough independent threads in flight to cover the latency of
-// the dependent bit test.  Output identical to a push step from the same state.
+// (half-warp reduction), and one of them writes the visited word; k_bfs_diff then derives the
+// output frontier, level[] and the statistics, as after a diff-mode push.  The step is a
+// streaming pass over the visited bitmap and fnbr with enough independent threads in flight to
+// cover the latency of the dependent bit test.  Output identical to a push step from the same
+// state.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -29,9 +30,7 @@ constexpr int PULL_THREADS = 256;
 constexpr int PULL_ARCS = SG_PULL_ARCS;   // arcs in flight per step of a list scan
 
 __global__ void __launch_bounds__(PULL_THREADS)
-k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited,
-           uint64_t *__restrict__ out_bits, uint64_t *__restrict__ out_summ, uint32_t *__restrict__ level,
-           uint32_t next, DevStats *st, const uint32_t *next_ptr, uint32_t *const *level_pp) {
+k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st) {
     __shared__ unsigned long long s_arcs[PULL_THREADS / 32];
     const int lane = lane_id();
     const uint32_t *in32 = reinterpret_cast<const uint32_t *>(in_bits);
@@ -90,18 +89,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
         const uint64_t mine = (uint64_t)found << sh;
         const uint64_t nb = (uint64_t)__reduce_or_sync(half, (uint32_t)mine) |
                             ((uint64_t)__reduce_or_sync(half, (uint32_t)(mine >> 32)) << 32);
-        if (nb) {
-            if (found) {
-                uint32_t *lvl = level_pp ? *level_pp : level;
-                const uint32_t nx = next_ptr ? *next_ptr : next;
-                for (uint32_t f = found; f; f &= f - 1) lvl[v0 + __ffs(f) - 1] = nx;
-            }
-            if ((lane & 15) == 0) {
-                out_bits[w] = nb;
-                visited[w] = vis | nb;
-                atomic_or_u64(out_summ + (w >> 6), 1ull << (w & 63));
-            }
-        }
+        if (nb && (lane & 15) == 0) visited[w] = vis | nb;
     }
     arcs = warp_sum(arcs);
     if (lane == 0) s_arcs[threadIdx.x >> 5] = arcs;
@@ -113,16 +101,13 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
     }
 }
 
-void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, uint64_t *out_bits,
-                     uint64_t *out_summ, uint32_t *level, uint32_t next, DevStats *st, cudaStream_t s,
-                     const uint32_t *next_ptr, uint32_t *const *level_pp) {
+void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, cudaStream_t s) {
     // one thread per quad, no grid-stride loop up to 64 resident CTA waves
     int64_t blocks = (g.nw1 * 16 + PULL_THREADS - 1) / PULL_THREADS;
     if (blocks > 148 * 8 * 64) blocks = 148 * 8 * 64;
     if (blocks < 1) blocks = 1;
     note_launch();
-    k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, out_bits, out_summ, level, next, st, next_ptr,
-                                                    level_pp);
+    k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st);
 }
 
 }  // namespace sg

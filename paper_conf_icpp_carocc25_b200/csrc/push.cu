@@ -57,6 +57,7 @@ void launch_push_bfs(const PushLaunch &L, const BfsArgs &a, cudaStream_t s) {
     f.next_ptr = a.next_ptr;
     f.level_pp = a.level_pp;
     f.out = OutSink{a.out_bits, a.out_summ};
+    f.diff = a.diff;
     launch_push(L, f, s);
 }
 void launch_push_sssp(const PushLaunch &L, const SsspArgs &a, cudaStream_t s) {

@@ -141,6 +141,10 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
             const int64_t w = w0 + i;
             const uint64_t nb = s_vis[i] & ~f.visited[w];
             if (!nb) continue;
+            if (f.diff) {   // k_bfs_diff builds the output
+                atomic_or_u64(f.visited + w, nb);
+                continue;
+            }
             const uint64_t old = atomic_or_u64(f.visited + w, nb);
             const uint64_t flips = nb & ~old;
             if (!flips) continue;
