@@ -44,6 +44,7 @@ def parse():
     p.add_argument("--alpha", type=float, default=14.0)
     p.add_argument("--beta", type=float, default=24.0)
     p.add_argument("--heavy-degree", type=int, default=0, help="CTA/grid-tier degree threshold (0: library default)")
+    p.add_argument("--scsr", type=int, default=0, help="segmented push advance: 0 auto, 1 off, 2 always")
     p.add_argument("--e2e-steps", type=int, default=3)
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -220,7 +221,8 @@ def main():
     G = sg.graph_load_csr(rp_h, ci_h)                     # host -> device copy (not timed)
     deg = torch.diff(rp_h.to(dev))
     direction = {"auto": sg.SG_DIR_AUTO, "push": sg.SG_DIR_PUSH, "pull": sg.SG_DIR_PULL}[args.direction]
-    o = sg.opts(stream=stream, direction=direction, alpha=args.alpha, beta=args.beta, heavy_degree=args.heavy_degree)
+    o = sg.opts(stream=stream, direction=direction, alpha=args.alpha, beta=args.beta, heavy_degree=args.heavy_degree,
+                 scsr=args.scsr)
     level = torch.empty(g.n, dtype=torch.int32, device=dev)
 
     # m_s per root (untimed; BFS results are deterministic per root)

@@ -82,7 +82,10 @@ typedef struct {
     int32_t coarsening;       /* push: layer-1 words per warp grab (CF); 0 = auto */
     int32_t sssp_delta;       /* run_sssp: 0 = frontier Bellman-Ford (the paper); D > 0 = near-far
                                  delta-stepping with bucket width D (P:161 refs [23,34]) */
-    int32_t reserved[3];
+    int32_t scsr;             /* run_bfs: heavy push supersteps over the destination-segmented arc copy
+                                 (visited slice in shared memory, built at the first run_bfs that can use
+                                 it, nnz x 4 B extra): 0 = auto (frontier arcs >= 4 Mi), 1 = off, 2 = always */
+    int32_t reserved[2];
 } sg_opts;
 
 typedef struct {

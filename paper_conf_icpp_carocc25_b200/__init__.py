@@ -35,7 +35,7 @@ class SgOpts(ctypes.Structure):
                 ("beta", ctypes.c_double), ("max_iters", ctypes.c_int64), ("heavy_degree", ctypes.c_int32),
                 ("small_degree", ctypes.c_int32), ("host_loop", ctypes.c_int32), ("segmented", ctypes.c_int32),
                 ("one_layer", ctypes.c_int32), ("coarsening", ctypes.c_int32), ("sssp_delta", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 3)]
+                ("scsr", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2)]
 
 
 class SgStats(ctypes.Structure):
@@ -155,15 +155,17 @@ def _ptr_mem(a):
 
 
 def opts(stream=None, direction=SG_DIR_AUTO, alpha=14.0, beta=24.0, max_iters=0, heavy_degree=0, small_degree=0,
-         host_loop=False, segmented=0, one_layer=False, coarsening=0, sssp_delta=0):
+         host_loop=False, segmented=0, one_layer=False, coarsening=0, sssp_delta=0, scsr=0):
     """segmented: BFS hub tier with the visited slice in shared memory (0 auto, 1 off, 2 always);
-    one_layer: ablation without the summary layer; coarsening: words per warp grab (0 auto)."""
+    one_layer: ablation without the summary layer; coarsening: words per warp grab (0 auto);
+    scsr: BFS heavy push over the destination-segmented arc copy (0 auto, 1 off, 2 always)."""
     o = SgOpts()
     load().sg_opts_default(ctypes.byref(o))
     o.stream = _stream_ptr(stream)
     o.direction, o.alpha, o.beta, o.max_iters = direction, alpha, beta, max_iters
     o.heavy_degree, o.small_degree, o.host_loop = heavy_degree, small_degree, int(host_loop)
     o.segmented, o.one_layer, o.coarsening, o.sssp_delta = segmented, int(one_layer), coarsening, sssp_delta
+    o.scsr = scsr
     return o
 
 

@@ -101,7 +101,7 @@ struct Workspace {
     cudaGraph_t bfs_graph = nullptr;
     cudaGraphExec_t bfs_exec = nullptr;
     uint32_t *bfs_level = nullptr;
-    int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1, bfs_cf = -1;
+    int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1, bfs_cf = -1, bfs_scsr = -1;
     SegItem *seg = nullptr;        // destination-segmented hub queue (BFS)
     uint32_t seg_cap = 0;
     // source-batched BC (bcb.cu)
@@ -123,6 +123,8 @@ struct sg_graph {
     int32_t *hub_vertex = nullptr;
     uint32_t *hub_off = nullptr;    // [nhubs][nseg+1] segment offsets within the hub's row
     int64_t nhubs = 0;
+    ScsrStore scsr;                 // destination-segmented copy of the arcs (BFS heavy push), built lazily
+    int scsr_state = 0;             // 0 not built, 1 built, -1 unavailable (segment block >= 2^32 arcs, unsorted rows)
     uint32_t max_w = 0;
     int device = 0;
     Workspace *ws = nullptr;
@@ -133,12 +135,12 @@ static const int32_t kDefaultSmall = 32;
 
 static int alloc_frontier_bufs(sg_frontier *f, const sg_graph *g, bool own_st) {
     f->g = g;
-    CK(cudaMalloc(&f->bits, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMalloc(&f->bits, sizeof(uint64_t) * (size_t)(g->v.nw1 + 8)));   // +8: 16-B bulk copies of a unit's tail
     CK(cudaMalloc(&f->summ, sizeof(uint64_t) * (size_t)g->v.nw2));
     CK(cudaMalloc(&f->offsets, sizeof(uint32_t) * (size_t)g->v.nw1));
     if (own_st) CK(cudaMalloc(&f->st, sizeof(DevStats)));
     f->owns_st = own_st;
-    CK(cudaMemset(f->bits, 0, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMemset(f->bits, 0, sizeof(uint64_t) * (size_t)(g->v.nw1 + 8)));
     CK(cudaMemset(f->summ, 0, sizeof(uint64_t) * (size_t)g->v.nw2));
     if (own_st) CK(cudaMemset(f->st, 0, sizeof(DevStats)));
     return SG_OK;
@@ -361,6 +363,7 @@ SG_API int graph_free(sg_graph *g) {
     cudaFree(g->hub_idx);
     cudaFree(g->hub_vertex);
     cudaFree(g->hub_off);
+    if (g->scsr_state == 1) scsr_free(&g->scsr);
     delete g;
     return SG_OK;
 }
@@ -554,7 +557,27 @@ struct Tiers {
     int32_t heavy, small;
     int32_t seg;   // destination-segmented hub tier for BFS: 0 off, 1 auto, 2 always
     int32_t cf;    // words per warp grab (coarsening factor); 0 = auto
+    int32_t scsr;  // BFS push over the segment-major arc copy: 0 off, 1 auto (m_f >= threshold), 2 always
 };
+// auto mode: the sweep (scsr.cu) takes a push superstep whose estimated frontier arcs reach
+// SG_SWEEP_FRAC64/64 of all arcs (it streams every arc of each active 4096-vertex unit, so it
+// pays only when most arcs are active); the copy is built only for graphs of at least
+// SG_SWEEP_MIN_M Mi arcs unless forced (scsr = 2)
+#ifndef SG_SWEEP_FRAC64
+#define SG_SWEEP_FRAC64 32
+#endif
+#ifndef SG_SWEEP_MIN_M
+#define SG_SWEEP_MIN_M 16
+#endif
+static unsigned long long env_or(const char *name, long long dflt) {
+    const char *e = getenv(name);
+    return (unsigned long long)(e ? atoll(e) : dflt);
+}
+static unsigned long long sweep_threshold(int64_t nnz) {
+    const unsigned long long f = env_or("SG_SWEEP_FRAC64", SG_SWEEP_FRAC64);
+    const unsigned long long t = (unsigned long long)nnz * f / 64ull;
+    return t ? t : 1ull;
+}
 // auto mode: the segmented tier pays for its per-segment slice loads only on heavy supersteps
 #ifndef SG_SEG_THRESHOLD_M
 #define SG_SEG_THRESHOLD_M 32
@@ -562,13 +585,14 @@ struct Tiers {
 static const unsigned long long kSegThreshold = (unsigned long long)SG_SEG_THRESHOLD_M << 20;   // est. frontier arcs
 
 static Tiers tiers_from(const sg_opts *o) {
-    Tiers t{kDefaultHeavy, kDefaultSmall, 1, 0};
+    Tiers t{kDefaultHeavy, kDefaultSmall, 1, 0, 1};
     if (o && o->coarsening > 0) t.cf = o->coarsening > 64 ? 64 : o->coarsening;
     if (o && o->heavy_degree > 0) t.heavy = o->heavy_degree;
     if (o && o->small_degree > 0) t.small = o->small_degree;
     if (o && o->small_degree < 0) t.small = 0;           // no thread tier
     if (t.small > t.heavy) t.small = t.heavy;
     if (o) t.seg = o->segmented == 1 ? 0 : (o->segmented == 2 ? 2 : 1);
+    if (o) t.scsr = o->scsr == 1 ? 0 : (o->scsr == 2 ? 2 : 1);
     return t;
 }
 
@@ -750,6 +774,26 @@ static int add_cond(cudaGraph_t graph, const std::vector<cudaGraphNode_t> &deps,
     return SG_OK;
 }
 
+// The segment-major arc copy (scsr.cu), built at the first run_bfs that may use it.  A graph
+// whose segment blocks would exceed 2^32 arcs, whose rows are not sorted, or for which the
+// memory is not available keeps the word path (the copy is a performance structure only).
+static bool scsr_ready(sg_graph *g, const Tiers &t, cudaStream_t s) {
+    if (t.scsr == 0) return false;
+    if (g->scsr_state == 0) {
+        if (t.scsr == 1 && (unsigned long long)g->v.nnz < (env_or("SG_SWEEP_MIN_M", SG_SWEEP_MIN_M) << 20))
+            return false;
+        const int32_t sw = (int32_t)env_or("SG_SCSR_WORDS", 0);   // test knob: narrower segments (0: 16,384 words)
+        const cudaError_t e = scsr_build(g->rp, g->col, g->v.n, g->v.nnz, sw, &g->scsr, s);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            g->scsr_state = -1;
+        } else {
+            g->scsr_state = 1;
+        }
+    }
+    return g->scsr_state == 1;
+}
+
 static int build_bfs_graph(sg_graph *g, Tiers t) {
     Workspace *ws = g->ws;
     const GraphView &G = g->v;
@@ -802,9 +846,13 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         TRY(add_cond(body, deps, h_pull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
+        const bool sc = t.scsr != 0 && g->scsr_state == 1;
+        const unsigned long long thr = t.scsr == 2 ? 0ull : sweep_threshold(G.nnz);
+        if (sc) L.skip_mf = thr;   // the word path stands down when the segmented advance runs
         BfsArgs a{ws->visited, nullptr, 0u, nullptr, nullptr, &ws->ctrl->next, &ws->ctrl->level, 1u};
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
+        if (sc) launch_push_sweep(g->scsr.v, in->bits, in->summ, G.nw2, in->st, ws->visited, thr, cs);
         TRY(capture_end(cs, leaves));
         TRY(capture_begin(cs, b_pull, {}));
         launch_pull_bfs(G, in->bits, ws->visited, in->st, cs);
@@ -822,6 +870,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     ws->bfs_small = t.small;
     ws->bfs_seg = t.seg;
     ws->bfs_cf = t.cf;
+    ws->bfs_scsr = t.scsr != 0 && g->scsr_state == 1 ? t.scsr : 0;
     return SG_OK;
 }
 
@@ -829,8 +878,9 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
                          sg_stats *stats) {
     Workspace *ws = g->ws;
     cudaStream_t s = stream_of(&o);
+    const int32_t sc_mode = t.scsr != 0 && g->scsr_state == 1 ? t.scsr : 0;
     if (!ws->bfs_exec || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small || ws->bfs_seg != t.seg ||
-        ws->bfs_cf != t.cf)
+        ws->bfs_cf != t.cf || ws->bfs_scsr != sc_mode)
         TRY(build_bfs_graph(g, t));
     BfsCtrl &c = *ws->h_ctrl;
     memset(&c, 0, sizeof c);
@@ -856,9 +906,11 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
     {
         // kernels the graph executed: prologue (seed, compact, stats, decide) + per WHILE body
-        // (2 x clear, compact, stats, decide) + the taken IF bodies (push = 2 kernels, pull = 1)
+        // (2 x clear, diff, compact, decide) + the taken IF bodies (push = word + CTA tier
+        // [+ hub segment tier] [+ segmented advance], pull = 1)
         const long long bodies = (long long)(c.iters + 1) / 2;
-        const long long k = 4 + 8 * bodies + 2 * (long long)c.push_steps + (long long)c.pull_steps;
+        const long long per_push = 2 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0) + (sc_mode ? 1 : 0);
+        const long long k = 4 + 8 * bodies + per_push * (long long)c.push_steps + (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }
     if (stats) {
@@ -892,6 +944,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
+    const bool scsr_on = !o.one_layer && scsr_ready(g, t, s);
     if (!ws->prof.on && !o.host_loop && !o.one_layer) return run_bfs_graph(g, src, level, o, t, max_iters, stats);
     CK(cudaEventRecord(ws->ev0, s));
     CK(cudaMemsetAsync(level, 0xFF, sizeof(uint32_t) * (size_t)G.n, s));
@@ -932,6 +985,9 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         if (pull) {
             launch_pull_bfs(G, in->bits, ws->visited, in->st, s);
             pull_steps++;
+        } else if (scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz))) {
+            launch_push_sweep(g->scsr.v, in->bits, in->summ, G.nw2, in->st, ws->visited, 0ull, s);
+            push_steps++;
         } else {
             PushLaunch L = push_launch(g, in, t, o.one_layer ? G.nw1 : count);
             if (o.one_layer) {   // Fig. 7 ablation: no summary layer, every word is visited

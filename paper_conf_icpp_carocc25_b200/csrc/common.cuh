@@ -25,6 +25,18 @@ struct GraphView {
     int32_t nseg;                          // ceil(n / SEG_V)
 };
 
+// Destination-segmented copy of the arcs (scsr.cu): segment b = vertices [b*sv, (b+1)*sv), sv =
+// 64*sw <= 2^20; block b = for u = 0..n-1 the arcs of u into segment b, each stored as
+// (u mod 4096) << 20 | (v - b*sv).
+struct ScsrView {
+    const uint32_t *__restrict__ col;    // tagged segment-major arcs (+64 B padding)
+    const uint32_t *__restrict__ base;   // [nseg][nw1+1] first arc of word w's parts, relative to start[b]
+    const int64_t *__restrict__ start;   // [nseg] first arc of block b
+    uint32_t *qc;                        // [nseg] work-item counters (zeroed before each advance)
+    int64_t nw1, sv;
+    int32_t nseg, sw;
+};
+
 // Per-superstep control block, device resident; host reads it back with one 64-B copy.
 struct DevStats {
     unsigned long long count;        // non-zero layer-1 words listed in offsets (summary compaction)

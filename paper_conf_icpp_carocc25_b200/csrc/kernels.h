@@ -51,6 +51,7 @@ struct PushLaunch {
     uint32_t seg_cap = 0;
     int32_t seg_mode = 0;            // 0 off, 1 auto, 2 always
     unsigned long long seg_threshold = 0;
+    unsigned long long skip_mf = ~0ull;   // k_push_words returns at once if the frontier's m_f >= skip_mf (SCSR path)
 };
 void launch_hub_mark(const int64_t *rp, int64_t n, int32_t *hub_idx, int32_t *hub_vertex, unsigned int *count,
                      cudaStream_t s);
@@ -94,6 +95,26 @@ void launch_min_over_bits(const GraphView &g, const uint64_t *bits, const uint32
 // pull_cc.cu — pull label-propagation step (dense CC supersteps)
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,
                     cudaStream_t s);
+
+// scsr.cu — destination-segmented copy of the arcs + the sweep advance (BFS, diff mode)
+struct ScsrStore {
+    ScsrView v{};
+    uint32_t *col = nullptr;
+    uint32_t *base = nullptr;
+    int64_t *start = nullptr;
+    uint32_t *qc = nullptr;
+    uint32_t nx = 0;        // vertices with a part >= 255 arcs (build statistics)
+    size_t bytes = 0;
+};
+// sw: slice words (<= 16,384; out of range = default).  cudaErrorInvalidValue: a segment block
+// would exceed 2^32 arcs or a row is not sorted (the caller keeps the word path).
+cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int32_t sw, ScsrStore *out,
+                       cudaStream_t s);
+void scsr_free(ScsrStore *S);
+// visited |= every neighbour of the input frontier's active vertices (zeroes v.qc first); runs
+// only if the frontier's m_f >= min_mf (0: always), so a CUDA graph can hold both push paths
+void launch_push_sweep(const ScsrView &v, const uint64_t *in_bits, const uint64_t *in_summ, int64_t nw2, DevStats *st,
+                       uint64_t *visited, unsigned long long min_mf, cudaStream_t s);
 
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,

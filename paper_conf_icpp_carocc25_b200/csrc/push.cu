@@ -21,6 +21,7 @@ static PushParams make_params(const PushLaunch &L) {
     p.seg_cap = L.seg_cap;
     p.seg_mode = L.seg_mode;
     p.seg_threshold = L.seg_threshold;
+    p.skip_mf = L.skip_mf;
     return p;
 }
 

@@ -47,6 +47,7 @@ struct PushParams {
     uint32_t seg_cap;
     int32_t seg_mode;      // 0 off, 1 auto (when the frontier's m_f >= seg_threshold), 2 always
     unsigned long long seg_threshold;
+    unsigned long long skip_mf;   // the segmented (SCSR) advance handles this superstep: m_f >= skip_mf
 };
 
 template <class F>
@@ -245,6 +246,7 @@ template <class F>
 __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) {
     __shared__ PushWarpSmem<F> s_warp[PUSH_WARPS];
     __shared__ unsigned long long s_arcs[PUSH_WARPS];
+    if (p.st->mf >= p.skip_mf) return;
     const uint32_t count = (uint32_t)p.st->count;
     const int wid = threadIdx.x >> 5;
     unsigned long long arcs = 0;

@@ -71,10 +71,13 @@ def test_config4_bfs_kron24_two_roots(sg, c4):
 def test_config4_push_only_matches(sg, c4):
     g, G = c4
     s = int(gen.config_sources(4, g)[5])
-    a, _ = sg.run_bfs(G, s, direction=sg.SG_DIR_PUSH)
+    a, sa = sg.run_bfs(G, s, direction=sg.SG_DIR_PUSH)             # heavy levels: segmented advance
+    c, sc = sg.run_bfs(G, s, direction=sg.SG_DIR_PUSH, scsr=1)     # word path only
     b, _ = sg.run_bfs(G, s)
     ref = oracle.bfs(g, s)
     assert np.array_equal(sg.as_u32(a), ref) and np.array_equal(sg.as_u32(b), ref)
+    assert np.array_equal(sg.as_u32(c), ref)
+    assert sa.arcs_pushed == sc.arcs_pushed                       # both inspect every reached vertex's arcs
 
 
 def test_config4_all_roots_bfs_invariants(sg, c4):

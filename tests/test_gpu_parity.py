@@ -233,6 +233,59 @@ def test_bfs_rmat16_many_sources(sg, direction):
         assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s)))
 
 
+# ------------------------------------------- destination-segmented (SCSR) push advance
+@pytest.mark.parametrize("sw", [0, 1, 3, 64])
+@pytest.mark.parametrize("host_loop", [False, True])
+def test_bfs_scsr_forced(sg, monkeypatch, sw, host_loop):
+    """Every push superstep through the segment-major arc copy (scsr=2) with segments of 64*sw
+    vertices (sw=0: the default 24,576 words, one segment here; sw=1: 256 segments of 64
+    vertices; sw=3: ragged last segment), push-only and direction-optimising."""
+    if sw:
+        monkeypatch.setenv("SG_SCSR_WORDS", str(sw))
+    for g in (gen.rmat(14, 16, permute=True), gen.rmat(12, 8)):
+        G = load(sg, g)
+        for s in list(gen.sources(g, 2)) + [int(np.argmax(g.degrees()))]:
+            for d in (sg.SG_DIR_PUSH, sg.SG_DIR_AUTO):
+                lv, _ = sg.run_bfs(G, int(s), direction=d, scsr=2, host_loop=host_loop)
+                assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (sw, s, d)
+
+
+@pytest.mark.parametrize("deg", [254, 255, 256, 511, 70_000])
+@pytest.mark.parametrize("sw", [0, 8])
+def test_bfs_scsr_part_length_escapes(sg, monkeypatch, deg, sw):
+    """Part lengths >= 255 arcs (a hub's neighbours inside one segment) take the exact offset
+    table: a star of degree `deg` plus a tail path, segments of 64*sw vertices."""
+    if sw:
+        monkeypatch.setenv("SG_SCSR_WORDS", str(sw))
+    n = deg + 1 + 50
+    u = np.concatenate([np.zeros(deg, np.int64), np.arange(deg, n - 1)])
+    v = np.concatenate([np.arange(1, deg + 1), np.arange(deg + 1, n)])
+    g = gen.from_edges(n, u, v)
+    G = load(sg, g)
+    for s in (0, 1, n - 1):
+        for hl in (False, True):
+            lv, _ = sg.run_bfs(G, s, direction=sg.SG_DIR_PUSH, scsr=2, host_loop=hl)
+            assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, s)), (deg, sw, s, hl)
+
+
+def test_bfs_scsr_auto_matches_word_path_multi_segment(sg, monkeypatch):
+    """Auto policy (sweep on supersteps with m_f >= nnz/8) with 8 segments (RMAT-17, 64*256-vertex
+    segments): scsr auto / off / always give identical levels and step counts."""
+    monkeypatch.setenv("SG_SCSR_WORDS", "256")
+    monkeypatch.setenv("SG_SWEEP_MIN_M", "0")
+    monkeypatch.setenv("SG_SWEEP_FRAC64", "8")
+    g = gen.rmat(17, 16, permute=True)
+    G = load(sg, g)
+    for s in gen.sources(g, 3):
+        ref = oracle.bfs(g, int(s))
+        stats = []
+        for mode in (0, 1, 2):
+            lv, st = sg.run_bfs(G, int(s), scsr=mode)
+            assert np.array_equal(sg.as_u32(lv), ref), mode
+            stats.append((st.iterations, st.push_steps, st.pull_steps, st.reached))
+        assert stats[0] == stats[1] == stats[2]
+
+
 # ---------------------------------------------------------------------- one advance step
 def test_single_bfs_advance_step_set_semantics(sg):
     import torch
