@@ -810,11 +810,13 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     cudaGraph_t root;
     CK(cudaGraphCreate(&root, 0));
     ws->bfs_graph = root;
-    cudaGraphConditionalHandle h_loop, h_push[2], h_pull[2];
+    cudaGraphConditionalHandle h_loop, h_push[2], h_pull[2], h_sweep[2];
+    const bool sc = t.scsr != 0 && g->scsr_state == 1;
     CK(cudaGraphConditionalHandleCreate(&h_loop, root, 0, cudaGraphCondAssignDefault));
     for (int i = 0; i < 2; i++) {
         CK(cudaGraphConditionalHandleCreate(&h_push[i], root, 0, cudaGraphCondAssignDefault));
         CK(cudaGraphConditionalHandleCreate(&h_pull[i], root, 0, cudaGraphCondAssignDefault));
+        if (sc) CK(cudaGraphConditionalHandleCreate(&h_sweep[i], root, 0, cudaGraphCondAssignDefault));
     }
     sg_frontier *F[2] = {&ws->fr[0], &ws->fr[1]};
     std::vector<cudaGraphNode_t> leaves;
@@ -831,7 +833,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     launch_bfs_seed(ws->ctrl, F[0]->bits, F[0]->summ, ws->visited, ws->vis_old, cs);
     launch_compact(F[0]->summ, G.nw2, F[0]->offsets, F[0]->st, cs);
     launch_frontier_stats(G, F[0]->bits, F[0]->st, cs);
-    launch_bfs_decide(ws->ctrl, F[0]->st, nullptr, h_loop, h_push[0], h_pull[0], 1, cs);
+    launch_bfs_decide(ws->ctrl, F[0]->st, nullptr, h_loop, h_push[0], h_pull[0], sc ? h_sweep[0] : 0ull, 1, cs);
     TRY(capture_end(cs, leaves));
     cudaGraphNode_t wnode;
     cudaGraph_t body;
@@ -844,25 +846,32 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         cudaGraph_t b_push, b_pull;
         TRY(add_cond(body, deps, h_push[half], cudaGraphCondTypeIf, &n_push, &b_push));
         TRY(add_cond(body, deps, h_pull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
+        cudaGraphNode_t n_sweep = nullptr;
+        cudaGraph_t b_sweep = nullptr;
+        if (sc) TRY(add_cond(body, deps, h_sweep[half], cudaGraphCondTypeIf, &n_sweep, &b_sweep));
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
-        const bool sc = t.scsr != 0 && g->scsr_state == 1;
-        const unsigned long long thr = t.scsr == 2 ? 0ull : sweep_threshold(G.nnz);
-        if (sc) L.skip_mf = thr;   // the word path stands down when the segmented advance runs
         BfsArgs a{ws->visited, nullptr, 0u, nullptr, nullptr, &ws->ctrl->next, &ws->ctrl->level, 1u};
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
-        if (sc) launch_push_sweep(g->scsr.v, in->bits, in->summ, G.nw2, in->st, ws->visited, thr, cs);
         TRY(capture_end(cs, leaves));
+        if (sc) {   // dense push supersteps (k_bfs_decide: m_f >= threshold) take the sweep instead
+            TRY(capture_begin(cs, b_sweep, {}));
+            launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, cs);
+            TRY(capture_end(cs, leaves));
+        }
         TRY(capture_begin(cs, b_pull, {}));
         launch_pull_bfs(G, in->bits, ws->visited, in->st, cs);
         TRY(capture_end(cs, leaves));
-        TRY(capture_begin(cs, body, {n_push, n_pull}));
+        std::vector<cudaGraphNode_t> ends{n_push, n_pull};
+        if (n_sweep) ends.push_back(n_sweep);
+        TRY(capture_begin(cs, body, ends));
         launch_clear_listed(in->bits, in->summ, in->offsets, in->st, G.nw1, G.nw2, out->st, cs);
         launch_bfs_diff(G, ws->visited, ws->vis_old, out->bits, out->summ, nullptr, 0u, &ws->ctrl->next,
                         &ws->ctrl->level, out->st, cs);
         launch_compact(out->summ, G.nw2, out->offsets, out->st, cs);
-        launch_bfs_decide(ws->ctrl, out->st, in->st, h_loop, h_push[half ^ 1], h_pull[half ^ 1], 0, cs);
+        launch_bfs_decide(ws->ctrl, out->st, in->st, h_loop, h_push[half ^ 1], h_pull[half ^ 1],
+                          sc ? h_sweep[half ^ 1] : 0ull, 0, cs);
         TRY(capture_end(cs, deps));
     }
     CK(cudaGraphInstantiate(&ws->bfs_exec, root, 0));
@@ -894,6 +903,8 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     c.pull = o.direction == SG_DIR_PULL;
     c.auto_dir = o.direction == SG_DIR_AUTO;
     c.reached = 1;
+    c.sweep_mode = (uint32_t)sc_mode;
+    c.sweep_thr = sweep_threshold(g->v.nnz);
     CK(cudaEventRecord(ws->ev0, s));
     CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, sizeof(BfsCtrl), cudaMemcpyHostToDevice, s));
     CK(cudaGraphLaunch(ws->bfs_exec, s));
@@ -909,8 +920,9 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         // (2 x clear, diff, compact, decide) + the taken IF bodies (push = word + CTA tier
         // [+ hub segment tier] [+ segmented advance], pull = 1)
         const long long bodies = (long long)(c.iters + 1) / 2;
-        const long long per_push = 2 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0) + (sc_mode ? 1 : 0);
-        const long long k = 4 + 8 * bodies + per_push * (long long)c.push_steps + (long long)c.pull_steps;
+        const long long per_push = 2 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
+        const long long k = 4 + 8 * bodies + per_push * (long long)(c.push_steps - c.sweep_steps) +
+                            2 * (long long)c.sweep_steps + (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }
     if (stats) {
@@ -986,7 +998,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
             launch_pull_bfs(G, in->bits, ws->visited, in->st, s);
             pull_steps++;
         } else if (scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz))) {
-            launch_push_sweep(g->scsr.v, in->bits, in->summ, G.nw2, in->st, ws->visited, 0ull, s);
+            launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, s);
             push_steps++;
         } else {
             PushLaunch L = push_launch(g, in, t, o.one_layer ? G.nw1 : count);

@@ -62,7 +62,9 @@ struct BfsCtrl {
     uint32_t pull;           // direction of the superstep being launched
     uint32_t auto_dir;
     uint32_t overflow;       // iteration cap hit
-    uint32_t pad;
+    uint32_t sweep_mode;     // push supersteps through the sweep: 0 never, 1 when m_f >= sweep_thr, 2 always
+    unsigned long long sweep_thr;
+    unsigned long long sweep_steps;
 };
 
 // Device-resident control of one source-batched BC batch (bcb.cu).

@@ -19,7 +19,8 @@ __device__ __forceinline__ void set_cond(unsigned long long h, unsigned v) {
 // `prev` (nullable) is the control block of the frontier just advanced: its arcs counter is
 // folded into the per-direction totals.
 __global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
-                             unsigned long long h_push, unsigned long long h_pull, int first) {
+                             unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep,
+                             int first) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     if (prev) {
         if (c->pull) c->arcs_pulled += prev->arcs;
@@ -45,7 +46,11 @@ __global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *pre
         else c->push_steps++;
         c->iters++;
     }
-    set_cond(h_push, go && !c->pull);
+    const bool push = go && !c->pull;
+    const bool sweep = push && (c->sweep_mode == 2 || (c->sweep_mode == 1 && st->mf >= c->sweep_thr));
+    if (sweep) c->sweep_steps++;
+    set_cond(h_push, push && !sweep);
+    set_cond(h_sweep, sweep);
     set_cond(h_pull, go && c->pull);
     set_cond(h_loop, go);
 }
@@ -99,9 +104,10 @@ __global__ void k_zero_u64(unsigned long long *p, int64_t n) {
 }
 
 void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
-                       unsigned long long h_push, unsigned long long h_pull, int first, cudaStream_t s) {
+                       unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep, int first,
+                       cudaStream_t s) {
     note_launch();
-    k_bfs_decide<<<1, 32, 0, s>>>(c, st, prev, h_loop, h_push, h_pull, first);
+    k_bfs_decide<<<1, 32, 0, s>>>(c, st, prev, h_loop, h_push, h_pull, h_sweep, first);
 }
 void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,
                      cudaStream_t s) {

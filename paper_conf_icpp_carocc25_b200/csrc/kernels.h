@@ -113,12 +113,14 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
 void scsr_free(ScsrStore *S);
 // visited |= every neighbour of the input frontier's active vertices (zeroes v.qc first); runs
 // only if the frontier's m_f >= min_mf (0: always), so a CUDA graph can hold both push paths
-void launch_push_sweep(const ScsrView &v, const uint64_t *in_bits, const uint64_t *in_summ, int64_t nw2, DevStats *st,
-                       uint64_t *visited, unsigned long long min_mf, cudaStream_t s);
+void launch_push_sweep(const ScsrView &v, const int64_t *rp, const uint64_t *in_bits, const uint64_t *in_summ,
+                       const uint32_t *offsets, int64_t nw2, DevStats *st, uint64_t *visited,
+                       unsigned long long min_mf, cudaStream_t s);
 
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
-                       unsigned long long h_push, unsigned long long h_pull, int first, cudaStream_t s);
+                       unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep, int first,
+                       cudaStream_t s);
 void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,
                      cudaStream_t s);
 void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s);

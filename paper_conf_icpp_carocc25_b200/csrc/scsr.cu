@@ -51,6 +51,9 @@ constexpr int SW_QUADS = SW_CONSUMERS * SW_QPT;  // quads per ring slot
 constexpr int SW_ACT_BYTES = 512;                // the unit's 64 input-frontier words, copied with the arcs
 constexpr int SW_SLOT_BYTES = SW_ACT_BYTES + SW_QUADS * 16;
 
+#ifndef SG_SW_NOPROBE
+#define SG_SW_NOPROBE 1   // 1: OR every active arc's bit without probing it first (measured faster: ATOMS beat LDS + branch)
+#endif
 #ifndef SG_SW_UNITS
 #define SG_SW_UNITS 16
 #endif
@@ -140,6 +143,39 @@ __global__ void k_scsr_xoff(const int64_t *__restrict__ rp, const int32_t *__res
             else hi = mid;
         }
         xoff[t] = (uint32_t)lo;
+    }
+}
+
+// Every (segment, unit) range is padded to a multiple of 4 arcs (16 B) so that ranges start and
+// end on 16-B boundaries: the sweep's slots then hold whole quads.  The pad is added to the
+// unit's last word; k_scsr_padfill fills it with copies of the range's first arc (idempotent).
+__global__ void k_scsr_pad(unsigned long long *__restrict__ wsum, int64_t nw1, int64_t nw2, int nseg,
+                           uint8_t *__restrict__ upad, unsigned long long *total_pad) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nw2 * nseg; t += stride) {
+        const int64_t b = t / nw2, u = t % nw2;
+        unsigned long long *ws = wsum + (size_t)b * nw1;
+        const int64_t w0 = u * 64, w1 = min(nw1, w0 + 64);
+        unsigned long long real = 0;
+        for (int64_t w = w0; w < w1; w++) real += ws[w];
+        const uint32_t pad = (uint32_t)((4u - (uint32_t)(real & 3u)) & 3u);
+        upad[t] = (uint8_t)pad;
+        if (pad) {
+            ws[w1 - 1] += pad;
+            atomicAdd(total_pad, (unsigned long long)pad);
+        }
+    }
+}
+__global__ void k_scsr_padfill(const uint8_t *__restrict__ upad, ScsrView s, int64_t nw2, uint32_t *__restrict__ scol) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nw2 * s.nseg; t += stride) {
+        const uint32_t pad = upad[t];
+        if (!pad) continue;
+        const int64_t b = t / nw2, u = t % nw2;
+        const uint32_t *base = s.base + (size_t)b * (s.nw1 + 1);
+        const int64_t lo = s.start[b] + base[u * 64], hi = s.start[b] + base[min(u * 64 + 64, s.nw1)];
+        const uint32_t first = scol[lo];
+        for (uint32_t i = 1; i <= pad; i++) scol[hi - i] = first;
     }
 }
 
@@ -330,7 +366,6 @@ __global__ void __launch_bounds__(SW_THREADS, 1) k_push_sweep(SweepParams p) {
     uint64_t *s_vis = reinterpret_cast<uint64_t *>(sw_smem + (size_t)SW_STAGES * SW_SLOT_BYTES);
     __shared__ SwRec s_rec[SW_STAGES];
     __shared__ __align__(8) uint64_t s_full[SW_STAGES], s_empty[SW_STAGES];
-    __shared__ unsigned long long s_arcs[SW_THREADS / 32];
     __shared__ SwTask s_task[SW_TASKS];
     __shared__ uint32_t s_thead, s_ttail;
     if (p.min_mf && p.st->mf < p.min_mf) return;
@@ -346,7 +381,6 @@ __global__ void __launch_bounds__(SW_THREADS, 1) k_push_sweep(SweepParams p) {
         s_thead = s_ttail = 0;
     }
     __syncthreads();
-    unsigned long long arcs = 0;
     if (warp == 1) {
         // ---------------- scheduler: items -> active unit ranges ----------------
         // grabs work items (segment, SW_UNITS units), loads their summary words and block
@@ -423,19 +457,17 @@ __global__ void __launch_bounds__(SW_THREADS, 1) k_push_sweep(SweepParams p) {
                 }
                 // the unit's layer-1 words (16-B multiple; frontier buffers carry 8 words of padding)
                 const uint32_t act_bytes = (uint32_t)(((min((int64_t)64, S.nw1 - (int64_t)t.u * 64) + 1) & ~1ll) * 8);
-                // slots hold whole 16-B-aligned quads: after the first, every chunk of the range
-                // starts aligned and all but the last fill the slot exactly (no masking)
+                // ranges are padded to whole quads and start 16-B aligned (k_scsr_pad): every slot
+                // but a range's last is full
                 for (int64_t c = t.lo; c < t.hi;) {
-                    const int64_t a0 = c & ~3ll;
-                    const int64_t nx = min(t.hi, a0 + (int64_t)SW_QUADS * 4);
+                    const int64_t nx = min(t.hi, c + (int64_t)SW_QUADS * 4);
                     const uint32_t n = (uint32_t)(nx - c);
-                    const int64_t a1 = (nx + 3) & ~3ll;
-                    const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
-                    const int s = slot(SW_DATA, n, (uint32_t)(c - a0), t.u);
+                    const uint32_t bytes = n * 4u;
+                    const int s = slot(SW_DATA, n, 0u, t.u);
                     unsigned char *dst = sw_smem + (size_t)s * SW_SLOT_BYTES;
                     sw_mbar_arrive_tx(s_full + s, bytes + act_bytes);
                     sw_bulk_g2s(dst, p.in_bits + (int64_t)t.u * 64, act_bytes, s_full + s);
-                    sw_bulk_g2s(dst + SW_ACT_BYTES, S.col + a0, bytes, s_full + s);
+                    sw_bulk_g2s(dst + SW_ACT_BYTES, S.col + c, bytes, s_full + s);
                     c = nx;
                 }
             }
@@ -473,7 +505,6 @@ __global__ void __launch_bounds__(SW_THREADS, 1) k_push_sweep(SweepParams p) {
                 const unsigned char *slot_p = sw_smem + (size_t)s * SW_SLOT_BYTES;
                 const uint32_t *act32 = reinterpret_cast<const uint32_t *>(slot_p);
                 const uint4 *qs = reinterpret_cast<const uint4 *>(slot_p + SW_ACT_BYTES);
-                const uint32_t end = r.skew + r.n;
                 uint4 q[SW_QPT];
 #pragma unroll
                 for (int h = 0; h < SW_QPT; h++) {
@@ -495,30 +526,27 @@ __global__ void __launch_bounds__(SW_THREADS, 1) k_push_sweep(SweepParams p) {
 #pragma unroll
                 for (int j = 0; j < NA; j++) {
                     aw[j] = act32[v[j] >> 25];
+#if !SG_SW_NOPROBE
                     vw[j] = s_vis32[(v[j] >> 10) & 0x7fffu];
+#endif
                 }
-                // quads straddling [skew, end) (a range's first and last slot only): lanes outside
-                // get a zero activity word
+                // ranges are padded to whole quads: only quads past the slot's end are masked
 #pragma unroll
-                for (int h = 0; h < SW_QPT; h++) {
-                    const int i0 = (h * SW_CONSUMERS + ct) * 4;
-                    const int lo = (int)r.skew - i0, hi = (int)end - i0;   // valid lanes: [lo, hi)
-                    if (lo > 0 || hi < 4) {
+                for (int h = 0; h < SW_QPT; h++)
+                    if ((uint32_t)(h * SW_CONSUMERS + ct) * 4 >= r.n)
 #pragma unroll
-                        for (int j = 0; j < 4; j++)
-                            if (j < lo || j >= hi) aw[4 * h + j] = 0u;
-                    }
-                }
-                uint32_t cnt = 0;
+                        for (int j = 0; j < 4; j++) aw[4 * h + j] = 0u;
 #pragma unroll
                 for (int j = 0; j < NA; j++) {
                     const uint32_t a = __funnelshift_r(aw[j], 0u, v[j]);          // bit 0: source active
                     const uint32_t db = v[j] >> 5;                                 // low 5 bits: destination bit
+#if SG_SW_NOPROBE
+                    if (a & 1u) atomicOr(s_vis32 + ((v[j] >> 10) & 0x7fffu), __funnelshift_l(0u, 1u, db));
+#else
                     const uint32_t d = __funnelshift_r(vw[j], 0u, db);             // bit 0: destination visited
-                    cnt += a & 1u;
                     if ((a & ~d) & 1u) atomicOr(s_vis32 + ((v[j] >> 10) & 0x7fffu), __funnelshift_l(0u, 1u, db));
+#endif
                 }
-                arcs += cnt;
             }
             __syncwarp();
             if (lane == 0) sw_mbar_arrive(s_empty + s);
@@ -526,13 +554,41 @@ __global__ void __launch_bounds__(SW_THREADS, 1) k_push_sweep(SweepParams p) {
         consumer_sync();
         if (loaded >= 0) flush();
     }
-    arcs = warp_sum(arcs);
-    if (lane == 0) s_arcs[warp] = arcs;
+}
+
+// The statistics of a sweep step: the exact sum of the input frontier's degrees (the arcs a push
+// step inspects, as the word path counts them), one thread per listed word, 4 row_ptr pairs in
+// flight per iteration.
+__global__ void __launch_bounds__(256) k_frontier_arcs(const int64_t *__restrict__ rp, const uint64_t *__restrict__ in_bits,
+                                                       const uint32_t *__restrict__ offsets, DevStats *st,
+                                                       unsigned long long min_mf) {
+    __shared__ unsigned long long s_a[8];
+    if (min_mf && st->mf < min_mf) return;
+    const uint32_t count = (uint32_t)st->count;
+    unsigned long long acc = 0;
+    const uint32_t stride = gridDim.x * blockDim.x;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) {
+        const int64_t w = offsets[i];
+        uint64_t x = __ldg(in_bits + w);
+        while (x) {
+            int64_t v[4];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                v[k] = x ? w * 64 + (__ffsll((long long)x) - 1) : -1;
+                x &= x - 1;
+            }
+#pragma unroll
+            for (int k = 0; k < 4; k++)
+                if (v[k] >= 0) acc += (unsigned long long)(__ldg(rp + v[k] + 1) - __ldg(rp + v[k]));
+        }
+    }
+    acc = warp_sum(acc);
+    if (lane_id() == 0) s_a[threadIdx.x >> 5] = acc;
     __syncthreads();
     if (threadIdx.x == 0) {
         unsigned long long t = 0;
-        for (int i = 0; i < SW_THREADS / 32; i++) t += s_arcs[i];
-        if (t) atomicAdd(&p.st->arcs, t);
+        for (int i = 0; i < 8; i++) t += s_a[i];
+        if (t) atomicAdd(&st->arcs, t);
     }
 }
 
@@ -571,6 +627,9 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
     std::vector<unsigned long long> h(nseg + 1);
     std::vector<int64_t> start(nseg);
     unsigned int nx = 0, bad = 0;
+    unsigned long long tpad = 0;
+    uint8_t *upad = nullptr;
+    const int64_t nw2 = (nw1 + 63) / 64;
     int64_t acc = 0;
     bool too_big = false;
     const int64_t max_x = nnz / 255 + 1;
@@ -591,10 +650,19 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
         k_scsr_count<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(rp, col, n, npad, nw1, nseg, sv, cnt, wsum, xidx,
                                                                     xvert, nx_d);
     }
+    SCK(cudaMalloc(&upad, (size_t)nseg * nw2));
+    {
+        int64_t bl = (nseg * nw2 + 255) / 256;
+        if (bl > sm_count() * 8) bl = sm_count() * 8;
+        note_launch();
+        k_scsr_pad<<<(int)(bl < 1 ? 1 : bl), 256, 0, s>>>(wsum, nw1, nw2, nseg, upad,
+                                                           reinterpret_cast<unsigned long long *>(nx_d + 2));
+    }
     SCK(cudaMalloc(&S.base, sizeof(uint32_t) * (size_t)nseg * (nw1 + 1)));
     note_launch();
     k_scsr_scan<<<nseg, 1024, 0, s>>>(wsum, nw1, S.base, tot);
     SCK(cudaMemcpyAsync(&nx, nx_d, sizeof(unsigned int), cudaMemcpyDeviceToHost, s));
+    SCK(cudaMemcpyAsync(&tpad, nx_d + 2, sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
     SCK(cudaMemcpyAsync(h.data(), tot, sizeof(unsigned long long) * nseg, cudaMemcpyDeviceToHost, s));
     SCK(cudaStreamSynchronize(s));
     SCK(cudaGetLastError());
@@ -603,7 +671,7 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
         acc += (int64_t)h[b];
         too_big |= h[b] >= 0xffffffffull;
     }
-    if (too_big || acc != nnz) {   // segment block >= 2^32 arcs, or ids outside [0, n)
+    if (too_big || acc != nnz + (int64_t)tpad) {   // segment block >= 2^32 arcs, or ids outside [0, n)
         e = cudaErrorInvalidValue;
         goto done;
     }
@@ -618,8 +686,8 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
         note_launch();
         k_scsr_xoff<<<(int)bl, 256, 0, s>>>(rp, col, xvert, nx, nseg, sv, xoff);
     }
-    SCK(cudaMalloc(&S.col, sizeof(uint32_t) * (size_t)nnz + 64));
-    SCK(cudaMemsetAsync((char *)S.col + sizeof(uint32_t) * (size_t)nnz, 0, 64, s));
+    SCK(cudaMalloc(&S.col, sizeof(uint32_t) * (size_t)acc + 64));
+    SCK(cudaMemsetAsync((char *)S.col + sizeof(uint32_t) * (size_t)acc, 0, 64, s));
     SCK(cudaMalloc(&S.qc, sizeof(uint32_t) * (size_t)nseg));
     S.v.col = S.col;
     S.v.base = S.base;
@@ -631,12 +699,16 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
         SCK(cudaMemsetAsync(nx_d, 0, sizeof(unsigned int), s));
         note_launch();
         k_scsr_fill<<<(int)(bl < 1 ? 1 : bl), 256, 0, s>>>(rp, col, n, S.v, ScsrBuild{cnt, xidx, xoff}, S.col, nx_d);
+        int64_t bp = (nseg * nw2 + 255) / 256;
+        if (bp > sm_count() * 8) bp = sm_count() * 8;
+        note_launch();
+        k_scsr_padfill<<<(int)(bp < 1 ? 1 : bp), 256, 0, s>>>(upad, S.v, nw2, S.col);
     }
     SCK(cudaMemcpyAsync(&bad, nx_d, sizeof(unsigned int), cudaMemcpyDeviceToHost, s));
     SCK(cudaStreamSynchronize(s));
     SCK(cudaGetLastError());
     if (bad) e = cudaErrorInvalidValue;   // unsorted rows: keep the word path
-    S.bytes = sizeof(uint32_t) * (size_t)nnz + sizeof(uint32_t) * (size_t)nseg * (nw1 + 1);
+    S.bytes = sizeof(uint32_t) * (size_t)acc + sizeof(uint32_t) * (size_t)nseg * (nw1 + 1);
 done:
 #undef SCK
     cudaFree(cnt);
@@ -645,6 +717,7 @@ done:
     cudaFree(xvert);
     cudaFree(xoff);
     cudaFree(nx_d);
+    cudaFree(upad);
     if (e != cudaSuccess) scsr_free(out);
     return e;
 }
@@ -657,8 +730,9 @@ void scsr_free(ScsrStore *S) {
     *S = ScsrStore{};
 }
 
-void launch_push_sweep(const ScsrView &v, const uint64_t *in_bits, const uint64_t *in_summ, int64_t nw2, DevStats *st,
-                       uint64_t *visited, unsigned long long min_mf, cudaStream_t s) {
+void launch_push_sweep(const ScsrView &v, const int64_t *rp, const uint64_t *in_bits, const uint64_t *in_summ,
+                       const uint32_t *offsets, int64_t nw2, DevStats *st, uint64_t *visited,
+                       unsigned long long min_mf, cudaStream_t s) {
     static bool attr = false;
     // the whole 128 KB slice is always allocated: masked lanes may probe any 15-bit word index
     const size_t smem = (size_t)SW_STAGES * SW_SLOT_BYTES + (size_t)SCSR_MAX_SW * sizeof(uint64_t);
@@ -678,6 +752,8 @@ void launch_push_sweep(const ScsrView &v, const uint64_t *in_bits, const uint64_
     cudaMemsetAsync(v.qc, 0, sizeof(uint32_t) * (size_t)v.nseg, s);
     note_launch();
     k_push_sweep<<<sm_count(), SW_THREADS, smem, s>>>(p);
+    note_launch();
+    k_frontier_arcs<<<sm_count() * 8, 256, 0, s>>>(rp, in_bits, offsets, st, min_mf);
 }
 
 }  // namespace sg
