@@ -46,6 +46,7 @@ def parse():
     p.add_argument("--heavy-degree", type=int, default=0, help="CTA/grid-tier degree threshold (0: library default)")
     p.add_argument("--scsr", type=int, default=0, help="segmented push advance: 0 auto, 1 off, 2 always")
     p.add_argument("--e2e-steps", type=int, default=3)
+    p.add_argument("--dense-roots", type=int, default=3, help="push-only BFS roots for roofline_dense_push (0: skip)")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--no-cpu-baseline", action="store_true")
     return p.parse_args()
@@ -292,6 +293,40 @@ def main():
                                 "GBps": (v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] else 0.0}
                             for k, v in prof.items()}}
 
+    # ---- the north star's HBM bar: the dense top-down advance (direction optimisation off) ----
+    # push-only BFS over a few of the same roots, host-driven with per-class events; the dense
+    # supersteps go through the destination-segmented sweep (class advance_sweep)
+    dense = None
+    if args.direction != "pull" and args.dense_roots > 0:
+        od = sg.opts(stream=stream, direction=sg.SG_DIR_PUSH, heavy_degree=args.heavy_degree, scsr=args.scsr)
+        d_roots = [int(roots[i % len(roots)]) for i in range(args.dense_roots)]
+        sg.profile(G, True)
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        q0.record(stream)
+        for s in d_roots:
+            sg.run_bfs(G, s, level, od)
+        q1.record(stream)
+        torch.cuda.synchronize()
+        dprof = sg.profile_read(G)
+        sg.profile(G, False)
+        ms_d = q0.elapsed_time(q1)
+        for s in d_roots:
+            if s not in ms_of:
+                sg.run_bfs(G, s, level, o)
+                ms_of[s] = m_s_of(level, deg)
+        D = dprof.get("advance_sweep", {"launches": 0})
+        if D["launches"]:
+            ach = (D["bytes"] / D["launches"]) / (D["ms"] / D["launches"] / 1e3) / 1e9
+            dense = {"bound": "hbm", "kernel": "k_push_sweep (advance_sweep)", "achieved": ach, "peak": peak,
+                     "unit": "GB/s", "frac": ach / peak, "peak_source": peak_src,
+                     "traffic": (tr or {}).get("advance_sweep", {}).get("dram_bytes_per_launch") if tr else None,
+                     "ncu_dram_pct_of_peak": (tr or {}).get("advance_sweep", {}).get("ncu_dram_pct_of_peak") if tr else None,
+                     "bytes_per_launch": D["bytes"] / D["launches"], "ms_per_launch": D["ms"] / D["launches"],
+                     "launches": D["launches"], "share_of_step": D["ms"] / ms_d if ms_d else None,
+                     "push_only_gteps_host_loop": sum(ms_of[s] for s in d_roots) / (ms_d / 1e3) / 1e9,
+                     "measured_in": f"push-only BFS (direction optimisation off) from {len(d_roots)} of the roots, "
+                                    "host-driven loop, CUDA events per launch on the launching stream"}
+
     # ---- end to end through the C ABI with host buffers ----
     e2e = None
     if args.e2e_steps > 0:
@@ -358,7 +393,7 @@ def main():
                 "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
                 "config": dict(workload_config(args, g, world), graph_gen_s=round(t_gen, 1)),
-                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
+                "roofline": roofline, "roofline_dense_push": dense, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches),
                 "clocks": clk.summary(), "per_step": avg}
         print(json.dumps(line), flush=True)
     if world > 1:

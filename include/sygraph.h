@@ -177,7 +177,8 @@ SG_API int run_bc(const sg_graph *g, const int32_t *sources, int32_t k, double *
                   sg_stats *stats);
 
 /* ---- measurement (bench.py roofline; not needed for correctness) ----------------------- */
-enum { SG_K_COMPACT = 0, SG_K_STATS = 1, SG_K_PUSH = 2, SG_K_PULL = 3, SG_K_BC = 4, SG_K_COUNT = 5 };
+enum { SG_K_COMPACT = 0, SG_K_STATS = 1, SG_K_PUSH = 2, SG_K_PULL = 3, SG_K_BC = 4, SG_K_SWEEP = 5, SG_K_COUNT = 6 };
+/* SG_K_SWEEP: push supersteps taken by the destination-segmented sweep (sg_opts.scsr). */
 typedef struct {
     double ms;                /* summed CUDA-event time of the class's launches (launching stream) */
     double bytes;             /* summed algorithmic HBM bytes */

@@ -68,8 +68,8 @@ class SgKprof(ctypes.Structure):
     _fields_ = [("ms", ctypes.c_double), ("bytes", ctypes.c_double), ("launches", ctypes.c_int64)]
 
 
-SG_K_COMPACT, SG_K_STATS, SG_K_PUSH, SG_K_PULL, SG_K_BC, SG_K_COUNT = 0, 1, 2, 3, 4, 5
-K_NAMES = ["compact", "stats", "advance_push", "advance_pull", "bc"]
+SG_K_COMPACT, SG_K_STATS, SG_K_PUSH, SG_K_PULL, SG_K_BC, SG_K_SWEEP, SG_K_COUNT = 0, 1, 2, 3, 4, 5, 6
+K_NAMES = ["compact", "stats", "advance_push", "advance_pull", "bc", "advance_sweep"]
 
 # every symbol include/sygraph.h declares (checked by tests/test_abi.py)
 EXPORTS = ["graph_load_csr", "graph_free", "graph_info", "frontier_init", "frontier_free", "frontier_insert",

@@ -993,11 +993,12 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         }
         nf_prev = nf;
         const int64_t reached_before = reached;
-        const int pr = prof_begin(ws, pull ? SG_K_PULL : SG_K_PUSH, s);
+        const bool sweep = !pull && scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz));
+        const int pr = prof_begin(ws, pull ? SG_K_PULL : (sweep ? SG_K_SWEEP : SG_K_PUSH), s);
         if (pull) {
             launch_pull_bfs(G, in->bits, ws->visited, in->st, s);
             pull_steps++;
-        } else if (scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz))) {
+        } else if (sweep) {
             launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, s);
             push_steps++;
         } else {

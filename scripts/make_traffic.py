@@ -2,17 +2,18 @@
 
     ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
         --csv --log-file launches.csv python scripts/profile_one_bfs.py auto
-    python scripts/make_traffic.py launches.csv > profiles/traffic.json
+    python scripts/make_traffic.py launches.csv [push_only_launches.csv] > profiles/traffic.json
 
 Per bench roofline class: mean DRAM bytes (read + write) per advance launch, where one push
-advance = k_push_words + k_push_heavy (+ k_push_seg) and one pull advance = k_pull_bfs."""
+advance = k_push_words + k_push_heavy (+ k_push_seg) and one pull advance = k_pull_bfs; from the
+optional push-only list, the dense supersteps' sweep (k_push_sweep + k_frontier_arcs)."""
 import collections
 import csv
 import json
 import sys
 
 
-def main(path):
+def load(path):
     lines = open(path).read().splitlines()
     start = [i for i, l in enumerate(lines) if l.startswith('"ID"')][0]
     rows = list(csv.reader(lines[start:]))
@@ -22,6 +23,11 @@ def main(path):
     for r in rows[1:]:
         key = (int(r[ii]), r[ki].split("(")[0].replace("void ", ""))
         launches.setdefault(key, {})[r[mi]] = float(r[vi].replace(",", ""))
+    return launches
+
+
+def main(path, push_path=None):
+    launches = load(path)
     # keep the last BFS: from the last k_seed on
     items = list(launches.items())
     last_seed = max(i for i, ((_, k), _) in enumerate(items) if "k_seed" in k)
@@ -47,8 +53,26 @@ def main(path):
         "advance_pull": {"dram_bytes_per_launch": sum(b for b, _ in pull) / max(len(pull), 1), "launches": len(pull),
                          "ncu_ms_total": sum(t for _, t in pull) / 1e6},
     }
+    if push_path:
+        sw = []
+        for (_, k), m in load(push_path).items():
+            b = m.get("dram__bytes_read.sum", 0.0) + m.get("dram__bytes_write.sum", 0.0)
+            t = m.get("gpu__time_duration.sum", 0.0)
+            if "k_push_sweep" in k:
+                sw.append([b, t, m.get("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed")])
+            elif "k_frontier_arcs" in k and sw:
+                sw[-1][0] += b
+                sw[-1][1] += t
+        heavy = max(sw, key=lambda x: x[1]) if sw else None
+        out["advance_sweep"] = {
+            "source": f"ncu launch list of one push-only BFS ({push_path})",
+            "dram_bytes_per_launch": sum(b for b, _, _ in sw) / max(len(sw), 1), "launches": len(sw),
+            "ncu_ms_total": sum(t for _, t, _ in sw) / 1e6,
+            "ncu_dram_pct_of_peak": heavy[2] if heavy else None,
+            "heaviest_launch": {"dram_bytes": heavy[0], "ms": heavy[1] / 1e6,
+                                "GBps": heavy[0] / heavy[1] if heavy and heavy[1] else None} if heavy else None}
     print(json.dumps(out, indent=1))
 
 
 if __name__ == "__main__":
-    main(sys.argv[1])
+    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None)
