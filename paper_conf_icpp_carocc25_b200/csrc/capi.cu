@@ -794,6 +794,13 @@ static bool scsr_ready(sg_graph *g, const Tiers &t, cudaStream_t s) {
     return g->scsr_state == 1;
 }
 
+// pull supersteps write their output frontier / levels themselves (1, default) or mark visited
+// only with k_bfs_diff after them (SG_PULL_FUSED=0, A/B knob)
+static bool pull_fused() {
+    static const bool on = env_or("SG_PULL_FUSED", 1) != 0;
+    return on;
+}
+
 static int build_bfs_graph(sg_graph *g, Tiers t) {
     Workspace *ws = g->ws;
     const GraphView &G = g->v;
@@ -852,23 +859,30 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
         BfsArgs a{ws->visited, nullptr, 0u, nullptr, nullptr, &ws->ctrl->next, &ws->ctrl->level, 1u};
+        // output of the superstep (out->st was zeroed by the previous k_bfs_decide / the prologue)
+        const BfsOut bo{ws->vis_old, out->bits, out->summ, nullptr, 0u, &ws->ctrl->next, &ws->ctrl->level, out->st};
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
+        launch_bfs_diff(G, ws->visited, bo, cs);
         TRY(capture_end(cs, leaves));
         if (sc) {   // dense push supersteps (k_bfs_decide: m_f >= threshold) take the sweep instead
             TRY(capture_begin(cs, b_sweep, {}));
             launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, cs);
+            launch_bfs_diff(G, ws->visited, bo, cs);
             TRY(capture_end(cs, leaves));
         }
         TRY(capture_begin(cs, b_pull, {}));
-        launch_pull_bfs(G, in->bits, ws->visited, in->st, cs);
+        if (pull_fused()) {
+            launch_pull_bfs(G, in->bits, ws->visited, in->st, bo, cs);   // writes its output itself
+        } else {
+            launch_pull_bfs(G, in->bits, ws->visited, in->st, BfsOut{}, cs);
+            launch_bfs_diff(G, ws->visited, bo, cs);
+        }
         TRY(capture_end(cs, leaves));
         std::vector<cudaGraphNode_t> ends{n_push, n_pull};
         if (n_sweep) ends.push_back(n_sweep);
         TRY(capture_begin(cs, body, ends));
-        launch_clear_listed(in->bits, in->summ, in->offsets, in->st, G.nw1, G.nw2, out->st, cs);
-        launch_bfs_diff(G, ws->visited, ws->vis_old, out->bits, out->summ, nullptr, 0u, &ws->ctrl->next,
-                        &ws->ctrl->level, out->st, cs);
+        launch_clear_listed(in->bits, in->summ, in->offsets, in->st, G.nw1, G.nw2, nullptr, cs);
         launch_compact(out->summ, G.nw2, out->offsets, out->st, cs);
         launch_bfs_decide(ws->ctrl, out->st, in->st, h_loop, h_push[half ^ 1], h_pull[half ^ 1],
                           sc ? h_sweep[half ^ 1] : 0ull, 0, cs);
@@ -916,13 +930,13 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     CK(cudaGetLastError());
     if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
     {
-        // kernels the graph executed: prologue (seed, compact, stats, decide) + per WHILE body
-        // (2 x clear, diff, compact, decide) + the taken IF bodies (push = word + CTA tier
-        // [+ hub segment tier] [+ segmented advance], pull = 1)
+        // kernels the graph executed: prologue (level init, seed, compact, stats, decide) + per
+        // WHILE body (2 x clear, compact, decide) + the taken IF bodies (push = word + CTA tier
+        // [+ hub segment tier] + diff, sweep = arc count + sweep + diff, pull = 1 [+ diff])
         const long long bodies = (long long)(c.iters + 1) / 2;
-        const long long per_push = 2 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
-        const long long k = 4 + 8 * bodies + per_push * (long long)(c.push_steps - c.sweep_steps) +
-                            2 * (long long)c.sweep_steps + (long long)c.pull_steps;
+        const long long per_push = 3 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
+        const long long k = 5 + 6 * bodies + per_push * (long long)(c.push_steps - c.sweep_steps) +
+                            3 * (long long)c.sweep_steps + (pull_fused() ? 1 : 2) * (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }
     if (stats) {
@@ -994,9 +1008,11 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         nf_prev = nf;
         const int64_t reached_before = reached;
         const bool sweep = !pull && scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz));
+        CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
+        const BfsOut bo{ws->vis_old, out->bits, out->summ, level, d + 1, nullptr, nullptr, out->st};
         const int pr = prof_begin(ws, pull ? SG_K_PULL : (sweep ? SG_K_SWEEP : SG_K_PUSH), s);
         if (pull) {
-            launch_pull_bfs(G, in->bits, ws->visited, in->st, s);
+            launch_pull_bfs(G, in->bits, ws->visited, in->st, pull_fused() ? bo : BfsOut{}, s);
             pull_steps++;
         } else if (sweep) {
             launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, s);
@@ -1017,9 +1033,8 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         prof_end(ws, pr, s);
         TRY(clear_frontier(in, s));
         const int pc = prof_begin(ws, SG_K_COMPACT, s);
-        // output of the superstep: new = visited & ~vis_old -> out 2LB, level, n_f / m_f
-        CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
-        launch_bfs_diff(G, ws->visited, ws->vis_old, out->bits, out->summ, level, d + 1, nullptr, nullptr, out->st, s);
+        // output of a push superstep: new = visited & ~vis_old -> out 2LB, level, n_f / m_f
+        if (!pull || !pull_fused()) launch_bfs_diff(G, ws->visited, bo, s);
         launch_compact(out->summ, G.nw2, out->offsets, out->st, s);
         prof_end(ws, pc, s);
         TRY(read_stats(ws, s));

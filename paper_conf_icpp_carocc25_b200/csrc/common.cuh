@@ -107,6 +107,13 @@ struct SegItem {
 
 __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 
+// 8-bit log-coded degree (graph load, frontier.cu k_deg8): exact below 32, else 3 mantissa bits
+__device__ __forceinline__ uint32_t deg8_decode(uint32_t c) {
+    if (c < 32u) return c;
+    const uint32_t e = ((c - 32u) >> 3) + 5u, m = (c - 32u) & 7u;
+    return ((8u + m) << (e - 3u)) + (1u << (e - 4u));
+}
+
 __device__ __forceinline__ unsigned long long atomic_or_u64(uint64_t *p, uint64_t m) {
     return atomicOr(reinterpret_cast<unsigned long long *>(p), (unsigned long long)m);
 }

@@ -17,8 +17,8 @@ __device__ __forceinline__ void set_cond(unsigned long long h, unsigned v) {
 
 // Decide the next superstep from the freshly compacted frontier's control block `st`.
 // `prev` (nullable) is the control block of the frontier just advanced: its arcs counter is
-// folded into the per-direction totals.
-__global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
+// folded into the per-direction totals, then it is zeroed (it is the next superstep's output).
+__global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
                              unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep,
                              int first) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
@@ -53,6 +53,7 @@ __global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *pre
     set_cond(h_sweep, sweep);
     set_cond(h_pull, go && c->pull);
     set_cond(h_loop, go);
+    if (prev) *prev = DevStats{};
 }
 
 // BFS prologue on the device: level[src] = 0, in = {src}, visited |= {src} (src, level from ctrl).
@@ -103,7 +104,7 @@ __global__ void k_zero_u64(unsigned long long *p, int64_t n) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += stride) p[i] = 0ull;
 }
 
-void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
+void launch_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
                        unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep, int first,
                        cudaStream_t s) {
     note_launch();

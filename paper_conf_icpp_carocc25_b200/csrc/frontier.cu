@@ -97,11 +97,7 @@ k_compact(const uint64_t *__restrict__ summ, int64_t nw2, uint32_t *__restrict__
 // the Beamer heuristic, so it is read from the graph's 8-bit log-coded degree array (16 MB for
 // 2^24 vertices, L2 resident; <= 1/16 relative error per vertex) instead of row_ptr (134 MB).
 // One thread per layer-1 word, no offsets indirection: bits + 64 code bytes per non-zero word.
-__device__ __forceinline__ uint32_t deg8_decode(uint32_t c) {
-    if (c < 32u) return c;
-    const uint32_t e = ((c - 32u) >> 3) + 5u, m = (c - 32u) & 7u;
-    return ((8u + m) << (e - 3u)) + (1u << (e - 4u));
-}
+// deg8_decode: common.cuh
 
 __global__ void __launch_bounds__(256) k_frontier_stats(const uint64_t *__restrict__ bits, int64_t nw1,
                                                         const uint8_t *__restrict__ deg8, DevStats *st) {
@@ -351,61 +347,88 @@ void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src,
     k_seed<<<1, 1, 0, s>>>(bits, summ, visited, src, vis_old);
 }
 
-// Output of a diff-mode BFS superstep (FnBfs::diff, pull.cu): the vertices first visited by
-// the step are new = visited & ~vis_old.  A warp reads 32 word pairs (one per lane, coalesced)
-// and skips the unchanged ones by ballot; the changed words are processed two at a time, one
-// per half-warp, one thread per quad of 4 vertices: the quad's level entries and degree codes,
-// the word's new bits written by the half-warp's first thread with the summary bit and vis_old.
-// n_f / m_f of the output frontier (direction policy) come out of the same pass.
-__global__ void __launch_bounds__(256) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited,
-                                                  uint64_t *__restrict__ vis_old, uint64_t *__restrict__ out_bits,
-                                                  uint64_t *__restrict__ out_summ, uint32_t *level, uint32_t next,
-                                                  const uint32_t *next_ptr, uint32_t *const *level_pp, DevStats *st) {
+// Output of a diff-mode BFS superstep (FnBfs::diff, the sweep): the vertices first visited by
+// the step are new = visited & ~vis_old.  A warp owns 32 layer-1 words (half a layer-2 word): it
+// reads the 32 word pairs coalesced (one per lane), writes the changed words' vis_old and output
+// bits and ORs its half of the layer-2 word (one atomic per warp).  The changed words' vertices
+// are then handled 8 words per round, one half-warp per word: a thread reads the degree codes of
+// a quad of 4 vertices (m_f; the 4 loads of a round issued together, so a round costs one memory
+// latency) and stores the levels of vertices lane16 + 16 i (whole 64-B runs of level[] per store
+// instruction).  n_f / m_f of the output frontier (direction policy) come out of the same pass.
+#ifndef SG_DIFF_WPR
+#define SG_DIFF_WPR 8
+#endif
+#ifndef SG_DIFF_MINB
+#define SG_DIFF_MINB 1
+#endif
+constexpr int DIFF_WORDS_PER_ROUND = SG_DIFF_WPR;
+__global__ void __launch_bounds__(256, SG_DIFF_MINB) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited, BfsOut o) {
     const int lane = lane_id();
+    const int half = lane >> 4;
+    const int sh = (lane & 15) * 4;
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int sh = (lane & 15) * 4;
+    const int64_t nchunks = (g.nw1 + 31) >> 5;
     unsigned long long nf = 0, mf = 0;
     uint32_t *lvl = nullptr;
     uint32_t nx = 0;
-    for (int64_t base = gw * 32; base < g.nw1; base += nwarps * 32) {
-        const int64_t wl = base + lane;
-        uint64_t nv = 0, ov = 0;
-        if (wl < g.nw1) {
-            nv = visited[wl];
-            ov = vis_old[wl];
+    for (int64_t ck = gw; ck < nchunks; ck += nwarps) {
+        const int64_t w0 = ck * 32;
+        const int64_t wa = w0 + lane;
+        uint64_t na = 0, oa = 0;
+        if (wa < g.nw1) {
+            na = visited[wa];
+            oa = o.vis_old[wa];
         }
-        uint32_t changed = __ballot_sync(0xffffffffu, nv != ov);
-        if (changed && !lvl) {
-            lvl = level_pp ? *level_pp : level;
-            nx = next_ptr ? *next_ptr : next;
+        const uint64_t da = na & ~oa;
+        uint32_t ch = __ballot_sync(0xffffffffu, da != 0);
+        if (!ch) continue;
+        if (!lvl) {
+            lvl = o.level_pp ? *o.level_pp : o.level;
+            nx = o.next_ptr ? *o.next_ptr : o.next;
         }
-        while (changed) {
-            const int i0 = __ffs(changed) - 1;
-            changed &= changed - 1;
-            const int i1 = changed ? __ffs(changed) - 1 : -1;
-            if (i1 >= 0) changed &= changed - 1;
-            const int mi = lane < 16 ? i0 : i1;
-            const uint64_t wn = __shfl_sync(0xffffffffu, nv, mi < 0 ? 0 : mi);
-            const uint64_t wo = __shfl_sync(0xffffffffu, ov, mi < 0 ? 0 : mi);
-            if (mi < 0) continue;
-            const int64_t w = base + mi;
-            const uint64_t nb = wn & ~wo;
-            const uint32_t mine = (uint32_t)(nb >> sh) & 0xfu;
-            if (mine) {
-                const uint32_t codes = __ldg(reinterpret_cast<const uint32_t *>(g.deg8 + w * 64 + sh));
-                nf += __popc(mine);
-                for (uint32_t f = mine; f; f &= f - 1) {
-                    const int k = __ffs(f) - 1;
-                    lvl[w * 64 + sh + k] = nx;
-                    mf += deg8_decode((codes >> (8 * k)) & 0xffu);
-                }
+        if (da) {
+            o.vis_old[wa] = na;
+            o.out_bits[wa] = da;
+        }
+        if (lane == 0) atomic_or_u64(o.out_summ + (w0 >> 6), (uint64_t)ch << (w0 & 63));
+        while (ch) {
+            int wi[DIFF_WORDS_PER_ROUND / 2];   // this half-warp's words of the round (-1: none)
+#pragma unroll
+            for (int j = 0; j < DIFF_WORDS_PER_ROUND / 2; j++) {
+                const int i0 = ch ? __ffs(ch) - 1 : -1;
+                ch &= ch - 1;
+                const int i1 = ch ? __ffs(ch) - 1 : -1;
+                ch &= ch - 1;
+                wi[j] = half ? i1 : i0;
             }
-            if ((lane & 15) == 0) {
-                vis_old[w] = wn;
-                if (nb) {
-                    out_bits[w] = nb;
-                    atomic_or_u64(out_summ + (w >> 6), 1ull << (w & 63));
+            uint32_t mine[DIFF_WORDS_PER_ROUND / 2], codes[DIFF_WORDS_PER_ROUND / 2], spread[DIFF_WORDS_PER_ROUND / 2];
+#pragma unroll
+            for (int j = 0; j < DIFF_WORDS_PER_ROUND / 2; j++) {
+                const uint64_t x = __shfl_sync(0xffffffffu, da, wi[j] < 0 ? 0 : wi[j]);
+                const uint64_t d = wi[j] < 0 ? 0ull : x;
+                mine[j] = (uint32_t)(d >> sh) & 0xfu;
+                const uint64_t t = d >> (lane & 15);   // bits lane16, 16 + lane16, 32 + .., 48 + ..
+                spread[j] = (uint32_t)(t & 1u) | (uint32_t)((t >> 15) & 2u) | (uint32_t)((t >> 30) & 4u) |
+                            (uint32_t)((t >> 45) & 8u);
+            }
+#pragma unroll
+            for (int j = 0; j < DIFF_WORDS_PER_ROUND / 2; j++)
+                codes[j] = mine[j] ? __ldg(reinterpret_cast<const uint32_t *>(g.deg8 + (w0 + wi[j]) * 64 + sh)) : 0u;
+#pragma unroll
+            for (int j = 0; j < DIFF_WORDS_PER_ROUND / 2; j++) {
+                nf += __popc(mine[j]);
+#pragma unroll
+                for (int k = 0; k < 4; k++)
+                    mf += ((mine[j] >> k) & 1u) ? deg8_decode((codes[j] >> (8 * k)) & 0xffu) : 0u;
+                // level stores strided over the half-warp (vertex 16 i + lane16): each store
+                // instruction writes 64 contiguous bytes of level[] instead of 16 scattered quads
+                const uint32_t sp = spread[j];
+                if (sp) {
+                    uint32_t *lw = lvl + (w0 + wi[j]) * 64 + (lane & 15);
+#pragma unroll
+                    for (int i = 0; i < 4; i++)
+                        if ((sp >> i) & 1u) lw[16 * i] = nx;
                 }
             }
         }
@@ -425,18 +448,17 @@ __global__ void __launch_bounds__(256) k_bfs_diff(GraphView g, const uint64_t *_
             b += s_nf[i];
         }
         if (a | b) {
-            atomicAdd(&st->mf, a);
-            atomicAdd(&st->nf, b);
+            atomicAdd(&o.st->mf, a);
+            atomicAdd(&o.st->nf, b);
         }
     }
 }
-void launch_bfs_diff(const GraphView &g, const uint64_t *visited, uint64_t *vis_old, uint64_t *out_bits,
-                     uint64_t *out_summ, uint32_t *level, uint32_t next, const uint32_t *next_ptr,
-                     uint32_t *const *level_pp, DevStats *st, cudaStream_t s) {
+void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s) {
+    int64_t blocks = ((g.nw1 + 31) / 32 * 32 + 255) / 256;   // one warp per 32 layer-1 words
+    if (blocks > 148 * 8 * 4) blocks = 148 * 8 * 4;
+    if (blocks < 1) blocks = 1;
     note_launch();
-    k_bfs_diff<<<grid_for((g.nw1 + 31) / 32 * 32, 256, 148 * 16), 256, 0, s>>>(g, visited, vis_old, out_bits,
-                                                                             out_summ, level, next, next_ptr,
-                                                                             level_pp, st);
+    k_bfs_diff<<<(int)blocks, 256, 0, s>>>(g, visited, o);
 }
 void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(p, n); }
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s) {

@@ -76,14 +76,24 @@ void launch_push_bc(const PushLaunch &L, const BcArgs &a, cudaStream_t s);
 int push_max_grid_words();
 int push_max_grid_heavy();
 
-// pull.cu — bottom-up BFS step (direction-optimising, Beamer): marks visited only,
-// k_bfs_diff builds the output frontier / level / statistics
-void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, cudaStream_t s);
-// frontier.cu — output of a diff-mode BFS superstep: new = visited & ~vis_old -> out 2LB,
-// level[new] = next, vis_old |= new, out->st n_f / m_f (st zeroed before)
-void launch_bfs_diff(const GraphView &g, const uint64_t *visited, uint64_t *vis_old, uint64_t *out_bits,
-                     uint64_t *out_summ, uint32_t *level, uint32_t next, const uint32_t *next_ptr,
-                     uint32_t *const *level_pp, DevStats *st, cudaStream_t s);
+// Output of a BFS superstep: new = visited & ~vis_old -> out 2LB (+ summary), level[new] = next,
+// vis_old |= new, st->nf / st->mf of the output frontier (st zeroed before).  Graph mode reads
+// `next` / `level` through next_ptr / level_pp (BfsCtrl).
+struct BfsOut {
+    uint64_t *vis_old;
+    uint64_t *out_bits, *out_summ;
+    uint32_t *level;
+    uint32_t next;
+    const uint32_t *next_ptr;
+    uint32_t *const *level_pp;
+    DevStats *st;
+};
+// pull.cu — bottom-up BFS step (direction-optimising, Beamer): writes its output `o`
+// itself (no k_bfs_diff after it); o.out_bits == NULL: marks visited only (k_bfs_diff after it)
+void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,
+                     cudaStream_t s);
+// frontier.cu — output of a diff-mode BFS superstep (push word path / sweep): see BfsOut
+void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s);
 
 // filter.cu — filter::inplace / external, compute::execute (Table 2)
 void launch_filter(const GraphView &g, const uint64_t *in_bits, uint64_t *out_bits, uint64_t *out_summ, int pred,
@@ -118,7 +128,7 @@ void launch_push_sweep(const ScsrView &v, const int64_t *rp, const uint64_t *in_
                        unsigned long long min_mf, cudaStream_t s);
 
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
-void launch_bfs_decide(BfsCtrl *c, const DevStats *st, const DevStats *prev, unsigned long long h_loop,
+void launch_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
                        unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep, int first,
                        cudaStream_t s);
 void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,

@@ -13,11 +13,12 @@
 // no loop in the common path: the thread reads the visited word and, if one of its vertices is
 // unvisited, their 4 candidates with one 16-B load, then tests them (the only random reads, on
 // a 2 MB bitmap that stays in L2).  The 16 threads of a word OR their found bits together
-// (half-warp reduction), and one of them writes the visited word; k_bfs_diff then derives the
-// output frontier, level[] and the statistics, as after a diff-mode push.  The step is a
-// streaming pass over the visited bitmap and fnbr with enough independent threads in flight to
-// cover the latency of the dependent bit test.  Output identical to a push step from the same
-// state.
+// (half-warp reduction).  The step writes its own output (no k_bfs_diff pass after a pull): the
+// thread adds n_f / m_f of the vertices it found (degree codes, one 4-B load) and stores the
+// levels of the word's new vertices lane16 + 16 i (64-B runs per store); the half-warp's first thread writes the word's new bits to visited, vis_old and the
+// output frontier (+ its summary bit).  The step is a streaming pass over the visited bitmap and
+// fnbr with enough independent threads in flight to cover the latency of the dependent bit
+// test.  Output identical to a push step from the same state.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -27,28 +28,39 @@ constexpr int PULL_THREADS = 256;
 #ifndef SG_PULL_ARCS
 #define SG_PULL_ARCS 2
 #endif
-constexpr int PULL_ARCS = SG_PULL_ARCS;   // arcs in flight per step of a list scan
+constexpr int PULL_ARCS = SG_PULL_ARCS;
+#ifndef SG_PULL_WAVES
+#define SG_PULL_WAVES 16   // CTAs per SM in the grid (x 148)
+#endif   // arcs in flight per step of a list scan
 
-__global__ void __launch_bounds__(PULL_THREADS)
-k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st) {
-    __shared__ unsigned long long s_arcs[PULL_THREADS / 32];
+template <bool FUSED>
+__global__ void __launch_bounds__(PULL_THREADS, 8)
+k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
+           BfsOut o) {
+    __shared__ unsigned long long s_arcs[PULL_THREADS / 32], s_nf[PULL_THREADS / 32], s_mf[PULL_THREADS / 32];
+    uint32_t *const lvl = o.level_pp ? *o.level_pp : o.level;
+    const uint32_t nx = o.next_ptr ? *o.next_ptr : o.next;
+    unsigned long long nf = 0, mf = 0;
     const int lane = lane_id();
     const uint32_t *in32 = reinterpret_cast<const uint32_t *>(in_bits);
     const int64_t nq = g.nw1 * 16;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;   // multiple of 16: a word's quads stay in one half-warp
     const uint32_t half = (lane < 16) ? 0x0000ffffu : 0xffff0000u;
     unsigned long long arcs = 0;
-    for (int64_t qd = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; qd < nq; qd += stride) {
+    // whole warps iterate (qd - lane = the warp's first quad), lanes past the end idle
+    for (int64_t qd = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; qd - lane < nq; qd += stride) {
+        const bool ok = qd < nq;
         const int64_t w = qd >> 4;
         const int sh = (int)(qd & 15) * 4;
-        const uint64_t vis = visited[w];
+        const uint64_t vis = ok ? visited[w] : ~0ull;
         const int64_t v0 = w * 64 + sh;
         const int64_t rem = g.n - v0;
-        const uint32_t valid = rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
+        const uint32_t valid = !ok ? 0u : rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
         const uint32_t unv = (uint32_t)(~vis >> sh) & valid;
-        uint32_t found = 0;
+        uint32_t found = 0, codes = 0;
         if (unv) {
             const int4 c4 = __ldg(reinterpret_cast<const int4 *>(g.fnbr + v0));
+            if (FUSED) codes = __ldg(reinterpret_cast<const uint32_t *>(g.deg8 + v0));   // in flight with c4
             const int32_t c[4] = {c4.x, c4.y, c4.z, c4.w};
             uint32_t x[4];
 #pragma unroll
@@ -89,25 +101,71 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
         const uint64_t mine = (uint64_t)found << sh;
         const uint64_t nb = (uint64_t)__reduce_or_sync(half, (uint32_t)mine) |
                             ((uint64_t)__reduce_or_sync(half, (uint32_t)(mine >> 32)) << 32);
-        if (nb && (lane & 15) == 0) visited[w] = vis | nb;
+        if (FUSED && found) {   // the output: n_f / m_f of the vertices found here
+            nf += __popc(found);
+#pragma unroll
+            for (int k = 0; k < 4; k++) mf += ((found >> k) & 1u) ? deg8_decode((codes >> (8 * k)) & 0xffu) : 0u;
+        }
+        if (FUSED && nb) {   // level[] of the word's new vertices, strided over the half-warp (vertex
+                             // 16 i + lane16): each store instruction writes 64 contiguous bytes
+            const uint64_t t = nb >> (lane & 15);
+            uint32_t *lw = lvl + w * 64 + (lane & 15);
+#pragma unroll
+            for (int i = 0; i < 4; i++)
+                if ((t >> (16 * i)) & 1u) lw[16 * i] = nx;
+        }
+        if (FUSED) {
+            // the warp's two words share a layer-2 word (stride and blocks are multiples of 32
+            // quads): one atomic per warp
+            const uint32_t act = __ballot_sync(0xffffffffu, nb != 0ull && (lane & 15) == 0);
+            if (nb && (lane & 15) == 0) {
+                visited[w] = vis | nb;
+                o.vis_old[w] = vis | nb;
+                o.out_bits[w] = nb;
+            }
+            if (lane == 0 && act) {
+                const int64_t wl = w & ~1ll;   // the warp's first word
+                atomic_or_u64(o.out_summ + (wl >> 6),
+                              ((act & 1u) ? 1ull << (wl & 63) : 0ull) | ((act >> 16) ? 2ull << (wl & 63) : 0ull));
+            }
+        } else if (nb && (lane & 15) == 0) {
+            visited[w] = vis | nb;
+        }
     }
     arcs = warp_sum(arcs);
-    if (lane == 0) s_arcs[threadIdx.x >> 5] = arcs;
+    nf = warp_sum(nf);
+    mf = warp_sum(mf);
+    if (lane == 0) {
+        s_arcs[threadIdx.x >> 5] = arcs;
+        s_nf[threadIdx.x >> 5] = nf;
+        s_mf[threadIdx.x >> 5] = mf;
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned long long t = 0;
-        for (int i = 0; i < PULL_THREADS / 32; i++) t += s_arcs[i];
+        unsigned long long t = 0, a = 0, b = 0;
+        for (int i = 0; i < PULL_THREADS / 32; i++) {
+            t += s_arcs[i];
+            a += s_nf[i];
+            b += s_mf[i];
+        }
         if (t) atomicAdd(&st->arcs, t);
+        if (a) {
+            atomicAdd(&o.st->nf, a);
+            atomicAdd(&o.st->mf, b);
+        }
     }
 }
 
-void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, cudaStream_t s) {
-    // one thread per quad, no grid-stride loop up to 64 resident CTA waves
+void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,
+                     cudaStream_t s) {
+    // one thread per quad in a grid-stride loop over one resident wave (8 CTAs per SM): few
+    // CTAs, so few same-address statistics atomics at their ends
     int64_t blocks = (g.nw1 * 16 + PULL_THREADS - 1) / PULL_THREADS;
-    if (blocks > 148 * 8 * 64) blocks = 148 * 8 * 64;
+    if (blocks > 148 * SG_PULL_WAVES) blocks = 148 * SG_PULL_WAVES;
     if (blocks < 1) blocks = 1;
     note_launch();
-    k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st);
+    if (o.out_bits) k_pull_bfs<true><<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);
+    else k_pull_bfs<false><<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);
 }
 
 }  // namespace sg
