@@ -1,0 +1,126 @@
+// bfsstep.cuh — end of a BFS superstep on the device, shared by k_bfs_diff (after push / sweep)
+// and the pull step: block-aggregated emission of the output frontier's layer-2 words and word
+// list, statistics, and the direction decision taken by the last CTA to finish (so a superstep
+// is its advance kernels + one output kernel, no compaction / clear / decide launches).
+#pragma once
+#include "common.cuh"
+#include "kernels.h"
+
+namespace sg {
+
+__device__ __forceinline__ void bfs_set_cond(unsigned long long h, unsigned v) {
+    if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, v);
+}
+
+// Beamer direction policy (R2) + loop control, from the freshly built output frontier's
+// control block `st`; `prev` (nullable) = the control block of the frontier just advanced: its
+// arcs counter is folded into the per-direction totals, then it is zeroed (it is the next
+// superstep's output).  One thread.
+__device__ __forceinline__ void bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
+                                           unsigned long long h_push, unsigned long long h_pull,
+                                           unsigned long long h_sweep, int first) {
+    // control blocks were filled by atomics of other CTAs / kernels: volatile (L2) reads
+    const volatile DevStats *vst = st;
+    if (prev) {
+        const unsigned long long pa = reinterpret_cast<const volatile DevStats *>(prev)->arcs;
+        if (c->pull) c->arcs_pulled += pa;
+        else c->arcs_pushed += pa;
+    }
+    const unsigned long long count = vst->count;
+    bool go = count > 0;
+    if (go && c->iters >= (unsigned long long)c->max_iters) {
+        c->overflow = 1;
+        go = false;
+    }
+    if (go) {
+        const long long nf = (long long)vst->nf, mf = (long long)vst->mf;
+        if (!first) c->reached += (unsigned long long)nf;
+        c->mu -= mf;
+        if (c->auto_dir) {
+            if (!c->pull && nf > c->nf_prev && (double)mf > (double)c->mu / c->alpha) c->pull = 1;
+            else if (c->pull && nf < c->nf_prev && (double)nf < (double)c->n / c->beta) c->pull = 0;
+        }
+        c->nf_prev = nf;
+        c->next = first ? 1u : c->next + 1u;
+        if (c->pull) c->pull_steps++;
+        else c->push_steps++;
+        c->iters++;
+    }
+    const bool push = go && !c->pull;
+    const bool sweep = push && (c->sweep_mode == 2 || (c->sweep_mode == 1 && vst->mf >= c->sweep_thr));
+    if (sweep) c->sweep_steps++;
+    bfs_set_cond(h_push, push && !sweep);
+    bfs_set_cond(h_sweep, sweep);
+    bfs_set_cond(h_pull, go && c->pull);
+    bfs_set_cond(h_loop, go);
+    if (prev) *prev = DevStats{};
+}
+
+// Emit a block's slice of the output frontier: `S` = the block's layer-2 words (in shared
+// memory, nS of them, the first = layer-2 word sw0), written as is; their set bits are appended
+// to the word list with one atomic per block (ascending within the block).  Call with the whole
+// block; ends with __syncthreads.
+__device__ __forceinline__ void bfs_emit_words(const BfsOut &o, int64_t nw2, int64_t sw0, const uint64_t *S, int nS,
+                                               uint32_t *s_base) {
+    if ((int)threadIdx.x < nS && sw0 + threadIdx.x < nw2) o.out_summ[sw0 + threadIdx.x] = S[threadIdx.x];
+    if (threadIdx.x == 0) {
+        uint32_t tot = 0;
+        for (int i = 0; i < nS; i++) tot += (uint32_t)__popcll(S[i]);
+        *s_base = tot ? (uint32_t)atomicAdd(&o.st->count, (unsigned long long)tot) : 0u;
+    }
+    __syncthreads();
+    for (int t = threadIdx.x; t < nS * 64; t += blockDim.x) {
+        const int i = t >> 6, b = t & 63;
+        const uint64_t x = S[i];
+        if ((x >> b) & 1ull) {
+            uint32_t pos = *s_base + (uint32_t)__popcll(x & ((1ull << b) - 1ull));
+            for (int j = 0; j < i; j++) pos += (uint32_t)__popcll(S[j]);
+            o.out_offsets[pos] = (uint32_t)((sw0 + i) * 64 + b);
+        }
+    }
+    __syncthreads();
+}
+
+// End of the output kernel: block sums of n_f / m_f (and `arcs` into the input's control block),
+// then the last CTA to finish takes the direction decision (graph mode).  Whole block.
+__device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long nf, unsigned long long mf,
+                                           unsigned long long arcs, DevStats *in_st) {
+    __shared__ unsigned long long s_r[3][32];
+    __shared__ bool s_last;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    nf = warp_sum(nf);
+    mf = warp_sum(mf);
+    arcs = warp_sum(arcs);
+    if (lane == 0) {
+        s_r[0][wid] = nf;
+        s_r[1][wid] = mf;
+        s_r[2][wid] = arcs;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long a = 0, b = 0, c = 0;
+        for (int i = 0; i < (int)(blockDim.x >> 5); i++) {
+            a += s_r[0][i];
+            b += s_r[1][i];
+            c += s_r[2][i];
+        }
+        if (a) {
+            atomicAdd(&o.st->nf, a);
+            atomicAdd(&o.st->mf, b);
+        }
+        if (c && in_st) atomicAdd(&in_st->arcs, c);
+        s_last = false;
+        if (o.ctrl) {
+            __threadfence();
+            s_last = atomicAdd(o.done, 1u) == gridDim.x - 1;
+        }
+    }
+    __syncthreads();
+    if (s_last && threadIdx.x == 0) {
+        __threadfence();
+        *o.done = 0u;
+        bfs_decide(o.ctrl, o.st, o.prev, o.h_loop, o.h_push, o.h_pull, o.h_sweep, 0);
+    }
+}
+
+}  // namespace sg

@@ -98,6 +98,7 @@ struct Workspace {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     // CUDA-graph driven BFS (ctrl.cu): instantiated once per (level buffer, tiers)
     BfsCtrl *ctrl = nullptr, *h_ctrl = nullptr;
+    unsigned int *bfs_done = nullptr;   // CTA completion counter of the BFS output kernels (self-resetting)
     cudaGraph_t bfs_graph = nullptr;
     cudaGraphExec_t bfs_exec = nullptr;
     uint32_t *bfs_level = nullptr;
@@ -238,6 +239,7 @@ static void free_ws(Workspace *ws) {
     }
     if (ws->cap_stream) cudaStreamDestroy(ws->cap_stream);
     cudaFree(ws->ctrl);
+    cudaFree(ws->bfs_done);
     cudaFreeHost(ws->h_ctrl);
     if (ws->ev0) cudaEventDestroy(ws->ev0);
     if (ws->ev1) cudaEventDestroy(ws->ev1);
@@ -794,13 +796,6 @@ static bool scsr_ready(sg_graph *g, const Tiers &t, cudaStream_t s) {
     return g->scsr_state == 1;
 }
 
-// pull supersteps write their output frontier / levels themselves (1, default) or mark visited
-// only with k_bfs_diff after them (SG_PULL_FUSED=0, A/B knob)
-static bool pull_fused() {
-    static const bool on = env_or("SG_PULL_FUSED", 1) != 0;
-    return on;
-}
-
 static int build_bfs_graph(sg_graph *g, Tiers t) {
     Workspace *ws = g->ws;
     const GraphView &G = g->v;
@@ -809,6 +804,10 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     ws->bfs_exec = nullptr;
     ws->bfs_graph = nullptr;
     if (!ws->cap_stream) CK(cudaStreamCreateWithFlags(&ws->cap_stream, cudaStreamNonBlocking));
+    if (!ws->bfs_done) {
+        CK(cudaMalloc(&ws->bfs_done, sizeof(unsigned int)));
+        CK(cudaMemset(ws->bfs_done, 0, sizeof(unsigned int)));
+    }
     if (!ws->ctrl) {
         CK(cudaMalloc(&ws->ctrl, sizeof(BfsCtrl)));
         CK(cudaMallocHost(&ws->h_ctrl, sizeof(BfsCtrl)));
@@ -859,34 +858,27 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
         BfsArgs a{ws->visited, nullptr, 0u, nullptr, nullptr, &ws->ctrl->next, &ws->ctrl->level, 1u};
-        // output of the superstep (out->st was zeroed by the previous k_bfs_decide / the prologue)
-        const BfsOut bo{ws->vis_old, out->bits, out->summ, nullptr, 0u, &ws->ctrl->next, &ws->ctrl->level, out->st};
+        // output of the superstep (out->st was zeroed by the previous decision / the prologue);
+        // the output kernel's last CTA decides the next superstep (handles of the other half)
+        const BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, nullptr, 0u, &ws->ctrl->next,
+                        &ws->ctrl->level, out->st, ws->ctrl, in->st, ws->bfs_done, (unsigned long long)h_loop,
+                        (unsigned long long)h_push[half ^ 1], (unsigned long long)h_pull[half ^ 1],
+                        sc ? (unsigned long long)h_sweep[half ^ 1] : 0ull};
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
         launch_bfs_diff(G, ws->visited, bo, cs);
         TRY(capture_end(cs, leaves));
-        if (sc) {   // dense push supersteps (k_bfs_decide: m_f >= threshold) take the sweep instead
+        if (sc) {   // dense push supersteps (m_f >= threshold) take the sweep instead
             TRY(capture_begin(cs, b_sweep, {}));
             launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, cs);
             launch_bfs_diff(G, ws->visited, bo, cs);
             TRY(capture_end(cs, leaves));
         }
         TRY(capture_begin(cs, b_pull, {}));
-        if (pull_fused()) {
-            launch_pull_bfs(G, in->bits, ws->visited, in->st, bo, cs);   // writes its output itself
-        } else {
-            launch_pull_bfs(G, in->bits, ws->visited, in->st, BfsOut{}, cs);
-            launch_bfs_diff(G, ws->visited, bo, cs);
-        }
+        launch_pull_bfs(G, in->bits, ws->visited, in->st, bo, cs);   // writes its output itself
         TRY(capture_end(cs, leaves));
-        std::vector<cudaGraphNode_t> ends{n_push, n_pull};
-        if (n_sweep) ends.push_back(n_sweep);
-        TRY(capture_begin(cs, body, ends));
-        launch_clear_listed(in->bits, in->summ, in->offsets, in->st, G.nw1, G.nw2, nullptr, cs);
-        launch_compact(out->summ, G.nw2, out->offsets, out->st, cs);
-        launch_bfs_decide(ws->ctrl, out->st, in->st, h_loop, h_push[half ^ 1], h_pull[half ^ 1],
-                          sc ? h_sweep[half ^ 1] : 0ull, 0, cs);
-        TRY(capture_end(cs, deps));
+        deps = {n_push, n_pull};
+        if (n_sweep) deps.push_back(n_sweep);
     }
     CK(cudaGraphInstantiate(&ws->bfs_exec, root, 0));
     ws->bfs_heavy = t.heavy;
@@ -930,13 +922,12 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     CK(cudaGetLastError());
     if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
     {
-        // kernels the graph executed: prologue (level init, seed, compact, stats, decide) + per
-        // WHILE body (2 x clear, compact, decide) + the taken IF bodies (push = word + CTA tier
-        // [+ hub segment tier] + diff, sweep = arc count + sweep + diff, pull = 1 [+ diff])
-        const long long bodies = (long long)(c.iters + 1) / 2;
+        // kernels the graph executed: prologue (level init, seed, compact, stats, decide) + the
+        // taken IF bodies (push = word + CTA tier [+ hub segment tier] + output, sweep = arc
+        // count + sweep + output, pull = 1)
         const long long per_push = 3 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
-        const long long k = 5 + 6 * bodies + per_push * (long long)(c.push_steps - c.sweep_steps) +
-                            3 * (long long)c.sweep_steps + (pull_fused() ? 1 : 2) * (long long)c.pull_steps;
+        const long long k = 5 + per_push * (long long)(c.push_steps - c.sweep_steps) + 3 * (long long)c.sweep_steps +
+                            (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }
     if (stats) {
@@ -1009,10 +1000,10 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         const int64_t reached_before = reached;
         const bool sweep = !pull && scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz));
         CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
-        const BfsOut bo{ws->vis_old, out->bits, out->summ, level, d + 1, nullptr, nullptr, out->st};
+        const BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, level, d + 1, nullptr, nullptr, out->st};
         const int pr = prof_begin(ws, pull ? SG_K_PULL : (sweep ? SG_K_SWEEP : SG_K_PUSH), s);
         if (pull) {
-            launch_pull_bfs(G, in->bits, ws->visited, in->st, pull_fused() ? bo : BfsOut{}, s);
+            launch_pull_bfs(G, in->bits, ws->visited, in->st, bo, s);   // writes its output itself
             pull_steps++;
         } else if (sweep) {
             launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, s);
@@ -1031,28 +1022,31 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
             push_steps++;
         }
         prof_end(ws, pr, s);
-        TRY(clear_frontier(in, s));
-        const int pc = prof_begin(ws, SG_K_COMPACT, s);
-        // output of a push superstep: new = visited & ~vis_old -> out 2LB, level, n_f / m_f
-        if (!pull || !pull_fused()) launch_bfs_diff(G, ws->visited, bo, s);
-        launch_compact(out->summ, G.nw2, out->offsets, out->st, s);
-        prof_end(ws, pc, s);
+        // output of a push superstep (the pull writes its own): new = visited & ~vis_old -> the
+        // whole out 2LB (no clearing needed) + word list, level, n_f / m_f
+        const int pc = pull ? -1 : prof_begin(ws, SG_K_COMPACT, s);
+        if (!pull) launch_bfs_diff(G, ws->visited, bo, s);
+        if (!pull) prof_end(ws, pc, s);
         TRY(read_stats(ws, s));
         {
             // algorithmic bytes of this step.  push: col_idx 4 B/arc, row_ptr 16 B
-            // per expanded vertex, 8 B per input word, 8 B per visited word updated; pull: 8 B per
-            // visited word read, 4 B per candidate / arc tested, 8 B per visited word updated;
-            // output pass (k_bfs_diff + compaction): visited and vis_old 16 B per word, level
-            // 4 B + degree code 1 B per new vertex, 16 B per output word + 4 B offset, summary
+            // per expanded vertex, 8 B per input word, 8 B per visited word updated.  Output pass
+            // (k_bfs_diff): visited + vis_old 16 B per word read, output word 8 B per word
+            // written, level 4 B + degree code 1 B per new vertex, vis_old 8 B + list entry 4 B
+            // per output word, layer 2 8 B per word.  pull (with its output): visited 8 B per
+            // word read, fnbr / col_idx 4 B per candidate / arc tested, output word 8 B per word,
+            // level + degree code 5 B per new vertex, visited + vis_old 16 B + list entry 4 B
+            // per output word, layer 2 8 B per word
             const DevStats &ho = ws->h_st[in_idx ^ 1];
             const double n_new = (double)ho.nf, c_out = (double)ho.count;
             double bytes;
             if (pull)
-                bytes = 8.0 * (double)G.nw1 + 4.0 * (double)ws->h_st[in_idx].arcs + 8.0 * c_out;
+                bytes = 16.0 * (double)G.nw1 + 4.0 * (double)ws->h_st[in_idx].arcs + 5.0 * n_new + 20.0 * c_out +
+                        8.0 * (double)G.nw2;
             else
                 bytes = 4.0 * (double)ws->h_st[in_idx].arcs + 16.0 * (double)nf + 8.0 * (double)count + 8.0 * c_out;
             prof_bytes(ws, pr, bytes);
-            prof_bytes(ws, pc, 16.0 * (double)G.nw1 + 5.0 * n_new + 20.0 * c_out + 8.0 * (double)G.nw2);
+            if (!pull) prof_bytes(ws, pc, 24.0 * (double)G.nw1 + 5.0 * n_new + 12.0 * c_out + 8.0 * (double)G.nw2);
         }
         if (pull) arcs_pulled += (int64_t)ws->h_st[in_idx].arcs;
         else arcs_pushed += (int64_t)ws->h_st[o.one_layer ? 2 : in_idx].arcs;

@@ -2,58 +2,24 @@
 //
 // Listing 1's host loop (P:172 `while (!in_frontier.empty())`, swap + clear at P:182-184) costs
 // one device->host round trip per superstep.  Here the whole BFS is one CUDA graph: a WHILE node
-// whose body runs two supersteps (A->B, B->A, so kernel arguments stay static), each superstep an
-// IF(push) / IF(pull) pair followed by clear + compaction + statistics + k_bfs_decide, which
-// applies the direction policy on the device and sets the conditional handles
-// (cudaGraphSetConditional).  Results are identical to the host loop (tested).
+// whose body runs two supersteps (A->B, B->A, so kernel arguments stay static), each superstep
+// IF(push) / IF(sweep) / IF(pull) nodes whose last kernel (k_bfs_diff, or the pull step itself)
+// writes the whole output frontier with its word list and statistics, and whose last CTA applies
+// the direction policy and sets the conditional handles (cudaGraphSetConditional, bfsstep.cuh).
+// Results are identical to the host loop (tested).
 #include "common.cuh"
 #include "kernels.h"
+#include "bfsstep.cuh"
 
 namespace sg {
 
-__device__ __forceinline__ void set_cond(unsigned long long h, unsigned v) {
-    if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, v);
-}
-
-// Decide the next superstep from the freshly compacted frontier's control block `st`.
-// `prev` (nullable) is the control block of the frontier just advanced: its arcs counter is
-// folded into the per-direction totals, then it is zeroed (it is the next superstep's output).
+// Decide the next superstep from the freshly compacted frontier's control block `st` (the
+// prologue; later supersteps decide in the last CTA of their output kernel, bfsstep.cuh).
 __global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
                              unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep,
                              int first) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    if (prev) {
-        if (c->pull) c->arcs_pulled += prev->arcs;
-        else c->arcs_pushed += prev->arcs;
-    }
-    const unsigned long long count = st->count;
-    bool go = count > 0;
-    if (go && c->iters >= (unsigned long long)c->max_iters) {
-        c->overflow = 1;
-        go = false;
-    }
-    if (go) {
-        const long long nf = (long long)st->nf, mf = (long long)st->mf;
-        if (!first) c->reached += (unsigned long long)nf;
-        c->mu -= mf;
-        if (c->auto_dir) {   // Beamer (R2)
-            if (!c->pull && nf > c->nf_prev && (double)mf > (double)c->mu / c->alpha) c->pull = 1;
-            else if (c->pull && nf < c->nf_prev && (double)nf < (double)c->n / c->beta) c->pull = 0;
-        }
-        c->nf_prev = nf;
-        c->next = first ? 1u : c->next + 1u;
-        if (c->pull) c->pull_steps++;
-        else c->push_steps++;
-        c->iters++;
-    }
-    const bool push = go && !c->pull;
-    const bool sweep = push && (c->sweep_mode == 2 || (c->sweep_mode == 1 && st->mf >= c->sweep_thr));
-    if (sweep) c->sweep_steps++;
-    set_cond(h_push, push && !sweep);
-    set_cond(h_sweep, sweep);
-    set_cond(h_pull, go && c->pull);
-    set_cond(h_loop, go);
-    if (prev) *prev = DevStats{};
+    bfs_decide(c, st, prev, h_loop, h_push, h_pull, h_sweep, first);
 }
 
 // BFS prologue on the device: level[src] = 0, in = {src}, visited |= {src} (src, level from ctrl).

@@ -5,6 +5,7 @@
 //   and the per-frontier statistics (n_f, m_f) the direction policy needs.
 #include "common.cuh"
 #include "kernels.h"
+#include "bfsstep.cuh"
 
 namespace sg {
 
@@ -348,32 +349,31 @@ void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src,
 }
 
 // Output of a diff-mode BFS superstep (FnBfs::diff, the sweep): the vertices first visited by
-// the step are new = visited & ~vis_old.  A warp owns 32 layer-1 words (half a layer-2 word): it
-// reads the 32 word pairs coalesced (one per lane), writes the changed words' vis_old and output
-// bits and ORs its half of the layer-2 word (one atomic per warp).  The changed words' vertices
-// are then handled 8 words per round, one half-warp per word: a thread reads the degree codes of
-// a quad of 4 vertices (m_f; the 4 loads of a round issued together, so a round costs one memory
-// latency) and stores the levels of vertices lane16 + 16 i (whole 64-B runs of level[] per store
-// instruction).  n_f / m_f of the output frontier (direction policy) come out of the same pass.
+// the step are new = visited & ~vis_old.  A CTA of 8 warps takes 256 layer-1 words (4 layer-2
+// words) per iteration, a warp 32 of them: it reads the word pairs coalesced (one per lane) and
+// writes every output word (zero or not) and the changed words' vis_old; the CTA then writes its
+// 4 layer-2 words and appends the changed words to the word list (bfs_emit_words).  The changed
+// words' vertices are handled 8 words per round, one half-warp per word: a thread reads the
+// degree codes of a quad of 4 vertices (m_f; the 4 loads of a round issued together, so a round
+// costs one memory latency) and stores the levels of vertices lane16 + 16 i (whole 64-B runs of
+// level[] per store instruction).  The last CTA decides the next superstep (graph mode).
 #ifndef SG_DIFF_WPR
 #define SG_DIFF_WPR 8
 #endif
-#ifndef SG_DIFF_MINB
-#define SG_DIFF_MINB 1
-#endif
 constexpr int DIFF_WORDS_PER_ROUND = SG_DIFF_WPR;
-__global__ void __launch_bounds__(256, SG_DIFF_MINB) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited, BfsOut o) {
-    const int lane = lane_id();
+constexpr int DIFF_THREADS = 256;
+__global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited, BfsOut o) {
+    __shared__ uint64_t s_S[DIFF_THREADS / 64];
+    __shared__ uint32_t s_ch[DIFF_THREADS / 32];
+    __shared__ uint32_t s_base;
+    const int lane = lane_id(), wid = threadIdx.x >> 5;
     const int half = lane >> 4;
     const int sh = (lane & 15) * 4;
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t nchunks = (g.nw1 + 31) >> 5;
     unsigned long long nf = 0, mf = 0;
     uint32_t *lvl = nullptr;
     uint32_t nx = 0;
-    for (int64_t ck = gw; ck < nchunks; ck += nwarps) {
-        const int64_t w0 = ck * 32;
+    for (int64_t base = blockIdx.x * (int64_t)DIFF_THREADS; base < g.nw1; base += (int64_t)gridDim.x * DIFF_THREADS) {
+        const int64_t w0 = base + wid * 32;
         const int64_t wa = w0 + lane;
         uint64_t na = 0, oa = 0;
         if (wa < g.nw1) {
@@ -382,16 +382,18 @@ __global__ void __launch_bounds__(256, SG_DIFF_MINB) k_bfs_diff(GraphView g, con
         }
         const uint64_t da = na & ~oa;
         uint32_t ch = __ballot_sync(0xffffffffu, da != 0);
-        if (!ch) continue;
-        if (!lvl) {
+        if (lane == 0) s_ch[wid] = ch;
+        if (wa < g.nw1) o.out_bits[wa] = da;
+        if (da) o.vis_old[wa] = na;
+        __syncthreads();
+        if (threadIdx.x < DIFF_THREADS / 64)
+            s_S[threadIdx.x] = (uint64_t)s_ch[2 * threadIdx.x] | ((uint64_t)s_ch[2 * threadIdx.x + 1] << 32);
+        __syncthreads();
+        bfs_emit_words(o, g.nw2, base >> 6, s_S, DIFF_THREADS / 64, &s_base);
+        if (ch && !lvl) {
             lvl = o.level_pp ? *o.level_pp : o.level;
             nx = o.next_ptr ? *o.next_ptr : o.next;
         }
-        if (da) {
-            o.vis_old[wa] = na;
-            o.out_bits[wa] = da;
-        }
-        if (lane == 0) atomic_or_u64(o.out_summ + (w0 >> 6), (uint64_t)ch << (w0 & 63));
         while (ch) {
             int wi[DIFF_WORDS_PER_ROUND / 2];   // this half-warp's words of the round (-1: none)
 #pragma unroll
@@ -433,32 +435,14 @@ __global__ void __launch_bounds__(256, SG_DIFF_MINB) k_bfs_diff(GraphView g, con
             }
         }
     }
-    __shared__ unsigned long long s_mf[8], s_nf[8];
-    mf = warp_sum(mf);
-    nf = warp_sum(nf);
-    if (lane == 0) {
-        s_mf[threadIdx.x >> 5] = mf;
-        s_nf[threadIdx.x >> 5] = nf;
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned long long a = 0, b = 0;
-        for (int i = 0; i < (int)(blockDim.x >> 5); i++) {
-            a += s_mf[i];
-            b += s_nf[i];
-        }
-        if (a | b) {
-            atomicAdd(&o.st->mf, a);
-            atomicAdd(&o.st->nf, b);
-        }
-    }
+    bfs_finish(o, nf, mf, 0ull, nullptr);
 }
 void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s) {
-    int64_t blocks = ((g.nw1 + 31) / 32 * 32 + 255) / 256;   // one warp per 32 layer-1 words
+    int64_t blocks = (g.nw1 + DIFF_THREADS - 1) / DIFF_THREADS;   // 256 layer-1 words per CTA
     if (blocks > 148 * 8 * 4) blocks = 148 * 8 * 4;
     if (blocks < 1) blocks = 1;
     note_launch();
-    k_bfs_diff<<<(int)blocks, 256, 0, s>>>(g, visited, o);
+    k_bfs_diff<<<(int)blocks, DIFF_THREADS, 0, s>>>(g, visited, o);
 }
 void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(p, n); }
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s) {

@@ -76,17 +76,25 @@ void launch_push_bc(const PushLaunch &L, const BcArgs &a, cudaStream_t s);
 int push_max_grid_words();
 int push_max_grid_heavy();
 
-// Output of a BFS superstep: new = visited & ~vis_old -> out 2LB (+ summary), level[new] = next,
-// vis_old |= new, st->nf / st->mf of the output frontier (st zeroed before).  Graph mode reads
-// `next` / `level` through next_ptr / level_pp (BfsCtrl).
+// Output of a BFS superstep: new = visited & ~vis_old -> out 2LB, level[new] = next,
+// vis_old |= new, the output's compacted word list (out offsets, st->count) and st->nf / st->mf
+// (st zeroed before).  Every layer-1 and layer-2 word of the output is written (zero or not), so
+// a BFS frontier never needs clearing.  Graph mode reads `next` / `level` through next_ptr /
+// level_pp and, with ctrl set, the last CTA to finish runs the device-side direction policy
+// (k_bfs_decide's logic: handles of the next superstep, prev = the input's control block).
 struct BfsOut {
     uint64_t *vis_old;
     uint64_t *out_bits, *out_summ;
+    uint32_t *out_offsets;
     uint32_t *level;
     uint32_t next;
     const uint32_t *next_ptr;
     uint32_t *const *level_pp;
     DevStats *st;
+    BfsCtrl *ctrl;                    // NULL: host loop (no device-side decision)
+    DevStats *prev;
+    unsigned int *done;               // CTA completion counter (self-resetting)
+    unsigned long long h_loop, h_push, h_pull, h_sweep;
 };
 // pull.cu — bottom-up BFS step (direction-optimising, Beamer): writes its output `o`
 // itself (no k_bfs_diff after it); o.out_bits == NULL: marks visited only (k_bfs_diff after it)
