@@ -8,6 +8,20 @@
 
 namespace sg {
 
+// m_f of a quad of 4 vertices: degree codes `codes` (4 bytes), vertices `mask` (4 bits), decoded
+// through a 256-entry table in shared memory (filled by deg8_lut_init; 1 LDS per vertex instead
+// of the ~10-op decode)
+__device__ __forceinline__ void deg8_lut_init(uint32_t *lut) {
+    for (int i = threadIdx.x; i < 256; i += blockDim.x) lut[i] = deg8_decode((uint32_t)i);
+}
+__device__ __forceinline__ unsigned long long quad_mf(const uint32_t *lut, uint32_t codes, uint32_t mask) {
+    unsigned long long m = 0;
+#pragma unroll
+    for (int k = 0; k < 4; k++)
+        if ((mask >> k) & 1u) m += lut[(codes >> (8 * k)) & 0xffu];
+    return m;
+}
+
 __device__ __forceinline__ void bfs_set_cond(unsigned long long h, unsigned v) {
     if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, v);
 }

@@ -365,7 +365,8 @@ constexpr int DIFF_THREADS = 256;
 __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited, BfsOut o) {
     __shared__ uint64_t s_S[DIFF_THREADS / 64];
     __shared__ uint32_t s_ch[DIFF_THREADS / 32];
-    __shared__ uint32_t s_base;
+    __shared__ uint32_t s_base, s_lut[256];
+    deg8_lut_init(s_lut);   // visible after the loop's first __syncthreads
     const int lane = lane_id(), wid = threadIdx.x >> 5;
     const int half = lane >> 4;
     const int sh = (lane & 15) * 4;
@@ -420,9 +421,7 @@ __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const ui
 #pragma unroll
             for (int j = 0; j < DIFF_WORDS_PER_ROUND / 2; j++) {
                 nf += __popc(mine[j]);
-#pragma unroll
-                for (int k = 0; k < 4; k++)
-                    mf += ((mine[j] >> k) & 1u) ? deg8_decode((codes[j] >> (8 * k)) & 0xffu) : 0u;
+                mf += quad_mf(s_lut, codes[j], mine[j]);
                 // level stores strided over the half-warp (vertex 16 i + lane16): each store
                 // instruction writes 64 contiguous bytes of level[] instead of 16 scattered quads
                 const uint32_t sp = spread[j];

@@ -36,6 +36,9 @@ constexpr int PULL_ARCS = SG_PULL_ARCS;
 #define SG_PULL_WAVES 16   // CTAs per SM in the grid (x 148)
 #endif   // arcs in flight per step of a list scan
 
+#ifndef SG_PULL_PF
+#define SG_PULL_PF 0   // 1: load the next round's visited word one round ahead
+#endif
 #ifndef SG_PULL_MINB
 #define SG_PULL_MINB 8
 #endif
@@ -43,7 +46,9 @@ __global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
            BfsOut o) {
     __shared__ uint64_t s_wm[PULL_THREADS / 32], s_S[1];
-    __shared__ uint32_t s_base;
+    __shared__ uint32_t s_base, s_lut[256];
+    deg8_lut_init(s_lut);
+    __syncthreads();
     uint32_t *const lvl = o.level_pp ? *o.level_pp : o.level;
     const uint32_t nx = o.next_ptr ? *o.next_ptr : o.next;
     unsigned long long nf = 0, mf = 0, arcs = 0;
@@ -52,6 +57,11 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
     const int64_t nq = g.nw1 * 16;
     const uint32_t half = (lane < 16) ? 0x0000ffffu : 0xffff0000u;
     // a CTA takes one layer-2 word (64 layer-1 words = 1,024 quads) in 4 rounds of 256 quads
+    // the next round's visited word is loaded one round ahead (it does not depend on this round)
+    auto vis_at = [&](int64_t qd) -> uint64_t { return qd < nq ? visited[qd >> 4] : ~0ull; };
+#if SG_PULL_PF
+    uint64_t vis_next = vis_at((int64_t)blockIdx.x * 1024 + threadIdx.x);
+#endif
     for (int64_t sw = blockIdx.x; sw < g.nw2; sw += gridDim.x) {
         uint64_t wm = 0;   // the warp's changed words within the layer-2 word
 #pragma unroll 1
@@ -60,7 +70,12 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             const bool ok = qd < nq;
             const int64_t w = qd >> 4;
             const int sh = (int)(qd & 15) * 4;
-            const uint64_t vis = ok ? visited[w] : ~0ull;
+#if SG_PULL_PF
+            const uint64_t vis = vis_next;
+            vis_next = vis_at(r < 3 ? qd + PULL_THREADS : (sw + gridDim.x) * 1024 + threadIdx.x);
+#else
+            const uint64_t vis = vis_at(qd);
+#endif
             const int64_t v0 = w * 64 + sh;
             const int64_t rem = g.n - v0;
             const uint32_t valid = !ok ? 0u : rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
@@ -111,8 +126,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                                 ((uint64_t)__reduce_or_sync(half, (uint32_t)(mine >> 32)) << 32);
             if (found) {   // n_f / m_f of the vertices found here
                 nf += __popc(found);
-#pragma unroll
-                for (int k = 0; k < 4; k++) mf += ((found >> k) & 1u) ? deg8_decode((codes >> (8 * k)) & 0xffu) : 0u;
+                mf += quad_mf(s_lut, codes, found);
             }
             if (nb) {   // level[] of the word's new vertices, strided over the half-warp (vertex
                         // 16 i + lane16): each store instruction writes 64 contiguous bytes
