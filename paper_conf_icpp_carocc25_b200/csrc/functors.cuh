@@ -46,6 +46,9 @@ __device__ __forceinline__ void insert_batch(const OutSink &out, const int32_t (
 // diff mode (run_bfs): the arc only ORs v's visited bit, a fire-and-forget RED with no result
 // to wait for; k_bfs_diff then derives the output frontier, level[] and the frontier
 // statistics from visited & ~visited_before in one pass over the bitmap (same result set).
+#ifndef SG_HEAVY_NOPROBE
+#define SG_HEAVY_NOPROBE 1
+#endif
 struct FnBfs {
     static constexpr bool kWeights = false;
     static constexpr bool kSeg = true;      // hubs may take the destination-segmented tier
@@ -60,6 +63,8 @@ struct FnBfs {
     uint32_t diff;              // 1: mark visited only (k_bfs_diff builds the output)
     __device__ __forceinline__ Ctx ctx(int32_t) const { return 0u; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return ld_word(visited + (v >> 6)); }
+    // CTA tier in diff mode: no probe, every arc issues its RED (no load latency to wait for)
+    __device__ __forceinline__ bool skip_probe() const { return SG_HEAVY_NOPROBE && diff; }
     template <int K>
     __device__ __forceinline__ void act_batch(const Ctx (&)[K], const int32_t (&v)[K], const uint32_t (&)[K],
                                               const Probe (&pr)[K], const bool (&ok)[K]) const {
@@ -101,6 +106,7 @@ struct FnSssp {
     uint32_t *dist;
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return *(volatile uint32_t *)(dist + u); }
+    __device__ __forceinline__ bool skip_probe() const { return false; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return dist[v]; }
     template <int K>
     __device__ __forceinline__ void act_batch(const Ctx (&du)[K], const int32_t (&v)[K], const uint32_t (&w)[K],
@@ -130,6 +136,7 @@ struct FnCc {
     int32_t *label;
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return *(volatile int32_t *)(label + u); }
+    __device__ __forceinline__ bool skip_probe() const { return false; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return label[v]; }
     template <int K>
     __device__ __forceinline__ void act_batch(const Ctx (&lu)[K], const int32_t (&v)[K], const uint32_t (&)[K],
@@ -160,6 +167,7 @@ struct FnBcSigma {
     uint32_t next;
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return sigma[u]; }
+    __device__ __forceinline__ bool skip_probe() const { return false; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return __ldg(visited + (v >> 6)); }
     template <int K>
     __device__ __forceinline__ void act_batch(const Ctx (&su)[K], const int32_t (&v)[K], const uint32_t (&)[K],

@@ -359,7 +359,7 @@ __global__ void __launch_bounds__(HEAVY_THREADS) k_push_heavy(PushParams p, F f)
                 cc[k] = c;
             }
 #pragma unroll
-            for (int k = 0; k < KH; k++) pr[k] = ok[k] ? f.probe(v[k]) : typename F::Probe{};
+            for (int k = 0; k < KH; k++) pr[k] = ok[k] && !f.skip_probe() ? f.probe(v[k]) : typename F::Probe{};
             f.act_batch(cc, v, w, pr, ok);
         }
         __syncthreads();   // buffer s fully consumed
