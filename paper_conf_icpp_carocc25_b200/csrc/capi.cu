@@ -857,6 +857,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         if (sc) TRY(add_cond(body, deps, h_sweep[half], cudaGraphCondTypeIf, &n_sweep, &b_sweep));
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
+        L.sparse_ok = 1;  // n_f of every BFS frontier is exact (prologue statistics / output kernels)
         BfsArgs a{ws->visited, nullptr, 0u, nullptr, nullptr, &ws->ctrl->next, &ws->ctrl->level, 1u};
         // output of the superstep (out->st was zeroed by the previous decision / the prologue);
         // the output kernel's last CTA decides the next superstep (handles of the other half)
@@ -1010,6 +1011,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
             push_steps++;
         } else {
             PushLaunch L = push_launch(g, in, t, o.one_layer ? G.nw1 : count);
+            L.sparse_ok = o.one_layer ? 0 : 1;
             if (o.one_layer) {   // Fig. 7 ablation: no summary layer, every word is visited
                 if (!ws->all_offsets) CK(cudaMalloc(&ws->all_offsets, sizeof(uint32_t) * (size_t)G.nw1));
                 launch_list_all(ws->all_offsets, ws->st + 2, in->st, G.nw1, s);

@@ -52,6 +52,7 @@ struct PushLaunch {
     int32_t seg_mode = 0;            // 0 off, 1 auto, 2 always
     unsigned long long seg_threshold = 0;
     unsigned long long skip_mf = ~0ull;   // k_push_words returns at once if the frontier's m_f >= skip_mf (SCSR path)
+    int32_t sparse_ok = 0;           // st->nf is exact (BFS): sparse frontiers take the thread-per-word path
 };
 void launch_hub_mark(const int64_t *rp, int64_t n, int32_t *hub_idx, int32_t *hub_vertex, unsigned int *count,
                      cudaStream_t s);

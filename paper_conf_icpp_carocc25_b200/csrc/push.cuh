@@ -26,6 +26,9 @@
 
 namespace sg {
 
+#ifndef SG_SPARSE_WORDS
+#define SG_SPARSE_WORDS 1
+#endif
 constexpr int PUSH_THREADS = 256;
 constexpr int PUSH_WARPS = PUSH_THREADS / 32;
 constexpr int HEAVY_THREADS = 256;
@@ -48,6 +51,8 @@ struct PushParams {
     int32_t seg_mode;      // 0 off, 1 auto (when the frontier's m_f >= seg_threshold), 2 always
     unsigned long long seg_threshold;
     unsigned long long skip_mf;   // the segmented (SCSR) advance handles this superstep: m_f >= skip_mf
+    int32_t sparse_ok;     // st->nf is exact: words with <= 2 active vertices on average take the
+                           // thread-per-word path (push_words_sparse)
 };
 
 template <class F>
@@ -242,6 +247,82 @@ __device__ __forceinline__ unsigned long long push_word(const PushParams &p, con
     return (unsigned long long)d_total;
 }
 
+// ---- sparse frontiers: one thread per word -------------------------------------------------
+// When the words hold <= 2 active vertices on average (n_f <= 2 count) of low average degree
+// (m_f <= 16 n_f: the leaf levels of a BFS),
+// a warp-per-word mapping runs the word's dependent load chain (word -> row_ptr -> col_idx ->
+// probe) once per word per warp.  Here each lane takes one word: its vertices' low-degree lists
+// are expanded by the lane itself (4 arcs in flight), up to 2 mid-degree vertices per lane are
+// expanded afterwards by the whole warp, hubs go to the CTA / segmented tiers as usual.
+template <class F>
+__device__ __forceinline__ void thread_expand(const GraphView &g, const F &f, int64_t s, int64_t e,
+                                              typename F::Ctx c) {
+    for (int64_t r = s; r < e; r += 4) {
+        int32_t v[4];
+        uint32_t w[4];
+        bool ok[4];
+        typename F::Probe pr[4];
+        typename F::Ctx cc[4];
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            ok[k] = r + k < e;
+            v[k] = ok[k] ? __ldg(g.col + r + k) : 0;
+            w[k] = ok[k] ? load_w<F>(g, r + k) : 0u;
+            cc[k] = c;
+        }
+#pragma unroll
+        for (int k = 0; k < 4; k++) pr[k] = ok[k] ? f.probe(v[k]) : typename F::Probe{};
+        f.act_batch(cc, v, w, pr, ok);
+    }
+}
+template <class F>
+__device__ __forceinline__ unsigned long long push_words_sparse(const PushParams &p, const F &f, uint32_t i,
+                                                                uint32_t count, bool seg_on) {
+    unsigned long long arcs = 0;
+    int64_t ds[2] = {0, 0}, de[2] = {0, 0};
+    int32_t du[2] = {-1, -1};
+    int nd = 0;
+    if (i < count) {
+        const int64_t w = p.offsets[i];
+        uint64_t x = __ldg(p.in_bits + w);
+        while (x) {
+            const int b = __ffsll((long long)x) - 1;
+            x &= x - 1;
+            const int32_t u = (int32_t)(w * 64 + b);
+            const int64_t s = __ldg(p.g.rp + u), e = __ldg(p.g.rp + u + 1);
+            const int64_t d = e - s;
+            arcs += (unsigned long long)d;
+            if constexpr (F::kSeg) {
+                if (seg_on && d >= SEG_MIN) {
+                    enqueue_seg(p, __ldg(p.g.hub_idx + u), s, e);
+                    continue;
+                }
+            }
+            if (d > p.heavy_deg) {
+                enqueue_heavy(p, u, s, e);
+            } else if (d > p.small_deg && nd < 2) {
+                ds[nd] = s;
+                de[nd] = e;
+                du[nd] = u;
+                nd++;
+            } else if (d > 0) {
+                thread_expand(p.g, f, s, e, f.ctx(u));
+            }
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < 2; k++) {   // mid-degree vertices: the whole warp, one at a time
+        uint32_t mm = __ballot_sync(0xffffffffu, du[k] >= 0);
+        while (mm) {
+            const int src = __ffs(mm) - 1;
+            mm &= mm - 1;
+            const int32_t u = __shfl_sync(0xffffffffu, du[k], src);
+            warp_expand(p.g, f, __shfl_sync(0xffffffffu, ds[k], src), __shfl_sync(0xffffffffu, de[k], src), f.ctx(u));
+        }
+    }
+    return arcs;
+}
+
 template <class F>
 __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) {
     __shared__ PushWarpSmem<F> s_warp[PUSH_WARPS];
@@ -261,13 +342,26 @@ __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) 
     if constexpr (F::kSeg)
         seg_on = p.g.hub_idx != nullptr && p.seg != nullptr &&
                  (p.seg_mode == 2 || (p.seg_mode == 1 && p.st->mf >= p.seg_threshold));
-    for (;;) {
-        uint32_t b0 = 0;
-        if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)batch);
-        b0 = __shfl_sync(0xffffffffu, b0, 0);
-        if (b0 >= count) break;
-        const uint32_t b1 = min(b0 + batch, count);
-        for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid], seg_on);
+    // sparse: <= 2 active vertices per word on average, of average degree <= 16 (else the
+    // warp-tier vertices of 32 words would serialise on one warp)
+    const bool sparse = SG_SPARSE_WORDS && p.sparse_ok && p.st->nf <= 2ull * count && p.st->mf <= 16ull * p.st->nf;
+    if (sparse) {
+        for (;;) {   // 32 words per warp grab, one per lane
+            uint32_t b0 = 0;
+            if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, 32ull);
+            b0 = __shfl_sync(0xffffffffu, b0, 0);
+            if (b0 >= count) break;
+            arcs += push_words_sparse(p, f, b0 + lane_id(), count, seg_on);
+        }
+    } else {
+        for (;;) {
+            uint32_t b0 = 0;
+            if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)batch);
+            b0 = __shfl_sync(0xffffffffu, b0, 0);
+            if (b0 >= count) break;
+            const uint32_t b1 = min(b0 + batch, count);
+            for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid], seg_on);
+        }
     }
     arcs = warp_sum(arcs);
     if (lane_id() == 0) s_arcs[wid] = arcs;
