@@ -357,6 +357,9 @@ void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src,
 // degree codes of a quad of 4 vertices (m_f; the 4 loads of a round issued together, so a round
 // costs one memory latency) and stores the levels of vertices lane16 + 16 i (whole 64-B runs of
 // level[] per store instruction).  The last CTA decides the next superstep (graph mode).
+#ifndef SG_DIFF_BLOCKS
+#define SG_DIFF_BLOCKS (148 * 4)   // grid cap (CTAs)
+#endif
 #ifndef SG_DIFF_WPR
 #define SG_DIFF_WPR 8
 #endif
@@ -438,7 +441,7 @@ __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const ui
 }
 void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s) {
     int64_t blocks = (g.nw1 + DIFF_THREADS - 1) / DIFF_THREADS;   // 256 layer-1 words per CTA
-    if (blocks > 148 * 8 * 4) blocks = 148 * 8 * 4;
+    if (blocks > SG_DIFF_BLOCKS) blocks = SG_DIFF_BLOCKS;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_bfs_diff<<<(int)blocks, DIFF_THREADS, 0, s>>>(g, visited, o);

@@ -46,6 +46,9 @@ __device__ __forceinline__ void insert_batch(const OutSink &out, const int32_t (
 // diff mode (run_bfs): the arc only ORs v's visited bit, a fire-and-forget RED with no result
 // to wait for; k_bfs_diff then derives the output frontier, level[] and the frontier
 // statistics from visited & ~visited_before in one pass over the bitmap (same result set).
+#ifndef SG_WORDS_NOPROBE
+#define SG_WORDS_NOPROBE 1
+#endif
 #ifndef SG_HEAVY_NOPROBE
 #define SG_HEAVY_NOPROBE 1
 #endif
@@ -65,6 +68,8 @@ struct FnBfs {
     __device__ __forceinline__ Probe probe(int32_t v) const { return ld_word(visited + (v >> 6)); }
     // CTA tier in diff mode: no probe, every arc issues its RED (no load latency to wait for)
     __device__ __forceinline__ bool skip_probe() const { return SG_HEAVY_NOPROBE && diff; }
+    // word-path tiers (warp / thread) in diff mode: SG_WORDS_NOPROBE = 1 skips their probes too
+    __device__ __forceinline__ bool skip_probe_words() const { return SG_WORDS_NOPROBE && diff; }
     template <int K>
     __device__ __forceinline__ void act_batch(const Ctx (&)[K], const int32_t (&v)[K], const uint32_t (&)[K],
                                               const Probe (&pr)[K], const bool (&ok)[K]) const {
@@ -106,6 +111,7 @@ struct FnSssp {
     uint32_t *dist;
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return *(volatile uint32_t *)(dist + u); }
+    __device__ __forceinline__ bool skip_probe_words() const { return false; }
     __device__ __forceinline__ bool skip_probe() const { return false; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return dist[v]; }
     template <int K>
@@ -136,6 +142,7 @@ struct FnCc {
     int32_t *label;
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return *(volatile int32_t *)(label + u); }
+    __device__ __forceinline__ bool skip_probe_words() const { return false; }
     __device__ __forceinline__ bool skip_probe() const { return false; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return label[v]; }
     template <int K>
@@ -167,6 +174,7 @@ struct FnBcSigma {
     uint32_t next;
     OutSink out;
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return sigma[u]; }
+    __device__ __forceinline__ bool skip_probe_words() const { return false; }
     __device__ __forceinline__ bool skip_probe() const { return false; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return __ldg(visited + (v >> 6)); }
     template <int K>

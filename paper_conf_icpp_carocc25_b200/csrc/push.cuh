@@ -83,7 +83,7 @@ __device__ __forceinline__ void warp_expand(const GraphView &g, const F &f, int6
         if (i >= 0) {
             const int32_t v[1] = {__ldg(g.col + i)};
             const uint32_t w[1] = {load_w<F>(g, i)};
-            const typename F::Probe pr[1] = {f.probe(v[0])};
+            const typename F::Probe pr[1] = {f.skip_probe_words() ? typename F::Probe{} : f.probe(v[0])};
             const typename F::Ctx cc[1] = {c};
             const bool ok[1] = {true};
             f.act_batch(cc, v, w, pr, ok);
@@ -107,7 +107,7 @@ __device__ __forceinline__ void warp_expand(const GraphView &g, const F &f, int6
         typename F::Ctx cc[8];
 #pragma unroll
         for (int k = 0; k < 8; k++) {
-            pr[k] = ok[k] ? f.probe(v[k]) : typename F::Probe{};
+            pr[k] = ok[k] && !f.skip_probe_words() ? f.probe(v[k]) : typename F::Probe{};
             cc[k] = c;
         }
         f.act_batch(cc, v, w, pr, ok);
@@ -237,8 +237,8 @@ __device__ __forceinline__ unsigned long long push_word(const PushParams &p, con
                 cc[1] = sm.ctx[k1];
             }
             typename F::Probe pr[2] = {};
-            if (ok0) pr[0] = f.probe(v[0]);
-            if (ok1) pr[1] = f.probe(v[1]);
+            if (ok0 && !f.skip_probe_words()) pr[0] = f.probe(v[0]);
+            if (ok1 && !f.skip_probe_words()) pr[1] = f.probe(v[1]);
             f.act_batch(cc, v, w, pr, ok);
             kb += __popcll(mask);
         }
@@ -271,7 +271,7 @@ __device__ __forceinline__ void thread_expand(const GraphView &g, const F &f, in
             cc[k] = c;
         }
 #pragma unroll
-        for (int k = 0; k < 4; k++) pr[k] = ok[k] ? f.probe(v[k]) : typename F::Probe{};
+        for (int k = 0; k < 4; k++) pr[k] = ok[k] && !f.skip_probe_words() ? f.probe(v[k]) : typename F::Probe{};
         f.act_batch(cc, v, w, pr, ok);
     }
 }
@@ -345,23 +345,25 @@ __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) 
     // sparse: <= 2 active vertices per word on average, of average degree <= 16 (else the
     // warp-tier vertices of 32 words would serialise on one warp)
     const bool sparse = SG_SPARSE_WORDS && p.sparse_ok && p.st->nf <= 2ull * count && p.st->mf <= 16ull * p.st->nf;
-    if (sparse) {
-        for (;;) {   // 32 words per warp grab, one per lane
-            uint32_t b0 = 0;
-            if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, 32ull);
-            b0 = __shfl_sync(0xffffffffu, b0, 0);
-            if (b0 >= count) break;
+    // a warp's first grab is static (warp id x grab), later ones dynamic (after all static
+    // grabs): a small frontier costs no atomic storm of idle warps on one counter
+    const uint32_t gwarp = (blockIdx.x * PUSH_THREADS + threadIdx.x) >> 5;
+    const uint32_t nwarps = gridDim.x * PUSH_WARPS;
+    const uint32_t grab = sparse ? 32u : batch;
+    const unsigned long long statics = (unsigned long long)nwarps * grab;
+    for (unsigned long long b0l = (unsigned long long)gwarp * grab;;) {
+        if (b0l >= count) break;
+        const uint32_t b0 = (uint32_t)b0l;
+        if (sparse) {   // 32 words per grab, one per lane
             arcs += push_words_sparse(p, f, b0 + lane_id(), count, seg_on);
-        }
-    } else {
-        for (;;) {
-            uint32_t b0 = 0;
-            if (lane_id() == 0) b0 = (uint32_t)atomicAdd(&p.st->batch, (unsigned long long)batch);
-            b0 = __shfl_sync(0xffffffffu, b0, 0);
-            if (b0 >= count) break;
-            const uint32_t b1 = min(b0 + batch, count);
+        } else {
+            const uint32_t b1 = min(b0 + grab, count);
             for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid], seg_on);
         }
+        if (statics >= count) break;
+        unsigned long long nb = 0;
+        if (lane_id() == 0) nb = statics + atomicAdd(&p.st->batch, (unsigned long long)grab);
+        b0l = __shfl_sync(0xffffffffu, nb, 0);
     }
     arcs = warp_sum(arcs);
     if (lane_id() == 0) s_arcs[wid] = arcs;
