@@ -828,18 +828,15 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     std::vector<cudaGraphNode_t> leaves;
     // prologue: level = INF, frontiers cleared, visited = isolated, seed src, compact + decide
     TRY(capture_begin(cs, root, {}));
-    launch_bfs_level_init(ws->ctrl, G.n, cs);
-    for (int i = 0; i < 2; i++) {
-        CK(cudaMemsetAsync(F[i]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
-        CK(cudaMemsetAsync(F[i]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
-    }
+    // (the output frontier F[1] is written whole by the first output kernel: only F[0] is zeroed)
+    CK(cudaMemsetAsync(F[0]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
+    CK(cudaMemsetAsync(F[0]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
     CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), cs));
     CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
     CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
-    launch_bfs_seed(ws->ctrl, F[0]->bits, F[0]->summ, ws->visited, ws->vis_old, cs);
-    launch_compact(F[0]->summ, G.nw2, F[0]->offsets, F[0]->st, cs);
-    launch_frontier_stats(G, F[0]->bits, F[0]->st, cs);
-    launch_bfs_decide(ws->ctrl, F[0]->st, nullptr, h_loop, h_push[0], h_pull[0], sc ? h_sweep[0] : 0ull, 1, cs);
+    launch_bfs_prologue(ws->ctrl, G.n, G.deg8, F[0]->bits, F[0]->summ, F[0]->offsets, F[0]->st, ws->visited,
+                        ws->vis_old, (unsigned long long)h_loop, (unsigned long long)h_push[0],
+                        (unsigned long long)h_pull[0], sc ? (unsigned long long)h_sweep[0] : 0ull, cs);
     TRY(capture_end(cs, leaves));
     cudaGraphNode_t wnode;
     cudaGraph_t body;
@@ -923,11 +920,11 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     CK(cudaGetLastError());
     if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
     {
-        // kernels the graph executed: prologue (level init, seed, compact, stats, decide) + the
+        // kernels the graph executed: the prologue kernel + the
         // taken IF bodies (push = word + CTA tier [+ hub segment tier] + output, sweep = arc
         // count + sweep + output, pull = 1)
         const long long per_push = 3 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
-        const long long k = 5 + per_push * (long long)(c.push_steps - c.sweep_steps) + 3 * (long long)c.sweep_steps +
+        const long long k = 1 + per_push * (long long)(c.push_steps - c.sweep_steps) + 3 * (long long)c.sweep_steps +
                             (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }

@@ -82,6 +82,53 @@ void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t 
     k_bfs_seed<<<1, 1, 0, s>>>(c, bits, summ, visited, vis_old);
 }
 
+// The whole BFS prologue in one kernel (graph mode): level[] = INF except level[src] = 0
+// (16-B stores, buffer pointer from ctrl), and on one thread: in = {src} (layer 1 / 2 bits, word
+// list, n_f = 1, m_f = src's coded degree, as the compaction + statistics kernels would give),
+// visited |= {src}, then the first direction decision.  The frontier's words were zeroed before.
+__global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
+                               uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
+                               unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
+                               unsigned long long h_sweep) {
+    uint32_t *level = c->level;
+    const int32_t src = c->src;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (((uintptr_t)level & 15) == 0) {
+        uint4 *l4 = reinterpret_cast<uint4 *>(level);
+        for (int64_t i = t; i < n / 4; i += stride) {
+            uint4 q = make_uint4(INF32, INF32, INF32, INF32);
+            if (i == (src >> 2)) (&q.x)[src & 3] = 0u;
+            l4[i] = q;
+        }
+        for (int64_t i = (n / 4) * 4 + t; i < n; i += stride) level[i] = i == src ? 0u : INF32;
+    } else {
+        for (int64_t i = t; i < n; i += stride) level[i] = i == src ? 0u : INF32;
+    }
+    if (t == 0) {
+        bits[src >> 6] = 1ull << (src & 63);
+        summ[src >> 12] = 1ull << ((src >> 6) & 63);
+        visited[src >> 6] |= 1ull << (src & 63);
+        vis_old[src >> 6] |= 1ull << (src & 63);
+        offsets[0] = (uint32_t)(src >> 6);
+        st->count = 1ull;
+        st->nf = 1ull;
+        st->mf = deg8_decode(deg8[src]);
+        bfs_decide(c, st, nullptr, h_loop, h_push, h_pull, h_sweep, 1);
+    }
+}
+void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
+                         uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
+                         unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
+                         unsigned long long h_sweep, cudaStream_t s) {
+    int64_t blocks = (n / 4 + 255) / 256;
+    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_bfs_prologue<<<(int)blocks, 256, 0, s>>>(c, n, deg8, bits, summ, offsets, st, visited, vis_old, h_loop, h_push,
+                                               h_pull, h_sweep);
+}
+
 // level[0..n) = UINT32_MAX with the buffer pointer taken from ctrl (16-B stores)
 __global__ void k_bfs_level_init(const BfsCtrl *c, int64_t n) {
     uint32_t *level = c->level;

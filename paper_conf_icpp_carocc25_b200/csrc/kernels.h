@@ -143,6 +143,11 @@ void launch_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned 
 void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,
                      cudaStream_t s);
 void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s);
+// level init + seed + the seed frontier's word list / statistics + first decision, one kernel
+void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
+                         uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
+                         unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
+                         unsigned long long h_sweep, cudaStream_t s);
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s);
 void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s);
