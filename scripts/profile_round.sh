@@ -18,6 +18,11 @@ ncu --set full --clock-control none --import-source on -k regex:k_pull_bfs -c 2 
     -o gpurun_out/${R}_full_pull python scripts/profile_one_bfs.py auto > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:k_push_sweep -c 1 \
     -o gpurun_out/${R}_full_sweep python scripts/profile_one_bfs.py push > /dev/null 2>&1
+# 4) the output pass of the dense push level and the level-2 CTA-tier (hub) push (DO)
+ncu --set full --clock-control none --import-source on -k regex:k_bfs_diff -s 2 -c 1 \
+    -o gpurun_out/${R}_full_diff python scripts/profile_one_bfs.py auto > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:k_push_heavy -s 2 -c 1 \
+    -o gpurun_out/${R}_full_heavy python scripts/profile_one_bfs.py auto > /dev/null 2>&1
 echo done
 # locally:
 #   python scripts/make_traffic.py gpurun_out/${R}_launches_do_dram.csv gpurun_out/${R}_launches_push_dram.csv > profiles/traffic.json
