@@ -27,7 +27,11 @@
 
 namespace sg {
 
-constexpr int PULL_THREADS = 256;
+#ifndef SG_PULL_THREADS
+#define SG_PULL_THREADS 256
+#endif
+constexpr int PULL_THREADS = SG_PULL_THREADS;   // 128, 256, 512 or 1024
+constexpr int PULL_ROUNDS = 1024 / PULL_THREADS;
 #ifndef SG_PULL_ARCS
 #define SG_PULL_ARCS 2
 #endif
@@ -65,14 +69,14 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
     for (int64_t sw = blockIdx.x; sw < g.nw2; sw += gridDim.x) {
         uint64_t wm = 0;   // the warp's changed words within the layer-2 word
 #pragma unroll 1
-        for (int r = 0; r < 4; r++) {
+        for (int r = 0; r < PULL_ROUNDS; r++) {
             const int64_t qd = sw * 1024 + r * PULL_THREADS + threadIdx.x;
             const bool ok = qd < nq;
             const int64_t w = qd >> 4;
             const int sh = (int)(qd & 15) * 4;
 #if SG_PULL_PF
             const uint64_t vis = vis_next;
-            vis_next = vis_at(r < 3 ? qd + PULL_THREADS : (sw + gridDim.x) * 1024 + threadIdx.x);
+            vis_next = vis_at(r < PULL_ROUNDS - 1 ? qd + PULL_THREADS : (sw + gridDim.x) * 1024 + threadIdx.x);
 #else
             const uint64_t vis = vis_at(qd);
 #endif
@@ -144,7 +148,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                 }
             }
             const uint32_t act = __ballot_sync(0xffffffffu, nb != 0ull && (lane & 15) == 0);
-            wm |= (uint64_t)((act & 1u) | ((act >> 15) & 2u)) << (r * 16 + wid * 2);
+            wm |= (uint64_t)((act & 1u) | ((act >> 15) & 2u)) << (r * (PULL_THREADS / 16) + wid * 2);
         }
         if (lane == 0) s_wm[wid] = wm;
         __syncthreads();
