@@ -13,25 +13,6 @@
 
 namespace sg {
 
-// Decide the next superstep from the freshly compacted frontier's control block `st` (the
-// prologue; later supersteps decide in the last CTA of their output kernel, bfsstep.cuh).
-__global__ void k_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
-                             unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep,
-                             int first) {
-    if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    bfs_decide(c, st, prev, h_loop, h_push, h_pull, h_sweep, first);
-}
-
-// BFS prologue on the device: level[src] = 0, in = {src}, visited |= {src} (src, level from ctrl).
-__global__ void k_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old) {
-    const int32_t src = c->src;
-    c->level[src] = 0u;
-    bits[src >> 6] = 1ull << (src & 63);
-    summ[src >> 12] = 1ull << ((src >> 6) & 63);
-    visited[src >> 6] |= 1ull << (src & 63);
-    if (vis_old) vis_old[src >> 6] |= 1ull << (src & 63);
-}
-
 // Clear a frontier after it was advanced (only its listed non-zero words + its summary) and
 // zero the control block of the frontier about to be compacted.
 __global__ void k_clear_listed(uint64_t *__restrict__ bits, uint64_t *__restrict__ summ,
@@ -68,18 +49,6 @@ void launch_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *st_src
 __global__ void k_zero_u64(unsigned long long *p, int64_t n) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += stride) p[i] = 0ull;
-}
-
-void launch_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
-                       unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep, int first,
-                       cudaStream_t s) {
-    note_launch();
-    k_bfs_decide<<<1, 32, 0, s>>>(c, st, prev, h_loop, h_push, h_pull, h_sweep, first);
-}
-void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,
-                     cudaStream_t s) {
-    note_launch();
-    k_bfs_seed<<<1, 1, 0, s>>>(c, bits, summ, visited, vis_old);
 }
 
 // The whole BFS prologue in one kernel (graph mode): level[] = INF except level[src] = 0
@@ -129,26 +98,6 @@ void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *b
                                                h_pull, h_sweep);
 }
 
-// level[0..n) = UINT32_MAX with the buffer pointer taken from ctrl (16-B stores)
-__global__ void k_bfs_level_init(const BfsCtrl *c, int64_t n) {
-    uint32_t *level = c->level;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (((uintptr_t)level & 15) == 0) {
-        uint4 *l4 = reinterpret_cast<uint4 *>(level);
-        for (int64_t i = t; i < n / 4; i += stride) l4[i] = make_uint4(INF32, INF32, INF32, INF32);
-        for (int64_t i = (n / 4) * 4 + t; i < n; i += stride) level[i] = INF32;
-    } else {
-        for (int64_t i = t; i < n; i += stride) level[i] = INF32;
-    }
-}
-void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s) {
-    int64_t blocks = (n / 4 + 255) / 256;
-    if (blocks > 148 * 8) blocks = 148 * 8;
-    if (blocks < 1) blocks = 1;
-    note_launch();
-    k_bfs_level_init<<<(int)blocks, 256, 0, s>>>(c, n);
-}
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s) {
     int64_t blocks = (nw1 + 255) / 256;

@@ -137,12 +137,6 @@ void launch_push_sweep(const ScsrView &v, const int64_t *rp, const uint64_t *in_
                        unsigned long long min_mf, cudaStream_t s);
 
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
-void launch_bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
-                       unsigned long long h_push, unsigned long long h_pull, unsigned long long h_sweep, int first,
-                       cudaStream_t s);
-void launch_bfs_seed(const BfsCtrl *c, uint64_t *bits, uint64_t *summ, uint64_t *visited, uint64_t *vis_old,
-                     cudaStream_t s);
-void launch_bfs_level_init(const BfsCtrl *c, int64_t n, cudaStream_t s);
 // level init + seed + the seed frontier's word list / statistics + first decision, one kernel
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                          uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
