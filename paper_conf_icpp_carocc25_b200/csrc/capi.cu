@@ -299,25 +299,25 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     g->v.nw2 = (g->v.nw1 + 63) / 64;
     const cudaMemcpyKind kind = mem == SG_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
     // col_idx/weights get 64 B of zero padding: 16-B bulk copies may read up to 12 B past nnz
-    CK(cudaMalloc(&g->rp, sizeof(int64_t) * (size_t)(n + 1)));
-    CK(cudaMalloc(&g->col, sizeof(int32_t) * (size_t)nnz + 64));
+    CK(dev_alloc(&g->rp, sizeof(int64_t) * (size_t)(n + 1), s));
+    CK(dev_alloc(&g->col, sizeof(int32_t) * (size_t)nnz + 64, s));
     CK(cudaMemsetAsync((char *)g->col + sizeof(int32_t) * (size_t)nnz, 0, 64, s));
     CK(cudaMemcpyAsync(g->rp, row_ptr, sizeof(int64_t) * (size_t)(n + 1), kind, s));
     if (nnz) CK(cudaMemcpyAsync(g->col, col_idx, sizeof(int32_t) * (size_t)nnz, kind, s));
     if (weights) {
-        CK(cudaMalloc(&g->w, (size_t)nnz + 64));
+        CK(dev_alloc(&g->w, (size_t)nnz + 64, s));
         CK(cudaMemsetAsync(g->w + nnz, 0, 64, s));
         if (nnz) CK(cudaMemcpyAsync(g->w, weights, (size_t)nnz, kind, s));
     }
     g->v.rp = g->rp;
     g->v.col = g->col;
     g->v.w = g->w;
-    CK(cudaMalloc(&g->deg8, (size_t)g->v.nw1 * 64));
+    CK(dev_alloc(&g->deg8, (size_t)g->v.nw1 * 64, s));
     launch_deg8(g->rp, n, g->v.nw1 * 64, g->deg8, s);
     g->v.deg8 = g->deg8;
-    CK(cudaMalloc(&g->isolated, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(dev_alloc(&g->isolated, sizeof(uint64_t) * (size_t)g->v.nw1, s));
     launch_isolated(g->deg8, n, g->v.nw1, g->isolated, s);
-    CK(cudaMalloc(&g->fnbr, sizeof(int32_t) * (size_t)(g->v.nw1 ? g->v.nw1 * 64 : 1)));   // padded: 16-B quad loads
+    CK(dev_alloc(&g->fnbr, sizeof(int32_t) * (size_t)(g->v.nw1 ? g->v.nw1 * 64 : 1), s));   // padded: 16-B quad loads
     launch_first_nbr(g->rp, g->col, g->deg8, n, g->v.nw1 * 64, g->fnbr, s);
     g->v.fnbr = g->fnbr;
     unsigned long long *dscr = nullptr;
@@ -327,8 +327,8 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     if (g->w) launch_max_weight(g->w, nnz, reinterpret_cast<unsigned int *>(dscr + 1), s);
     // hubs of the destination-segmented BFS tier (deg >= SEG_MIN): index map + vertex list
     const int64_t max_hubs = nnz / SEG_MIN + 1;
-    CK(cudaMalloc(&g->hub_idx, sizeof(int32_t) * (size_t)n));
-    CK(cudaMalloc(&g->hub_vertex, sizeof(int32_t) * (size_t)max_hubs));
+    CK(dev_alloc(&g->hub_idx, sizeof(int32_t) * (size_t)n, s));
+    CK(dev_alloc(&g->hub_vertex, sizeof(int32_t) * (size_t)max_hubs, s));
     launch_hub_mark(g->rp, n, g->hub_idx, g->hub_vertex, reinterpret_cast<unsigned int *>(dscr + 2), s);
     unsigned long long h[3] = {0, 0, 0};
     CK(cudaMemcpyAsync(h, dscr, 24, cudaMemcpyDeviceToHost, s));
@@ -343,7 +343,7 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     g->nhubs = (int64_t)(h[2] & 0xffffffffu);
     g->v.nseg = (int32_t)((n + SEG_V - 1) / SEG_V);
     if (g->nhubs > 0) {
-        CK(cudaMalloc(&g->hub_off, sizeof(uint32_t) * (size_t)g->nhubs * (size_t)(g->v.nseg + 1)));
+        CK(dev_alloc(&g->hub_off, sizeof(uint32_t) * (size_t)g->nhubs * (size_t)(g->v.nseg + 1), s));
         launch_hub_off(g->rp, g->col, g->hub_vertex, g->nhubs, g->v.nseg, g->hub_off, s);
         CK(cudaStreamSynchronize(s));
         CK(cudaGetLastError());
@@ -356,16 +356,17 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
 
 SG_API int graph_free(sg_graph *g) {
     if (!g) return SG_OK;
+    cudaDeviceSynchronize();   // no pending work may use the buffers (cudaFree did this implicitly)
     free_ws(g->ws);
-    cudaFree(g->rp);
-    cudaFree(g->col);
-    cudaFree(g->w);
-    cudaFree(g->deg8);
-    cudaFree(g->fnbr);
-    cudaFree(g->isolated);
-    cudaFree(g->hub_idx);
-    cudaFree(g->hub_vertex);
-    cudaFree(g->hub_off);
+    dev_free(g->rp);
+    dev_free(g->col);
+    dev_free(g->w);
+    dev_free(g->deg8);
+    dev_free(g->fnbr);
+    dev_free(g->isolated);
+    dev_free(g->hub_idx);
+    dev_free(g->hub_vertex);
+    dev_free(g->hub_off);
     if (g->scsr_state == 1) scsr_free(&g->scsr);
     delete g;
     return SG_OK;

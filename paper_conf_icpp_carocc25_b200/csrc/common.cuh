@@ -177,3 +177,31 @@ __device__ __forceinline__ void word_bounds(const GraphView &g, int64_t w, uint6
 }
 
 }  // namespace sg
+
+// ---- device memory: one stream-ordered pool per process that keeps freed blocks (release
+// threshold = infinity), so a graph loaded after another one of similar size reuses its memory
+// without new driver mappings (graph_load_csr / graph_free in a loop: the e2e step).
+namespace sg {
+inline cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s) {
+    static bool init = false;
+    if (!init) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t thr = ~0ull;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        }
+        init = true;
+    }
+    return cudaMallocAsync(p, bytes, s);
+}
+template <class T>
+inline cudaError_t dev_alloc(T **p, size_t bytes, cudaStream_t s) {
+    return dev_alloc(reinterpret_cast<void **>(p), bytes, s);
+}
+// the caller guarantees no pending work uses p (graph_free synchronises the device first)
+inline void dev_free(void *p) {
+    if (p) cudaFreeAsync(p, 0);
+}
+}  // namespace sg

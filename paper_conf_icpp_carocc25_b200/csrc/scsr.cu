@@ -658,7 +658,7 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
         k_scsr_pad<<<(int)(bl < 1 ? 1 : bl), 256, 0, s>>>(wsum, nw1, nw2, nseg, upad,
                                                            reinterpret_cast<unsigned long long *>(nx_d + 2));
     }
-    SCK(cudaMalloc(&S.base, sizeof(uint32_t) * (size_t)nseg * (nw1 + 1)));
+    SCK(dev_alloc(&S.base, sizeof(uint32_t) * (size_t)nseg * (nw1 + 1), s));
     note_launch();
     k_scsr_scan<<<nseg, 1024, 0, s>>>(wsum, nw1, S.base, tot);
     SCK(cudaMemcpyAsync(&nx, nx_d, sizeof(unsigned int), cudaMemcpyDeviceToHost, s));
@@ -676,7 +676,7 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
         goto done;
     }
     S.nx = nx;
-    SCK(cudaMalloc(&S.start, sizeof(int64_t) * (size_t)nseg));
+    SCK(dev_alloc(&S.start, sizeof(int64_t) * (size_t)nseg, s));
     SCK(cudaMemcpyAsync(S.start, start.data(), sizeof(int64_t) * nseg, cudaMemcpyHostToDevice, s));
     SCK(cudaMalloc(&xoff, sizeof(uint32_t) * (size_t)(nx ? nx : 1) * (nseg + 1)));
     if (nx) {
@@ -686,9 +686,9 @@ cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t
         note_launch();
         k_scsr_xoff<<<(int)bl, 256, 0, s>>>(rp, col, xvert, nx, nseg, sv, xoff);
     }
-    SCK(cudaMalloc(&S.col, sizeof(uint32_t) * (size_t)acc + 64));
+    SCK(dev_alloc(&S.col, sizeof(uint32_t) * (size_t)acc + 64, s));
     SCK(cudaMemsetAsync((char *)S.col + sizeof(uint32_t) * (size_t)acc, 0, 64, s));
-    SCK(cudaMalloc(&S.qc, sizeof(uint32_t) * (size_t)nseg));
+    SCK(dev_alloc(&S.qc, sizeof(uint32_t) * (size_t)nseg, s));
     S.v.col = S.col;
     S.v.base = S.base;
     S.v.start = S.start;
@@ -718,15 +718,18 @@ done:
     cudaFree(xoff);
     cudaFree(nx_d);
     cudaFree(upad);
-    if (e != cudaSuccess) scsr_free(out);
+    if (e != cudaSuccess) {
+        cudaDeviceSynchronize();
+        scsr_free(out);
+    }
     return e;
 }
 
 void scsr_free(ScsrStore *S) {
-    cudaFree(S->col);
-    cudaFree(S->base);
-    cudaFree(S->start);
-    cudaFree(S->qc);
+    dev_free(S->col);   // (callers synchronise first: graph_free)
+    dev_free(S->base);
+    dev_free(S->start);
+    dev_free(S->qc);
     *S = ScsrStore{};
 }
 
