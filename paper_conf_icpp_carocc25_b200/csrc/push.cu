@@ -43,7 +43,8 @@ static void launch_push(const PushLaunch &L, const F &f, cudaStream_t s) {
     if constexpr (F::kSeg) {
         if (p.seg && p.seg_mode && L.g.hub_idx) {
             note_launch();
-            k_push_seg<<<148, SEG_THREADS, SEG_SMEM, s>>>(p, f);
+            // one CTA per SM (192 KB slice); at least one per destination segment (SG_SEG_OWNER)
+            k_push_seg<<<L.g.nseg > 148 ? L.g.nseg : 148, SEG_THREADS, SEG_SMEM, s>>>(p, f);
         }
     }
 }

@@ -23,6 +23,9 @@ namespace sg {
 
 constexpr int SEG_THREADS = 1024;
 constexpr size_t SEG_SMEM = (size_t)SEG_WORDS * sizeof(uint64_t);
+#ifndef SG_SEG_OWNER
+#define SG_SEG_OWNER 1   // 1: a CTA owns one segment (one slice load / flush); 0: every CTA walks all
+#endif
 #ifndef SG_SEG_UNROLL
 #define SG_SEG_UNROLL 4
 #endif
@@ -37,15 +40,32 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
     const unsigned long long cnt = p.st->seg_count;
     const uint32_t nitems = (uint32_t)(cnt < p.seg_cap ? cnt : p.seg_cap);
     if (nitems == 0) return;
+    const int nseg = p.g.nseg, S1 = nseg + 1;
+#if SG_SEG_OWNER
+    // each CTA owns one destination segment and a share of the items: the CTAs are dealt to the
+    // segments in contiguous groups (gridDim.x >= nseg), so every slice is loaded and flushed by
+    // its group only (gridDim.x slices in total instead of gridDim.x * nseg)
+    const int G = (int)gridDim.x;
+    const int b_own = (int)((int64_t)blockIdx.x * nseg / G);
+    const int c_lo = (int)(((int64_t)b_own * G + nseg - 1) / nseg);       // first CTA of the group
+    const int c_hi = (int)(((int64_t)(b_own + 1) * G + nseg - 1) / nseg);  // one past its last
+    const uint32_t i0 = (uint32_t)((uint64_t)nitems * (blockIdx.x - c_lo) / (c_hi - c_lo));
+    const uint32_t i1 = (uint32_t)((uint64_t)nitems * (blockIdx.x - c_lo + 1) / (c_hi - c_lo));
+    if (i0 == i1) return;
+#else
     const uint32_t i0 = (uint32_t)((uint64_t)nitems * blockIdx.x / gridDim.x);
     const uint32_t i1 = (uint32_t)((uint64_t)nitems * (blockIdx.x + 1) / gridDim.x);
     if (i0 == i1) return;
-    const int nseg = p.g.nseg, S1 = nseg + 1;
+#endif
     const int warp = threadIdx.x >> 5, lane = lane_id();
     constexpr int NW = SEG_THREADS / 32;
     uint32_t *level = f.level_pp ? *f.level_pp : f.level;
     const uint32_t next = f.next_ptr ? *f.next_ptr : f.next;
+#if SG_SEG_OWNER
+    for (int b = b_own; b == b_own; b++) {
+#else
     for (int b = 0; b < nseg; b++) {
+#endif
         const int64_t w0 = (int64_t)b * SEG_WORDS;
         const int nw = (int)min((int64_t)SEG_WORDS, p.g.nw1 - w0);
         for (int i = threadIdx.x; i < nw; i += SEG_THREADS) s_vis[i] = f.visited[w0 + i];
