@@ -83,6 +83,7 @@ struct Workspace {
     DevStats *h_st = nullptr;      // pinned host mirror
     uint64_t *visited = nullptr;   // nw1 words
     uint64_t *vis_old = nullptr;   // nw1 words: visited before the current BFS superstep (k_bfs_diff)
+    uint32_t *dist_old = nullptr;  // n: distances before the current SSSP superstep (k_sssp_diff)
     uint32_t *all_offsets = nullptr;   // one-layer ablation: identity word list
     sg_frontier *far = nullptr;        // delta-stepping SSSP: far pile
     HeavyItem *heavy = nullptr;
@@ -206,6 +207,7 @@ static void free_ws(Workspace *ws) {
     cudaFreeHost(ws->h_st);
     cudaFree(ws->visited);
     cudaFree(ws->vis_old);
+    cudaFree(ws->dist_old);
     cudaFree(ws->heavy);
     cudaFree(ws->seg);
     cudaFree(ws->all_offsets);
@@ -1158,14 +1160,29 @@ SG_API int run_sssp(const sg_graph *gc, int32_t src, uint32_t *dist, const sg_op
         }
         arcs = -1;   // not accumulated in this mode
     }
+    // diff mode (default): the push only relaxes (fire-and-forget red.min), k_sssp_diff derives
+    // the output frontier (dist < dist_old) and its word list in one pass over dist
+    static const bool sssp_diff = env_or("SG_SSSP_DIFF", 1) != 0;
+    if (o.sssp_delta <= 0 && sssp_diff) {
+        if (!ws->dist_old) CK(cudaMalloc(&ws->dist_old, sizeof(uint32_t) * (size_t)(G.n ? G.n : 1)));
+        CK(cudaMemcpyAsync(ws->dist_old, dist, sizeof(uint32_t) * (size_t)G.n, cudaMemcpyDeviceToDevice, s));
+    }
     for (; o.sssp_delta <= 0;) {
         const int64_t count = (int64_t)ws->h_st[in_idx].count;
         if (count == 0) break;
         if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
         const PushLaunch L = push_launch(g, in, t, count);
-        launch_push_sssp(L, SsspArgs{dist, out->bits, out->summ}, s);
-        TRY(clear_frontier(in, s));
-        TRY(compact(g, out, false, s));
+        if (sssp_diff) {
+            CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
+            SsspArgs sa{dist, nullptr, nullptr};
+            sa.diff = 1;
+            launch_push_sssp(L, sa, s);
+            launch_sssp_diff(G, dist, ws->dist_old, out->bits, out->summ, out->offsets, out->st, s);
+        } else {
+            launch_push_sssp(L, SsspArgs{dist, out->bits, out->summ}, s);
+            TRY(clear_frontier(in, s));
+            TRY(compact(g, out, false, s));
+        }
         TRY(read_stats(ws, s));
         arcs += (int64_t)ws->h_st[in_idx].arcs;
         std::swap(in, out);

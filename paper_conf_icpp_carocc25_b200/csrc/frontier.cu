@@ -446,6 +446,69 @@ void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &
     note_launch();
     k_bfs_diff<<<(int)blocks, DIFF_THREADS, 0, s>>>(g, visited, o);
 }
+// Output of a diff-mode SSSP superstep (FnSssp::diff): the vertices whose distance decreased.
+// A CTA of 256 threads takes 64 layer-1 words (4,096 vertices, one layer-2 word): a thread
+// compares 4 x 4 distances (16-B loads of dist and dist_old), the half-warp ORs the word's
+// bits, every output word is written, and the CTA emits its layer-2 word and word list.
+__global__ void __launch_bounds__(256) k_sssp_diff(GraphView g, const uint32_t *__restrict__ dist,
+                                                   uint32_t *__restrict__ dist_old, BfsOut o) {
+    __shared__ uint64_t s_S[1];
+    __shared__ uint32_t s_base;
+    const int lane = lane_id();
+    const uint32_t half = (lane < 16) ? 0x0000ffffu : 0xffff0000u;
+    const bool vec = (((uintptr_t)dist | (uintptr_t)dist_old) & 15) == 0;
+    for (int64_t sw = blockIdx.x; sw < g.nw2; sw += gridDim.x) {
+        if (threadIdx.x == 0) s_S[0] = 0ull;
+        __syncthreads();
+#pragma unroll 1
+        for (int r = 0; r < 4; r++) {
+            const int64_t qd = sw * 1024 + r * 256 + threadIdx.x;   // quad of 4 vertices
+            const int64_t w = qd >> 4;
+            const int sh = (int)(qd & 15) * 4;
+            uint32_t m = 0;
+            if (w < g.nw1) {
+                const int64_t v0 = w * 64 + sh;
+                if (vec && v0 + 4 <= g.n) {
+                    const uint4 a = *reinterpret_cast<const uint4 *>(dist + v0);
+                    const uint4 b = *reinterpret_cast<const uint4 *>(dist_old + v0);
+                    m = (a.x < b.x ? 1u : 0u) | (a.y < b.y ? 2u : 0u) | (a.z < b.z ? 4u : 0u) | (a.w < b.w ? 8u : 0u);
+                    if (m) *reinterpret_cast<uint4 *>(dist_old + v0) = a;
+                } else {
+                    for (int k = 0; k < 4; k++) {
+                        if (v0 + k >= g.n) break;
+                        const uint32_t a = dist[v0 + k];
+                        if (a < dist_old[v0 + k]) {
+                            m |= 1u << k;
+                            dist_old[v0 + k] = a;
+                        }
+                    }
+                }
+            }
+            const uint64_t mine = (uint64_t)m << sh;
+            const uint64_t nb = (uint64_t)__reduce_or_sync(half, (uint32_t)mine) |
+                                ((uint64_t)__reduce_or_sync(half, (uint32_t)(mine >> 32)) << 32);
+            if ((lane & 15) == 0 && w < g.nw1) {
+                o.out_bits[w] = nb;
+                if (nb) atomicOr(reinterpret_cast<unsigned long long *>(s_S), 1ull << (w & 63));
+            }
+        }
+        __syncthreads();
+        bfs_emit_words(o, g.nw2, sw, s_S, 1, &s_base);
+    }
+}
+void launch_sssp_diff(const GraphView &g, const uint32_t *dist, uint32_t *dist_old, uint64_t *out_bits,
+                      uint64_t *out_summ, uint32_t *out_offsets, DevStats *st, cudaStream_t s) {
+    BfsOut o{};
+    o.out_bits = out_bits;
+    o.out_summ = out_summ;
+    o.out_offsets = out_offsets;
+    o.st = st;
+    int64_t blocks = g.nw2;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_sssp_diff<<<(int)blocks, 256, 0, s>>>(g, dist, dist_old, o);
+}
 void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(p, n); }
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s) {
     note_launch();

@@ -46,6 +46,9 @@ __device__ __forceinline__ void insert_batch(const OutSink &out, const int32_t (
 // diff mode (run_bfs): the arc only ORs v's visited bit, a fire-and-forget RED with no result
 // to wait for; k_bfs_diff then derives the output frontier, level[] and the frontier
 // statistics from visited & ~visited_before in one pass over the bitmap (same result set).
+#ifndef SG_SSSP_NOPROBE
+#define SG_SSSP_NOPROBE 0   // SSSP diff mode: 1 skips the dist[v] probe before the RED
+#endif
 #ifndef SG_WORDS_NOPROBE
 #define SG_WORDS_NOPROBE 1
 #endif
@@ -110,15 +113,27 @@ struct FnSssp {
     using Probe = uint32_t;
     uint32_t *dist;
     OutSink out;
+    uint32_t diff;   // 1: fire-and-forget REDs (min), k_sssp_diff builds the output frontier
     __device__ __forceinline__ Ctx ctx(int32_t u) const { return *(volatile uint32_t *)(dist + u); }
-    __device__ __forceinline__ bool skip_probe_words() const { return false; }
-    __device__ __forceinline__ bool skip_probe() const { return false; }
+    __device__ __forceinline__ bool skip_probe_words() const { return SG_SSSP_NOPROBE && diff; }
+    __device__ __forceinline__ bool skip_probe() const { return SG_SSSP_NOPROBE && diff; }
     __device__ __forceinline__ Probe probe(int32_t v) const { return dist[v]; }
     template <int K>
     __device__ __forceinline__ void act_batch(const Ctx (&du)[K], const int32_t (&v)[K], const uint32_t (&w)[K],
                                               const Probe (&pr)[K], const bool (&ok)[K]) const {
         uint32_t nd[K], old[K];
         bool cand[K], imp[K], done[K];
+        if (diff) {   // relax only: dist[v] = min(dist[v], du + w) with no result to wait for
+#pragma unroll
+            for (int k = 0; k < K; k++) {
+                nd[k] = du[k] + w[k];
+                // (a skipped probe reads as INF: every arc of a reached source relaxes)
+                const uint32_t p = skip_probe() ? INF32 : pr[k];
+                if (ok[k] && du[k] != INF32 && nd[k] < p)
+                    asm volatile("red.global.min.u32 [%0], %1;" ::"l"(dist + v[k]), "r"(nd[k]) : "memory");
+            }
+            return;
+        }
 #pragma unroll
         for (int k = 0; k < K; k++) {
             nd[k] = du[k] + w[k];

@@ -67,7 +67,7 @@ struct BfsArgs {
     uint32_t *const *level_pp = nullptr;
     uint32_t diff = 0;                     // 1: visited marks only; k_bfs_diff builds the output
 };
-struct SsspArgs { uint32_t *dist; uint64_t *out_bits, *out_summ; };
+struct SsspArgs { uint32_t *dist; uint64_t *out_bits, *out_summ; uint32_t diff = 0; };
 struct CcArgs { int32_t *label; uint64_t *out_bits, *out_summ; };
 struct BcArgs { const uint64_t *visited; double *sigma; uint32_t *level; uint32_t next; uint64_t *out_bits, *out_summ; };
 void launch_push_bfs(const PushLaunch &L, const BfsArgs &a, cudaStream_t s);
@@ -103,6 +103,12 @@ void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visi
                      cudaStream_t s);
 // frontier.cu — output of a diff-mode BFS superstep (push word path / sweep): see BfsOut
 void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s);
+
+// frontier.cu — output of a diff-mode SSSP superstep: the vertices whose distance decreased
+// (dist < dist_old) -> the whole output 2LB + word list + st->count (st zeroed before);
+// dist_old = dist
+void launch_sssp_diff(const GraphView &g, const uint32_t *dist, uint32_t *dist_old, uint64_t *out_bits,
+                      uint64_t *out_summ, uint32_t *out_offsets, DevStats *st, cudaStream_t s);
 
 // filter.cu — filter::inplace / external, compute::execute (Table 2)
 void launch_filter(const GraphView &g, const uint64_t *in_bits, uint64_t *out_bits, uint64_t *out_summ, int pred,

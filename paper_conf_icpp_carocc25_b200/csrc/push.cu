@@ -67,6 +67,7 @@ void launch_push_sssp(const PushLaunch &L, const SsspArgs &a, cudaStream_t s) {
     FnSssp f;
     f.dist = a.dist;
     f.out = OutSink{a.out_bits, a.out_summ};
+    f.diff = a.diff;
     launch_push(L, f, s);
 }
 void launch_push_cc(const PushLaunch &L, const CcArgs &a, cudaStream_t s) {
