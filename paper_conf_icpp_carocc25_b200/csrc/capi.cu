@@ -124,6 +124,8 @@ struct sg_graph {
     int32_t *hub_idx = nullptr;     // hub index of u (deg >= SEG_MIN) or -1
     int32_t *hub_vertex = nullptr;
     uint32_t *hub_off = nullptr;    // [nhubs][nseg+1] segment offsets within the hub's row
+    uint32_t *cbo = nullptr;        // [n][cbo_nb-1] first arc of each row into each CC label block (run_cc)
+    int cbo_nb = 0;
     int64_t nhubs = 0;
     ScsrStore scsr;                 // destination-segmented copy of the arcs (BFS heavy push), built lazily
     int scsr_state = 0;             // 0 not built, 1 built, -1 unavailable (segment block >= 2^32 arcs, unsorted rows)
@@ -369,6 +371,7 @@ SG_API int graph_free(sg_graph *g) {
     dev_free(g->hub_idx);
     dev_free(g->hub_vertex);
     dev_free(g->hub_off);
+    dev_free(g->cbo);
     if (g->scsr_state == 1) scsr_free(&g->scsr);
     delete g;
     return SG_OK;
@@ -1220,6 +1223,22 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
     L2Pin pin(label, sizeof(int32_t) * (size_t)G.n, s);   // labels are probed once per arc: keep them in L2
+    // label blocks for the pull step: labels of one block (<= SG_CC_LBLOCK_KB) stay in L2
+    const long long lblock = (long long)env_or("SG_CC_LBLOCK_KB", 32768) << 10;
+    int cc_nb = (int)(((long long)G.n * 4 + lblock - 1) / (lblock > 0 ? lblock : 1));
+    if (cc_nb < 1 || lblock <= 0) cc_nb = 1;
+    if (cc_nb > 64) cc_nb = 64;
+    if (cc_nb > 1 && o.direction != SG_DIR_PUSH && (g->cbo_nb != cc_nb)) {
+        if (g->cbo) {
+            CK(cudaStreamSynchronize(s));
+            dev_free(g->cbo);
+            g->cbo = nullptr;
+        }
+        const int64_t S = (G.n + cc_nb - 1) / cc_nb;
+        CK(dev_alloc(&g->cbo, sizeof(uint32_t) * (size_t)G.n * (size_t)(cc_nb - 1), s));
+        launch_cc_block_offsets(G.rp, G.col, G.n, cc_nb, S, g->cbo, s);
+        g->cbo_nb = cc_nb;
+    }
     CK(cudaEventRecord(ws->ev0, s));
     launch_iota_i32(label, G.n, s);
     sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
@@ -1237,7 +1256,11 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
         // its neighbours' labels without atomics; a sparse one pushes from the changed vertices
         const bool pull = o.direction == SG_DIR_PULL ||
                           (o.direction == SG_DIR_AUTO && (double)ws->h_st[in_idx].mf * 4.0 > (double)G.nnz);
-        if (pull) {
+        if (pull && cc_nb > 1) {   // label-blocked pull: one pass per L2-sized label block
+            for (int b = 0; b < cc_nb; b++) launch_pull_cc_block(G, label, out->bits, in->st, g->cbo, cc_nb, b, s);
+            launch_rebuild_summary(out->bits, out->summ, G.nw1, G.nw2, s);
+            pull_steps++;
+        } else if (pull) {
             launch_pull_cc(G, label, out->bits, out->summ, in->st, s);
             pull_steps++;
         } else {

@@ -117,6 +117,12 @@ void launch_compute(const GraphView &g, const uint64_t *bits, int op, void *arra
 void launch_min_over_bits(const GraphView &g, const uint64_t *bits, const uint32_t *a, unsigned int *out,
                           cudaStream_t s);
 
+// pull_cc.cu — label-blocked pull for CC: per-row offsets of each label block (rows sorted),
+// and one pass per block (out_bits written by pass 0, ORed by the others; summary by the caller)
+void launch_cc_block_offsets(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, uint32_t *cbo,
+                             cudaStream_t s);
+void launch_pull_cc_block(const GraphView &g, int32_t *label, uint64_t *out_bits, DevStats *st, const uint32_t *cbo,
+                          int nb, int b, cudaStream_t s);
 // pull_cc.cu — pull label-propagation step (dense CC supersteps)
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,
                     cudaStream_t s);

@@ -14,6 +14,32 @@
 namespace sg {
 
 constexpr int CCP_THREADS = 256;
+#ifndef SG_CC_HINTS
+#define SG_CC_HINTS 0   // bit 0: col_idx loads evict-first, bit 1: label loads evict-last (measured: no gain / slower)
+#endif
+// L2 residency hints: the 2.1 GB col_idx stream must not evict the 84 MB label array, whose
+// random probes otherwise cost a DRAM sector each (ncu: 23 GB of DRAM traffic per pull step for
+// 4.2 GB of algorithmic bytes)
+__device__ __forceinline__ int32_t ld_col(const int32_t *p, uint64_t pol) {
+#if SG_CC_HINTS & 1
+    int32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+#else
+    (void)pol;
+    return __ldg(p);
+#endif
+}
+__device__ __forceinline__ int32_t ld_label(const int32_t *p, uint64_t pol) {
+#if SG_CC_HINTS & 2
+    int32_t v;
+    asm volatile("ld.global.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+#else
+    (void)pol;
+    return *p;
+#endif
+}
 
 __global__ void __launch_bounds__(CCP_THREADS)
 k_pull_cc(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__ out_bits, uint64_t *__restrict__ out_summ,
@@ -23,6 +49,13 @@ k_pull_cc(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__ out_b
     const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     unsigned long long arcs = 0;
+    uint64_t pol_last = 0, pol_first = 0;
+#if SG_CC_HINTS & 1
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_first));
+#endif
+#if SG_CC_HINTS & 2
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
+#endif
     for (int64_t w = gw; w < g.nw1; w += nwarps) {
         const int64_t rem = g.n - w * 64;
         const uint64_t valid = rem >= 64 ? ~0ull : ((1ull << rem) - 1ull);
@@ -38,12 +71,12 @@ k_pull_cc(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__ out_b
             int32_t c[8];
 #pragma unroll
             for (int k = 0; k < 4; k++) {
-                c[k] = (ia + k < ea) ? __ldg(g.col + ia + k) : -1;
-                c[4 + k] = (ib + k < eb) ? __ldg(g.col + ib + k) : -1;
+                c[k] = (ia + k < ea) ? ld_col(g.col + ia + k, pol_first) : -1;
+                c[4 + k] = (ib + k < eb) ? ld_col(g.col + ib + k, pol_first) : -1;
             }
             int32_t l[8];
 #pragma unroll
-            for (int k = 0; k < 8; k++) l[k] = c[k] >= 0 ? label[c[k]] : 0x7fffffff;
+            for (int k = 0; k < 8; k++) l[k] = c[k] >= 0 ? ld_label(label + c[k], pol_last) : 0x7fffffff;
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 ma = min(ma, l[k]);
@@ -67,6 +100,112 @@ k_pull_cc(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__ out_b
         for (int i = 0; i < CCP_THREADS / 32; i++) t += s_arcs[i];
         if (t) atomicAdd(&st->arcs, t);
     }
+}
+
+// ---- label-blocked pull (graphs whose label array does not stay in L2) --------------------
+// A pull step probes one random label per arc; at config 3 (84 MB of labels, 2.1 GB of col_idx
+// streamed past them) nearly every probe misses L2 and moves a 32-B DRAM sector (ncu: 23 GB per
+// step for 4.2 GB of algorithmic bytes).  Rows are sorted, so the arcs of row v into label block
+// b (vertices [b*S, (b+1)*S)) are contiguous: the step runs one pass per block, each reading only
+// that block's labels (S*4 B <= ~32 MB, L2-resident) and the row parts that point into it.
+// cbo[v*(nb-1) + b-1] = first arc of row v into block b (b = 1..nb-1), built once per graph.
+__global__ void k_cc_block_offsets(const int64_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t n,
+                                   int nb, int64_t S, uint32_t *__restrict__ cbo) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += stride) {
+        const int64_t s0 = rp[v], e0 = rp[v + 1];
+        for (int b = 1; b < nb; b++) {   // lower_bound(col[s0..e0), b*S)
+            int64_t lo = s0, hi = e0;
+            const int64_t key = (int64_t)b * S;
+            while (lo < hi) {
+                const int64_t mid = (lo + hi) >> 1;
+                if ((int64_t)col[mid] < key) lo = mid + 1;
+                else hi = mid;
+            }
+            cbo[v * (nb - 1) + (b - 1)] = (uint32_t)(lo - s0);
+        }
+    }
+}
+void launch_cc_block_offsets(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, uint32_t *cbo,
+                             cudaStream_t s) {
+    int64_t blocks = (n + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    note_launch();
+    k_cc_block_offsets<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(rp, col, n, nb, S, cbo);
+}
+
+// one pass of the blocked pull: vertices take the min over their arcs into block b; the warp
+// owning word w writes (b == 0) or ORs (b > 0) the word's changed bits into the output frontier
+__global__ void __launch_bounds__(CCP_THREADS)
+k_pull_cc_block(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__ out_bits, DevStats *st,
+                const uint32_t *__restrict__ cbo, int nb, int b) {
+    __shared__ unsigned long long s_arcs[CCP_THREADS / 32];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    unsigned long long arcs = 0;
+    uint64_t pol_last = 0, pol_first = 0;
+#if SG_CC_HINTS & 1
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_first));
+#endif
+#if SG_CC_HINTS & 2
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
+#endif
+    auto part = [&](int64_t v, int64_t &s0, int64_t &e0) {
+        const int64_t r0 = __ldg(g.rp + v), r1 = __ldg(g.rp + v + 1);
+        s0 = b == 0 ? r0 : r0 + __ldg(cbo + v * (nb - 1) + (b - 1));
+        e0 = b == nb - 1 ? r1 : r0 + __ldg(cbo + v * (nb - 1) + b);
+    };
+    for (int64_t w = gw; w < g.nw1; w += nwarps) {
+        const int64_t va = w * 64 + lane, vb = va + 32;
+        const bool act_a = va < g.n, act_b = vb < g.n;
+        int64_t sa = 0, ea = 0, sb = 0, eb = 0;
+        if (act_a) part(va, sa, ea);
+        if (act_b) part(vb, sb, eb);
+        const int32_t own_a = act_a ? label[va] : 0x7fffffff, own_b = act_b ? label[vb] : 0x7fffffff;
+        int32_t ma = own_a, mb = own_b;
+        arcs += (unsigned long long)((ea - sa) + (eb - sb));
+        for (int64_t ia = sa, ib = sb; ia < ea || ib < eb; ia += 4, ib += 4) {
+            int32_t c[8];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                c[k] = (ia + k < ea) ? ld_col(g.col + ia + k, pol_first) : -1;
+                c[4 + k] = (ib + k < eb) ? ld_col(g.col + ib + k, pol_first) : -1;
+            }
+            int32_t l[8];
+#pragma unroll
+            for (int k = 0; k < 8; k++) l[k] = c[k] >= 0 ? ld_label(label + c[k], pol_last) : 0x7fffffff;
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                ma = min(ma, l[k]);
+                mb = min(mb, l[4 + k]);
+            }
+        }
+        const bool ca = ma < own_a, cb = mb < own_b;
+        if (ca) label[va] = ma;
+        if (cb) label[vb] = mb;
+        const uint64_t nbits = (uint64_t)__ballot_sync(0xffffffffu, ca) | ((uint64_t)__ballot_sync(0xffffffffu, cb) << 32);
+        if (lane == 0) {
+            if (b == 0) out_bits[w] = nbits;
+            else if (nbits) out_bits[w] |= nbits;
+        }
+    }
+    arcs = warp_sum(arcs);
+    if (lane == 0) s_arcs[threadIdx.x >> 5] = arcs;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t = 0;
+        for (int i = 0; i < CCP_THREADS / 32; i++) t += s_arcs[i];
+        if (t) atomicAdd(&st->arcs, t);
+    }
+}
+void launch_pull_cc_block(const GraphView &g, int32_t *label, uint64_t *out_bits, DevStats *st, const uint32_t *cbo,
+                          int nb, int b, cudaStream_t s) {
+    int64_t blocks = (g.nw1 * 32 + CCP_THREADS - 1) / CCP_THREADS;
+    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_pull_cc_block<<<(int)blocks, CCP_THREADS, 0, s>>>(g, label, out_bits, st, cbo, nb, b);
 }
 
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,

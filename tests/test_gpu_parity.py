@@ -429,6 +429,21 @@ def test_cc_directions_agree(sg, make):
         assert np.array_equal(lab.cpu().numpy(), ref), d
 
 
+@pytest.mark.parametrize("kb", [4, 64, 1000])
+@pytest.mark.parametrize("make", [lambda: gen.gnm(200_000, 1_000_000), lambda: gen.rmat(15, 16, permute=True),
+                                  lambda: gen.lattice(300, 300, 0.55), lambda: gen.gnm(100_003, 40_000, seed=7)])
+def test_cc_label_blocked_pull(sg, monkeypatch, make, kb):
+    """Label-blocked pull (one pass per label block of kb KB; block boundaries inside rows, ragged
+    last block, up to 64 blocks) reaches the union-find labels, for pull-only and auto."""
+    monkeypatch.setenv("SG_CC_LBLOCK_KB", str(kb))
+    g = make()
+    G = load(sg, g)
+    ref = oracle.cc(g)
+    for d in (sg.SG_DIR_PULL, sg.SG_DIR_AUTO):
+        lab, _ = sg.run_cc(G, direction=d)
+        assert np.array_equal(lab.cpu().numpy(), ref), (d, kb)
+
+
 # -------------------------------------------------------------------------------- BC
 @pytest.mark.parametrize("make,k", [(lambda: gen.random_simple(60, 0.08, 3), 60), (lambda: gen.path(300), 10),
                                     (lambda: gen.hypercube(10), 5), (lambda: gen.rmat(12, 16, permute=True), 8),
