@@ -84,6 +84,10 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             const int64_t rem = g.n - v0;
             const uint32_t valid = !ok ? 0u : rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
             const uint32_t unv = (uint32_t)(~vis >> sh) & valid;
+            if (__all_sync(0xffffffffu, unv == 0u)) {   // the warp's two words are fully visited:
+                if ((lane & 15) == 0 && ok) o.out_bits[w] = 0ull;   // no new vertices, no work
+                continue;
+            }
             uint32_t found = 0, codes = 0;
             if (unv) {
                 const int4 c4 = __ldg(reinterpret_cast<const int4 *>(g.fnbr + v0));
