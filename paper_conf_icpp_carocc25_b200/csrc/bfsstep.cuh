@@ -22,10 +22,6 @@ __device__ __forceinline__ unsigned long long quad_mf(const uint32_t *lut, uint3
     return m;
 }
 
-__device__ __forceinline__ bool st_mf_ge(const volatile DevStats *st, unsigned long long thr) {
-    return thr != 0ull && st->mf >= thr;
-}
-
 __device__ __forceinline__ void bfs_set_cond(unsigned long long h, unsigned v) {
     if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, v);
 }
@@ -67,7 +63,6 @@ __device__ __forceinline__ void bfs_decide(BfsCtrl *c, const DevStats *st, DevSt
     const bool push = go && !c->pull;
     const bool sweep = push && (c->sweep_mode == 2 || (c->sweep_mode == 1 && vst->mf >= c->sweep_thr));
     if (sweep) c->sweep_steps++;
-    if (push && c->sweep_mode == 0 && st_mf_ge(vst, c->sweep_thr)) c->sweep_wanted++;
     bfs_set_cond(h_push, push && !sweep);
     bfs_set_cond(h_sweep, sweep);
     bfs_set_cond(h_pull, go && c->pull);

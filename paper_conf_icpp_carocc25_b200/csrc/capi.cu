@@ -129,7 +129,6 @@ struct sg_graph {
     int64_t nhubs = 0;
     ScsrStore scsr;                 // destination-segmented copy of the arcs (BFS heavy push), built lazily
     int scsr_state = 0;             // 0 not built, 1 built, -1 unavailable (segment block >= 2^32 arcs, unsorted rows)
-    bool sweep_wanted = false;      // a BFS had a push superstep with m_f >= the sweep threshold (auto: build it)
     uint32_t max_w = 0;
     int device = 0;
     Workspace *ws = nullptr;
@@ -783,10 +782,11 @@ static int add_cond(cudaGraph_t graph, const std::vector<cudaGraphNode_t> &deps,
     return SG_OK;
 }
 
-// The segment-major arc copy (scsr.cu), built at the first run_bfs that uses it: at once when
-// forced (scsr = 2) or for a push-only BFS, else (auto) only after a BFS of this graph had a push
-// superstep dense enough for the sweep (g->sweep_wanted; a direction-optimising BFS normally pulls
-// those, and the copy costs ~13 ms and 4 GB at config 4).  A graph whose segment blocks would
+// The segment-major arc copy (scsr.cu), built at the first run_bfs that uses it: when forced
+// (scsr = 2) or for a push-only BFS.  A direction-optimising BFS pulls its dense supersteps, so
+// in auto mode it never builds the copy (~13 ms and 4 GB at config 4, which would otherwise land
+// inside whichever BFS first met a dense push superstep); it uses the copy if a push-only BFS of
+// the same graph built it.  A graph whose segment blocks would
 // exceed 2^32 arcs, whose rows are not sorted, or for which the memory is not available keeps
 // the word path (the copy is a performance structure only).
 static bool sweep_size_ok(const sg_graph *g) {
@@ -796,7 +796,7 @@ static bool scsr_ready(sg_graph *g, const Tiers &t, bool want_now, cudaStream_t 
     if (t.scsr == 0) return false;
     if (g->scsr_state == 0) {
         if (t.scsr == 1 && !sweep_size_ok(g)) return false;
-        if (t.scsr == 1 && !want_now && !g->sweep_wanted) return false;   // deferred
+        if (t.scsr == 1 && !want_now) return false;   // auto: only a push-only BFS builds it
         const int32_t sw = (int32_t)env_or("SG_SCSR_WORDS", 0);   // test knob: narrower segments (0: 16,384 words)
         const cudaError_t e = scsr_build(g->rp, g->col, g->v.n, g->v.nnz, sw, &g->scsr, s);
         if (e != cudaSuccess) {
@@ -932,7 +932,6 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
     CK(cudaGetLastError());
     if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
-    if (c.sweep_wanted && t.scsr == 1 && sweep_size_ok(g)) g->sweep_wanted = true;
     {
         // kernels the graph executed: the prologue kernel + the
         // taken IF bodies (push = word + CTA tier [+ hub segment tier] + output, sweep = arc
@@ -1012,9 +1011,6 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         nf_prev = nf;
         const int64_t reached_before = reached;
         const bool sweep = !pull && scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz));
-        if (!pull && !scsr_on && t.scsr == 1 && !o.one_layer && sweep_size_ok(g) &&
-            (unsigned long long)mf >= sweep_threshold(G.nnz))
-            g->sweep_wanted = true;
         CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
         const BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, level, d + 1, nullptr, nullptr, out->st};
         const int pr = prof_begin(ws, pull ? SG_K_PULL : (sweep ? SG_K_SWEEP : SG_K_PUSH), s);

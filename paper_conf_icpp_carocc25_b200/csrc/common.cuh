@@ -65,7 +65,6 @@ struct BfsCtrl {
     uint32_t sweep_mode;     // push supersteps through the sweep: 0 never, 1 when m_f >= sweep_thr, 2 always
     unsigned long long sweep_thr;
     unsigned long long sweep_steps;
-    unsigned long long sweep_wanted;   // push supersteps with m_f >= sweep_thr while the sweep was not available
 };
 
 // Device-resident control of one source-batched BC batch (bcb.cu).
