@@ -160,3 +160,66 @@ def dist_bfs(dg: DistGraph, src: int, exchange: SliceExchange, max_iters: int | 
         fin, fout = fout, fin
     exchange.gather_values(level)
     return level
+
+
+def _exchange_frontier(sg, exchange, fout):
+    import torch
+    bits, summ = sg.frontier_view(fout)
+    exchange.gather_bitmap(bits.view(torch.int64), summ.view(torch.int64))
+
+
+def dist_sssp(dg: DistGraph, src: int, exchange: SliceExchange, max_iters: int | None = None):
+    """Bellman-Ford by frontier over the 1-D partition: each rank relaxes the arcs of its
+    push block (only owned distances change, no cross-GPU atomics), then the owned slices of the
+    output frontier and of dist are all-gathered.  Returns the full dist array (int32 storage of
+    uint32 distances, UINT32_MAX = unreached), replicated on every rank."""
+    import torch
+    sg = dg.sg
+    n = dg.n
+    dev = torch.device("cuda", torch.cuda.current_device())
+    dist = torch.full((n,), -1, dtype=torch.int32, device=dev)
+    dist[src] = 0
+    fin, fout = sg.frontier_init(dg.G), sg.frontier_init(dg.G)
+    sg.frontier_insert(fin, np.array([src], dtype=np.int32))
+    cap = max_iters or n + 1
+    it = 0
+    while True:
+        sg.advance(dg.G, fin, fout, sg.SG_FN_SSSP, dict(dist=dist))
+        _exchange_frontier(sg, exchange, fout)
+        exchange.gather_values(dist)
+        if sg.frontier_count(fout) == 0:
+            break
+        it += 1
+        if it > cap:
+            raise RuntimeError("iteration cap reached")
+        sg.frontier_clear(fin)
+        fin, fout = fout, fin
+    return dist
+
+
+def dist_cc(dg: DistGraph, exchange: SliceExchange, max_iters: int | None = None):
+    """Label propagation over the 1-D partition: all vertices start active
+    (advance::vertices, P:137); each rank lowers the labels of its owned vertices from the arcs
+    of its push block, then the owned label slices and output-frontier slices are all-gathered.
+    Returns the full label array (component minimum ids), replicated on every rank."""
+    import torch
+    sg = dg.sg
+    n = dg.n
+    dev = torch.device("cuda", torch.cuda.current_device())
+    label = torch.arange(n, dtype=torch.int32, device=dev)
+    fin, fout = sg.frontier_init(dg.G), sg.frontier_init(dg.G)
+    sg.frontier_fill_all(fin)
+    cap = max_iters or n + 1
+    it = 0
+    while True:
+        sg.advance(dg.G, fin, fout, sg.SG_FN_CC, dict(label=label))
+        _exchange_frontier(sg, exchange, fout)
+        exchange.gather_values(label)
+        if sg.frontier_count(fout) == 0:
+            break
+        it += 1
+        if it > cap:
+            raise RuntimeError("iteration cap reached")
+        sg.frontier_clear(fin)
+        fin, fout = fout, fin
+    return label
