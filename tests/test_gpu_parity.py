@@ -203,6 +203,32 @@ def test_bfs_degree_tier_boundaries(sg, deg):
             assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, s)), (deg, s, d)
 
 
+@pytest.mark.parametrize("n", [4096 * 3 + 77, 4096 * 5, 64 * 70 + 1])
+@pytest.mark.parametrize("direction", ["pull", "auto"])
+def test_bfs_pull_fully_visited_words(sg, n, direction):
+    """Pull steps over frontiers where whole layer-2 words (4,096 vertices) and single layer-1
+    words are already visited (the pull's skip paths), next to words with a few unvisited
+    vertices left: a dense random core over the first half (visited after 2-3 levels), a long
+    path through the rest, small components scattered into otherwise visited words, isolated
+    vertices and a ragged tail."""
+    rng = np.random.default_rng(n)
+    h = n // 2
+    cu = rng.integers(0, h, 24 * h)
+    cv = rng.integers(0, h, 24 * h)
+    pu = np.arange(h - 1, n - 200)   # path from the core's last vertex through the second half
+    iso = rng.choice(np.arange(1, h), 40, replace=False)   # pairs / triangles inside the core words
+    tu = np.concatenate([iso[0:40:2]])
+    tv = np.concatenate([iso[1:40:2]])
+    keep = ~(np.isin(cu, iso) | np.isin(cv, iso))
+    g = gen.from_edges(n, np.concatenate([cu[keep], pu, tu]), np.concatenate([cv[keep], pu + 1, tv]))
+    G = load(sg, g)
+    for s in (0, 5, h + 1000, n - 201):
+        lv, st = sg.run_bfs(G, s, direction=_dir(sg, direction))
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, s)), (n, s)
+        lv2, _ = sg.run_bfs(G, s, direction=_dir(sg, direction), host_loop=True)
+        assert np.array_equal(sg.as_u32(lv2), oracle.bfs(g, s)), (n, s)
+
+
 def test_bfs_isolated_source_and_empty_graph(sg):
     g = gen.rmat(10, 16)
     iso = int(np.nonzero(g.degrees() == 0)[0][0])
