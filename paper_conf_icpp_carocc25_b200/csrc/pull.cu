@@ -21,6 +21,12 @@
 // itself, and the last CTA decides the next superstep (bfsstep.cuh).  The step is a streaming
 // pass over the visited bitmap and fnbr with enough independent threads in flight to cover the
 // latency of the dependent bit test.  Output identical to a push step from the same state.
+// Late pull steps leave a few unvisited vertices per word, and the quad rounds become
+// issue-bound (every warp runs the whole round for its one or two unvisited lanes).  So each
+// CTA first reads the 64 visited words of its layer-2 word: none unvisited -> 64 zero output
+// words; at most SG_PULL_WORD_MAX unvisited in every word -> word mode (a thread per layer-1
+// word walks its unvisited vertices, SG_PULL_WORD_BATCH candidate tests in flight); else the
+// quad rounds, where a warp whose two words are fully visited skips without loading them.
 #include "common.cuh"
 #include "kernels.h"
 #include "bfsstep.cuh"
@@ -43,14 +49,56 @@ constexpr int PULL_ARCS = SG_PULL_ARCS;
 #ifndef SG_PULL_PF
 #define SG_PULL_PF 0   // 1: load the next round's visited word one round ahead
 #endif
+#ifndef SG_PULL_WSKIP
+#define SG_PULL_WSKIP 1   // 1: per layer-2 word mask of fully visited layer-1 words (skip without loads)
+#endif
+#ifndef SG_PULL_WORD_MAX
+#define SG_PULL_WORD_MAX 16   // word mode when no layer-1 word of the layer-2 word has more unvisited
+#endif                       // vertices than this (0: off; needs SG_PULL_WSKIP)
+#ifndef SG_PULL_WORD_BATCH
+#define SG_PULL_WORD_BATCH 4   // word mode: vertices whose candidate tests are in flight together
+#endif
+#if SG_PULL_PF && SG_PULL_WSKIP
+#error "SG_PULL_PF assumes every round loads its visited word: build it with SG_PULL_WSKIP=0"
+#endif
 #ifndef SG_PULL_MINB
 #define SG_PULL_MINB 8
 #endif
+// list scan of v: true iff some u in N(v) is in the input frontier (stops at the first hit);
+// PULL_ARCS arcs in flight per step, `arcs` counts the arcs tested
+__device__ __forceinline__ bool pull_scan(const GraphView &g, const uint32_t *__restrict__ in32, int64_t v,
+                                          unsigned long long &arcs) {
+    int64_t rr = __ldg(g.rp + v);
+    const int64_t e = __ldg(g.rp + v + 1);
+    bool hit = false;
+    while (rr < e && !hit) {
+        int32_t u[PULL_ARCS];
+        uint32_t y[PULL_ARCS];
+#pragma unroll
+        for (int j = 0; j < PULL_ARCS; j++) u[j] = rr + j < e ? __ldg(g.col + rr + j) : -1;
+#pragma unroll
+        for (int j = 0; j < PULL_ARCS; j++) y[j] = u[j] >= 0 ? __ldg(in32 + (u[j] >> 5)) : 0u;
+#pragma unroll
+        for (int j = 0; j < PULL_ARCS; j++) {
+            if (!hit && u[j] >= 0) {
+                arcs++;
+                hit = (y[j] >> (u[j] & 31)) & 1u;
+            }
+        }
+        rr += PULL_ARCS;
+    }
+    return hit;
+}
+
 __global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
            BfsOut o) {
     __shared__ uint64_t s_wm[PULL_THREADS / 32], s_S[1];
     __shared__ uint32_t s_base, s_lut[256];
+#if SG_PULL_WSKIP
+    __shared__ uint32_t s_full[2][2], s_mx[2][2];   // double-buffered by iteration parity (no barrier at reuse)
+    int par = 0;
+#endif
     deg8_lut_init(s_lut);
     __syncthreads();
     uint32_t *const lvl = o.level_pp ? *o.level_pp : o.level;
@@ -68,11 +116,105 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
 #endif
     for (int64_t sw = blockIdx.x; sw < g.nw2; sw += gridDim.x) {
         uint64_t wm = 0;   // the warp's changed words within the layer-2 word
+#if SG_PULL_WSKIP
+        // bit i of `full`: layer-1 word sw*64+i has no unvisited vertex (or lies past the end).
+        // A layer-2 word with no unvisited vertex writes its 64 zero output words and is done;
+        // otherwise a warp whose two words are full skips its round without loading them.
+        uint64_t my_vis = ~0ull, my_unv = 0ull;   // threads < 64: layer-1 word sw*64+threadIdx.x
+        if (threadIdx.x < 64) {
+            const int64_t w = sw * 64 + threadIdx.x;
+            if (w < g.nw1) {
+                const int64_t rem = g.n - w * 64;
+                const uint64_t valid = rem >= 64 ? ~0ull : ((1ull << rem) - 1ull);
+                my_vis = visited[w];
+                my_unv = ~my_vis & valid;
+            }
+            const uint32_t b = __ballot_sync(0xffffffffu, my_unv == 0ull);
+            const uint32_t mx = __reduce_max_sync(0xffffffffu, (uint32_t)__popcll(my_unv));
+            if (lane == 0) {
+                s_full[par][wid] = b;
+                s_mx[par][wid] = mx;
+            }
+        }
+        __syncthreads();
+        const uint64_t full = (uint64_t)s_full[par][0] | ((uint64_t)s_full[par][1] << 32);
+        const uint32_t mxw = max(s_mx[par][0], s_mx[par][1]);
+        par ^= 1;
+        if (full == ~0ull) {
+            if (threadIdx.x < 64 && sw * 64 + threadIdx.x < g.nw1) o.out_bits[sw * 64 + threadIdx.x] = 0ull;
+            if (threadIdx.x == 0) o.out_summ[sw] = 0ull;
+            continue;
+        }
+#if SG_PULL_WORD_MAX > 0
+        if (mxw <= SG_PULL_WORD_MAX) {
+            // word mode (late pull steps: a few unvisited vertices per word): thread t < 64 owns
+            // layer-1 word sw*64+t and walks its unvisited vertices one by one (candidate test,
+            // then the list scan), so the CTA spends 2 warps instead of 32 quad rounds on it.
+            // Same tests in the same order per vertex as the quad mode: identical output / stats.
+            if (threadIdx.x < 64) {
+                const int64_t w = sw * 64 + threadIdx.x;
+                uint64_t nbw = 0;
+                // SG_PULL_WORD_BATCH vertices per pass: their candidates and frontier bits are loaded together
+                for (uint64_t m = my_unv; m;) {
+                    int b[SG_PULL_WORD_BATCH];
+                    int32_t c[SG_PULL_WORD_BATCH];
+                    uint32_t x[SG_PULL_WORD_BATCH];
+#pragma unroll
+                    for (int k = 0; k < SG_PULL_WORD_BATCH; k++) {
+                        b[k] = m ? __ffsll((long long)m) - 1 : -1;
+                        m &= m - 1;
+                    }
+#pragma unroll
+                    for (int k = 0; k < SG_PULL_WORD_BATCH; k++) c[k] = b[k] >= 0 ? __ldg(g.fnbr + w * 64 + b[k]) : -1;
+#pragma unroll
+                    for (int k = 0; k < SG_PULL_WORD_BATCH; k++) x[k] = c[k] >= 0 ? __ldg(in32 + (c[k] >> 5)) : 0u;
+#pragma unroll
+                    for (int k = 0; k < SG_PULL_WORD_BATCH; k++) {
+                        if (b[k] < 0) continue;
+                        bool hit = false;
+                        if (c[k] >= 0) {
+                            arcs++;
+                            hit = (x[k] >> (c[k] & 31)) & 1u;
+                        }
+                        if (!hit) hit = pull_scan(g, in32, w * 64 + b[k], arcs);
+                        if (hit) nbw |= 1ull << b[k];
+                    }
+                }
+                if (w < g.nw1) {
+                    o.out_bits[w] = nbw;
+                    if (nbw) {
+                        visited[w] = my_vis | nbw;
+                        o.vis_old[w] = my_vis | nbw;
+                        nf += __popcll(nbw);
+                        for (uint64_t m = nbw; m; m &= m - 1) {
+                            const int64_t v = w * 64 + (__ffsll((long long)m) - 1);
+                            lvl[v] = nx;
+                            mf += s_lut[__ldg(g.deg8 + v)];
+                        }
+                    }
+                }
+                const uint32_t b = __ballot_sync(0xffffffffu, nbw != 0ull);
+                if (lane == 0) s_wm[wid] = b;
+            }
+            __syncthreads();
+            if (threadIdx.x == 0) s_S[0] = s_wm[0] | (s_wm[1] << 32);
+            __syncthreads();
+            bfs_emit_words(o, g.nw2, sw, s_S, 1, &s_base);
+            continue;
+        }
+#endif
+#endif
 #pragma unroll 1
         for (int r = 0; r < PULL_ROUNDS; r++) {
             const int64_t qd = sw * 1024 + r * PULL_THREADS + threadIdx.x;
             const bool ok = qd < nq;
             const int64_t w = qd >> 4;
+#if SG_PULL_WSKIP
+            if (((full >> (r * (PULL_THREADS / 16) + wid * 2)) & 3ull) == 3ull) {
+                if ((lane & 15) == 0 && ok) o.out_bits[w] = 0ull;
+                continue;
+            }
+#endif
             const int sh = (int)(qd & 15) * 4;
 #if SG_PULL_PF
             const uint64_t vis = vis_next;
@@ -106,25 +248,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                 // 2. list scans of the vertices whose candidate missed
                 for (uint32_t miss = unv & ~found; miss; miss &= miss - 1) {
                     const int k = __ffs(miss) - 1;
-                    int64_t rr = __ldg(g.rp + v0 + k);
-                    const int64_t e = __ldg(g.rp + v0 + k + 1);
-                    bool hit = false;
-                    while (rr < e && !hit) {
-                        int32_t u[PULL_ARCS];
-                        uint32_t y[PULL_ARCS];
-#pragma unroll
-                        for (int j = 0; j < PULL_ARCS; j++) u[j] = rr + j < e ? __ldg(g.col + rr + j) : -1;
-#pragma unroll
-                        for (int j = 0; j < PULL_ARCS; j++) y[j] = u[j] >= 0 ? __ldg(in32 + (u[j] >> 5)) : 0u;
-#pragma unroll
-                        for (int j = 0; j < PULL_ARCS; j++) {
-                            if (!hit && u[j] >= 0) {
-                                arcs++;
-                                hit = (y[j] >> (u[j] & 31)) & 1u;
-                            }
-                        }
-                        rr += PULL_ARCS;
-                    }
+                    const bool hit = pull_scan(g, in32, v0 + k, arcs);
                     if (hit) found |= 1u << k;
                 }
             }
