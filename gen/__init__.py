@@ -56,7 +56,7 @@ def _load():
         lib.sgg_weights.restype = None
         lib.sgg_weights.argtypes = [i64, vp, vp, u64, ctypes.c_uint32, vp]
         lib.sgg_sources.restype = i64
-        lib.sgg_sources.argtypes = [i64, vp, u64, u64, i64, vp]
+        lib.sgg_sources.argtypes = [i64, vp, u64, u64, i64, vp, vp]
         lib.sgg_rnd.restype = u64
         lib.sgg_rnd.argtypes = [u64, u64, u64]
         _lib = lib
@@ -200,11 +200,29 @@ def with_weights(g: CSR, seed: int = 1, wmax: int = 64) -> CSR:
     return g
 
 
-def sources(g: CSR, k: int, seed: int = 1, stream: int = 5) -> np.ndarray:
-    """First k distinct rnd(seed, stream, i) mod n with degree > 0 (reading C15)."""
+def sources(g: CSR, k: int, seed: int = 1, stream: int = 5, eligible: np.ndarray | None = None) -> np.ndarray:
+    """First k distinct rnd(seed, stream, i) mod n with degree > 0 (reading C15), restricted to
+    eligible[v] != 0 when a mask is given."""
     out = np.empty(k, dtype=np.int32)
-    got = _load().sgg_sources(g.n, g.row_ptr.ctypes.data, seed, stream, k, out.ctypes.data)
+    if eligible is not None:
+        eligible = np.ascontiguousarray(eligible, dtype=np.uint8)
+        assert eligible.shape == (g.n,)
+    got = _load().sgg_sources(g.n, g.row_ptr.ctypes.data, seed, stream, k, out.ctypes.data,
+                              eligible.ctypes.data if eligible is not None else None)
     return out[:got].copy()
+
+
+def largest_component_mask(g: CSR) -> np.ndarray:
+    """uint8[n]: 1 on the vertices of the largest connected component (ties: the one holding the
+    smallest vertex id).  Source selection only (reading C15); computed with scipy's
+    connected_components, a library routine shared by neither the oracle nor the CUDA path."""
+    import scipy.sparse as sp
+    from scipy.sparse.csgraph import connected_components
+    A = sp.csr_matrix((np.ones(g.nnz, dtype=np.int8), g.col_idx, g.row_ptr), shape=(g.n, g.n))
+    _, lab = connected_components(A, directed=False)
+    cnt = np.bincount(lab)
+    big = int(np.argmax(cnt))          # argmax returns the first maximum: smallest label = smallest id
+    return (lab == big).astype(np.uint8)
 
 
 def rnd(seed: int, stream: int, i: int) -> int:
@@ -219,7 +237,8 @@ CONFIGS = {
     3: dict(workload="cc", graph=("gnm", dict(n=21_000_000, m=265_000_000))),
     4: dict(workload="bfs_do", graph=("rmat", dict(scale=24, edge_factor=32, permute=True)), n_sources=64,
             source_stream=5),
-    5: dict(workload="bc", graph=("lattice", dict(R=4000, C=6000, p=0.6)), n_sources=64, source_stream=6),
+    5: dict(workload="bc", graph=("lattice", dict(R=4000, C=6000, p=0.6)), n_sources=64, source_stream=6,
+            largest_component=True),   # reading C15
 }
 
 
@@ -237,4 +256,5 @@ def config_sources(cfg: int, g: CSR, seed: int = 1) -> np.ndarray:
     c = CONFIGS[cfg]
     if "sources" in c:
         return np.asarray(c["sources"], dtype=np.int32)
-    return sources(g, c["n_sources"], seed=seed, stream=c["source_stream"])
+    eligible = largest_component_mask(g) if c.get("largest_component") else None
+    return sources(g, c["n_sources"], seed=seed, stream=c["source_stream"], eligible=eligible)

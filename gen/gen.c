@@ -298,15 +298,17 @@ SGG_EXPORT void sgg_weights(int64_t n, const int64_t *row_ptr, const int32_t *co
         }
 }
 
-/* First k distinct vertices rnd(stream, i) mod n with degree > 0 (reading C15).
- * Returns the number found (< k only if fewer non-isolated vertices exist). */
+/* First k distinct vertices rnd(stream, i) mod n with degree > 0 (reading C15) and, when
+ * `eligible` is non-NULL, eligible[v] != 0 (config 5: the largest component, computed by the
+ * caller with a library routine).  Returns the number found (< k only if fewer exist). */
 SGG_EXPORT int64_t sgg_sources(int64_t n, const int64_t *row_ptr, uint64_t seed, uint64_t stream,
-                               int64_t k, int32_t *out) {
+                               int64_t k, int32_t *out, const uint8_t *eligible) {
     uint64_t b = stream_base(seed, stream);
     int64_t found = 0;
     for (uint64_t i = 0; found < k && i < (uint64_t)(64 * n + 1024); i++) {
         int64_t v = (int64_t)(rnd_b(b, i) % (uint64_t)n);
         if (row_ptr[v + 1] == row_ptr[v]) continue;
+        if (eligible && !eligible[v]) continue;
         int dup = 0;
         for (int64_t j = 0; j < found; j++) if (out[j] == v) { dup = 1; break; }
         if (!dup) out[found++] = (int32_t)v;

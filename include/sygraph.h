@@ -38,7 +38,21 @@ enum sg_status {
     SG_ERR_STATE = -6         /* missing functor state / iteration cap hit / handle misuse */
 };
 enum { SG_MEM_HOST = 0, SG_MEM_DEVICE = 1 };          /* where input arrays live */
-enum { SG_F_VALIDATE = 2 };                           /* graph_load_csr flags */
+/* graph_load_csr flags:
+ *   SG_F_BORROW    with SG_MEM_DEVICE: keep the caller's row_ptr / col_idx / weights pointers (no
+ *                  copy; e.g. torch tensors).  The caller keeps them alive and unmodified until
+ *                  graph_free.  col_idx must be 16-B aligned and its allocation must extend >= 64
+ *                  readable bytes past nnz*4 (16-B vector loads of a row's tail; torch's caching
+ *                  allocator rounds blocks to 512 B); weights likewise past nnz.  Checked, else
+ *                  SG_ERR_INVALID.
+ *   SG_F_VALIDATE  O(nnz log deg) device check of the CSR contract (§3.1; readings C8, C9):
+ *                  row_ptr[0] = 0, row_ptr[n] = nnz, row_ptr monotone, 0 <= col < n, every row
+ *                  strictly ascending (sorted, no multi-edges), no self-loops, and symmetric
+ *                  (every arc (u,v) has its reverse (v,u)).  Any violation -> SG_ERR_INVALID.
+ *   Without SG_F_VALIDATE row order is still checked (O(nnz), every load): a graph whose rows are
+ *   not sorted loads, but its hub-segmented push tier, segment-major sweep and label-blocked CC
+ *   pull (which binary-search sorted rows) are disabled for it; results stay exact.             */
+enum { SG_F_BORROW = 1, SG_F_VALIDATE = 2 };
 enum { SG_FN_BFS = 0, SG_FN_SSSP = 1, SG_FN_CC = 2, SG_FN_BC_SIGMA = 3 };   /* advance functors */
 enum { SG_DIR_AUTO = 0, SG_DIR_PUSH = 1, SG_DIR_PULL = 2 };                 /* BFS direction */
 
@@ -61,9 +75,13 @@ typedef struct {              /* CC label propagation: dst enters iff   
 typedef struct {              /* BC forward sigma (P:161 Brandes): dst not in `visited` (frozen for */
     uint32_t *level;          /* the step) gets sigma[dst] += sigma[src] and enters the output; its */
     uint64_t *visited;        /* inserting thread writes level[dst] = depth + 1.  The caller ORs   */
-    double *sigma;            /* the output into `visited` afterwards (frontier_or).               */
-    uint32_t depth;
-} sg_bc_state;
+    double *sigma;            /* the output into `visited` afterwards (frontier_or_into).           */
+    int32_t *exp2_per_level;  /* device int32[>= depth + 2]: sigma of level L is stored as          */
+    uint32_t depth;           /* sigma_true * 2^-E[L] (reading C20 / DESIGN R5).  After the step the */
+} sg_bc_state;                /* new level (the output frontier, which must start empty) is scaled */
+                              /* so its maximum lies in [1, 2) and E[depth+1] = E[depth] + k is     */
+                              /* written (E[0] = 0 is the caller's).  Without it sigma overflows    */
+                              /* fp64 on high-diameter graphs: NULL -> SG_ERR_STATE.                */
 
 typedef struct {
     void *stream;             /* cudaStream_t; NULL = legacy default stream */

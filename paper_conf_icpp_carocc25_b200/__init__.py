@@ -18,7 +18,7 @@ LIB_PATH = os.environ.get("SYGRAPH_LIB") or os.path.join(_PKG, "lib", "libsygrap
 
 SG_OK, SG_ERR_INVALID, SG_ERR_OOM, SG_ERR_CUDA, SG_ERR_NCCL, SG_ERR_UNSUPPORTED, SG_ERR_STATE = 0, -1, -2, -3, -4, -5, -6
 SG_MEM_HOST, SG_MEM_DEVICE = 0, 1
-SG_F_VALIDATE = 2
+SG_F_BORROW, SG_F_VALIDATE = 1, 2
 SG_FN_BFS, SG_FN_SSSP, SG_FN_CC, SG_FN_BC_SIGMA = 0, 1, 2, 3
 SG_DIR_AUTO, SG_DIR_PUSH, SG_DIR_PULL = 0, 1, 2
 INF32 = 0xFFFFFFFF
@@ -61,7 +61,7 @@ class SgCcState(ctypes.Structure):
 
 class SgBcState(ctypes.Structure):
     _fields_ = [("level", ctypes.c_void_p), ("visited", ctypes.c_void_p), ("sigma", ctypes.c_void_p),
-                ("depth", ctypes.c_uint32)]
+                ("exp2_per_level", ctypes.c_void_p), ("depth", ctypes.c_uint32)]
 
 
 class SgKprof(ctypes.Structure):
@@ -185,8 +185,10 @@ class Graph:
             pass
 
 
-def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None) -> Graph:
-    """row_ptr int64[n+1], col_idx int32[nnz], weights uint8[nnz] (numpy/host tensors or CUDA tensors)."""
+def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None, borrow=False) -> Graph:
+    """row_ptr int64[n+1], col_idx int32[nnz], weights uint8[nnz] (numpy/host tensors or CUDA tensors).
+    borrow (CUDA tensors only): keep the tensors' memory instead of copying (SG_F_BORROW); the
+    returned Graph holds references to them."""
     rp, m1 = _ptr_mem(row_ptr)
     ci, m2 = _ptr_mem(col_idx)
     w, m3 = _ptr_mem(weights)
@@ -196,9 +198,21 @@ def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None) 
     if len(mems) != 1:
         raise ValueError("row_ptr, col_idx and weights must all be host or all be device arrays")
     h = ctypes.c_void_p()
-    _check(load().graph_load_csr(n, nnz, rp, ci if nnz else None, w, m1, SG_F_VALIDATE if validate else 0,
-                                 _stream_ptr(stream), ctypes.byref(h)))
-    return Graph(h.value, n, nnz, weights is not None)
+    flags = (SG_F_VALIDATE if validate else 0) | (SG_F_BORROW if borrow else 0)
+    _check(load().graph_load_csr(n, nnz, rp, ci if nnz else None, w, m1, flags, _stream_ptr(stream), ctypes.byref(h)))
+    G = Graph(h.value, n, nnz, weights is not None)
+    if borrow:
+        G._borrowed = (row_ptr, col_idx, weights)
+    return G
+
+
+def graph_info(g: Graph):
+    """(n, nnz, row_ptr, col_idx, weights) — the device pointers the graph reads (ints; 0 = none)."""
+    n, nnz = ctypes.c_int64(), ctypes.c_int64()
+    rp, ci, w = ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p()
+    _check(load().graph_info(g.handle, ctypes.byref(n), ctypes.byref(nnz), ctypes.byref(rp), ctypes.byref(ci),
+                             ctypes.byref(w)))
+    return n.value, nnz.value, rp.value or 0, ci.value or 0, w.value or 0
 
 
 def graph_free(g: Graph):
@@ -294,7 +308,8 @@ def frontier_or_into(f: Frontier, dst, stream=None):
 # ---------------------------------------------------------------------------- advance
 def advance(g: Graph, fin: Frontier, fout: Frontier | None, functor: int, state: dict, stream=None):
     """One push advance superstep (stream ordered).  ``state`` holds the functor's tensors:
-    BFS {level, visited, depth}; SSSP {dist}; CC {label}; BC {level, visited, sigma, depth}."""
+    BFS {level, visited, depth}; SSSP {dist}; CC {label}; BC {level, visited, sigma, exp2_per_level,
+    depth}."""
     if functor == SG_FN_BFS:
         st = SgBfsState(state["level"].data_ptr(), state["visited"].data_ptr(), int(state["depth"]))
     elif functor == SG_FN_SSSP:
@@ -302,8 +317,9 @@ def advance(g: Graph, fin: Frontier, fout: Frontier | None, functor: int, state:
     elif functor == SG_FN_CC:
         st = SgCcState(state["label"].data_ptr())
     elif functor == SG_FN_BC_SIGMA:
+        e = state.get("exp2_per_level")
         st = SgBcState(state["level"].data_ptr(), state["visited"].data_ptr(), state["sigma"].data_ptr(),
-                       int(state["depth"]))
+                       e.data_ptr() if e is not None else None, int(state["depth"]))
     else:
         raise ValueError(functor)
     _check(load().advance(g.handle, fin.handle, fout.handle if fout is not None else None, functor,

@@ -37,7 +37,8 @@ __global__ void k_bc_level_max(const double *__restrict__ sigma, const uint64_t 
     if (lane_id() == 0 && mx) atomicMax(max_bits, mx);
 }
 
-// Scale level (level_idx) by 2^-k, record E[level_idx] and append the level to the BFS stack.
+// Scale level (level_idx) by 2^-k, record E[level_idx] and append the level to the BFS stack
+// (stack == NULL: no stack, the user-driven advance(SG_FN_BC_SIGMA) path).
 __global__ void k_bc_scale_stack(double *__restrict__ sigma, const uint64_t *__restrict__ bits,
                                  const uint32_t *__restrict__ offsets, const DevStats *st,
                                  const unsigned long long *max_bits, int32_t *exp_of_level, uint32_t level_idx,
@@ -51,7 +52,7 @@ __global__ void k_bc_scale_stack(double *__restrict__ sigma, const uint64_t *__r
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += stride) {
         const uint32_t w = offsets[i];
         uint64_t x = bits[w];
-        unsigned long long pos = atomicAdd(stack_top, (unsigned long long)__popcll(x));
+        unsigned long long pos = stack ? atomicAdd(stack_top, (unsigned long long)__popcll(x)) : 0ull;
         while (x) {
             const int b = __ffsll((long long)x) - 1;
             x &= x - 1;
@@ -59,7 +60,7 @@ __global__ void k_bc_scale_stack(double *__restrict__ sigma, const uint64_t *__r
             const double sv = ldexp(sigma[v], -k);
             if (sv < 2.2250738585072014e-308) atomicAdd(underflow, 1ull);   // subnormal: precision lost
             sigma[v] = sv;
-            stack[pos++] = (int32_t)v;
+            if (stack) stack[pos++] = (int32_t)v;
         }
     }
 }
@@ -94,14 +95,14 @@ static int grid_for(int64_t items, int threads, int max_blocks) {
 void launch_bc_level_max(const double *sigma, const uint64_t *bits, const uint32_t *offsets, const DevStats *st,
                          int64_t max_words, unsigned long long *max_bits, cudaStream_t s) {
     note_launch();
-    k_bc_level_max<<<grid_for(max_words, 256, 148 * 4), 256, 0, s>>>(sigma, bits, offsets, st, max_bits);
+    k_bc_level_max<<<grid_for(max_words, 256, num_sms() * 4), 256, 0, s>>>(sigma, bits, offsets, st, max_bits);
 }
 void launch_bc_level_scale_and_stack(double *sigma, const uint64_t *bits, const uint32_t *offsets,
                                      const DevStats *st, int64_t max_words, const unsigned long long *max_bits,
                                      int32_t *exp_of_level, uint32_t level_idx, int32_t *stack,
                                      unsigned long long *stack_top, unsigned long long *underflow, cudaStream_t s) {
     note_launch();
-    k_bc_scale_stack<<<grid_for(max_words, 256, 148 * 4), 256, 0, s>>>(sigma, bits, offsets, st, max_bits,
+    k_bc_scale_stack<<<grid_for(max_words, 256, num_sms() * 4), 256, 0, s>>>(sigma, bits, offsets, st, max_bits,
                                                                         exp_of_level, level_idx, stack, stack_top,
                                                                         underflow);
 }
@@ -110,7 +111,7 @@ void launch_bc_backward_level(const GraphView &g, const int32_t *stack, int64_t 
                               double *bc, int32_t src, cudaStream_t s) {
     if (hi <= lo) return;
     note_launch();
-    k_bc_backward<<<grid_for(hi - lo, 256, 148 * 8), 256, 0, s>>>(g, stack, lo, hi, level, sigma, delta,
+    k_bc_backward<<<grid_for(hi - lo, 256, num_sms() * 8), 256, 0, s>>>(g, stack, lo, hi, level, sigma, delta,
                                                                    exp_of_level, d, bc, src);
 }
 

@@ -470,7 +470,7 @@ cudaError_t bcb_run_batch(const BcbLaunch &L, cudaStream_t s) {
     e = cudaLaunchCooperativeKernel((const void *)k_bcb_backward, coop_blocks, BCB_THREADS, args, 0, s);
     if (e != cudaSuccess) return e;
     note_launch();
-    k_bcb_reset<<<148 * 8, 256, 0, s>>>(b);
+    k_bcb_reset<<<num_sms() * 8, 256, 0, s>>>(b);
     return cudaGetLastError();
 }
 

@@ -12,6 +12,8 @@
 #include <string>
 #include <vector>
 
+#include <cuda.h>   // CUdeviceptr / CUresult types for the driver entry point below (no -lcuda)
+
 #include "sygraph.h"
 #include "kernels.h"
 
@@ -131,8 +133,11 @@ struct sg_graph {
     int scsr_state = 0;             // 0 not built, 1 built, -1 unavailable (segment block >= 2^32 arcs, unsorted rows)
     uint32_t max_w = 0;
     int device = 0;
+    bool borrowed = false;          // SG_F_BORROW: rp / col / w are the caller's
+    bool sorted = true;             // every row strictly ascending (checked at load)
     Workspace *ws = nullptr;
 };
+static std::atomic<int> g_live_graphs{0};
 
 static const int32_t kDefaultHeavy = 2048;
 static const int32_t kDefaultSmall = 32;
@@ -277,6 +282,27 @@ SG_API void sg_opts_default(sg_opts *o) {
     o->beta = 24.0;
 }
 
+// bytes readable from p to the end of its allocation (driver allocation range), -1 if unknown
+// (cuMemGetAddressRange through cudaGetDriverEntryPoint: the library does not link libcuda)
+static long long bytes_to_alloc_end(const void *p) {
+    typedef CUresult (*range_fn)(CUdeviceptr *, size_t *, CUdeviceptr);
+    static range_fn fn = nullptr;
+    if (!fn) {
+        void *f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess || !f) {
+            cudaGetLastError();
+            return -1;
+        }
+        fn = (range_fn)f;
+    }
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (fn(&base, &size, (CUdeviceptr)p) != CUDA_SUCCESS) return -1;
+    return (long long)((unsigned long long)base + size - (unsigned long long)p);
+}
+
 SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const int32_t *col_idx,
                           const uint8_t *weights, int mem, int flags, void *stream, sg_graph **out) {
     t_err.clear();
@@ -286,6 +312,9 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     if (nnz < 0 || nnz > (1ll << 40)) return fail(SG_ERR_INVALID, "nnz=%lld outside [0, 2^40]", (long long)nnz);
     if (!row_ptr || (nnz > 0 && !col_idx)) return fail(SG_ERR_INVALID, "row_ptr/col_idx NULL");
     if (mem != SG_MEM_HOST && mem != SG_MEM_DEVICE) return fail(SG_ERR_INVALID, "mem must be SG_MEM_HOST or SG_MEM_DEVICE");
+    if (flags & ~(SG_F_BORROW | SG_F_VALIDATE)) return fail(SG_ERR_INVALID, "unknown flags 0x%x", flags);
+    const bool borrow = (flags & SG_F_BORROW) != 0;
+    if (borrow && mem != SG_MEM_DEVICE) return fail(SG_ERR_INVALID, "SG_F_BORROW needs SG_MEM_DEVICE arrays");
     if (mem == SG_MEM_DEVICE) {
         TRY(check_device(row_ptr));
         TRY(check_device(col_idx));
@@ -293,28 +322,60 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     } else {
         if (row_ptr[0] != 0 || row_ptr[n] != nnz) return fail(SG_ERR_INVALID, "row_ptr[0] != 0 or row_ptr[n] != nnz");
     }
+    if (borrow) {   // the kernels read 16-B vectors of col_idx (and u32 quads of weights) up to 12 B past nnz
+        if (((uintptr_t)col_idx & 15) || ((uintptr_t)row_ptr & 7))
+            return fail(SG_ERR_INVALID, "SG_F_BORROW: col_idx must be 16-B aligned, row_ptr 8-B aligned");
+        const long long cb = nnz ? bytes_to_alloc_end(col_idx) : 1 << 20;
+        const long long wb = weights ? bytes_to_alloc_end(weights) : 1 << 20;
+        if (cb < 0 || wb < 0) return fail(SG_ERR_INVALID, "SG_F_BORROW: cannot query the allocation of col_idx/weights");
+        if (cb < nnz * 4 + 64 || wb < nnz + 64)
+            return fail(SG_ERR_INVALID, "SG_F_BORROW: col_idx / weights allocations need >= 64 readable bytes past nnz");
+    }
     cudaStream_t s = (cudaStream_t)stream;
     sg_graph *g = new sg_graph();
+    g_live_graphs++;
     CK(cudaGetDevice(&g->device));
     g->v.n = n;
     g->v.nnz = nnz;
     g->v.nw1 = (n + 63) / 64;
     g->v.nw2 = (g->v.nw1 + 63) / 64;
-    const cudaMemcpyKind kind = mem == SG_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
-    // col_idx/weights get 64 B of zero padding: 16-B bulk copies may read up to 12 B past nnz
-    CK(dev_alloc(&g->rp, sizeof(int64_t) * (size_t)(n + 1), s));
-    CK(dev_alloc(&g->col, sizeof(int32_t) * (size_t)nnz + 64, s));
-    CK(cudaMemsetAsync((char *)g->col + sizeof(int32_t) * (size_t)nnz, 0, 64, s));
-    CK(cudaMemcpyAsync(g->rp, row_ptr, sizeof(int64_t) * (size_t)(n + 1), kind, s));
-    if (nnz) CK(cudaMemcpyAsync(g->col, col_idx, sizeof(int32_t) * (size_t)nnz, kind, s));
-    if (weights) {
-        CK(dev_alloc(&g->w, (size_t)nnz + 64, s));
-        CK(cudaMemsetAsync(g->w + nnz, 0, 64, s));
-        if (nnz) CK(cudaMemcpyAsync(g->w, weights, (size_t)nnz, kind, s));
+    g->borrowed = borrow;
+    if (borrow) {
+        g->rp = const_cast<int64_t *>(row_ptr);
+        g->col = const_cast<int32_t *>(col_idx);
+        g->w = const_cast<uint8_t *>(weights);
+    } else {
+        const cudaMemcpyKind kind = mem == SG_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+        // col_idx/weights get 64 B of zero padding: 16-B bulk copies may read up to 12 B past nnz
+        CK(dev_alloc(&g->rp, sizeof(int64_t) * (size_t)(n + 1), s));
+        CK(dev_alloc(&g->col, sizeof(int32_t) * (size_t)nnz + 64, s));
+        CK(cudaMemsetAsync((char *)g->col + sizeof(int32_t) * (size_t)nnz, 0, 64, s));
+        CK(cudaMemcpyAsync(g->rp, row_ptr, sizeof(int64_t) * (size_t)(n + 1), kind, s));
+        if (nnz) CK(cudaMemcpyAsync(g->col, col_idx, sizeof(int32_t) * (size_t)nnz, kind, s));
+        if (weights) {
+            CK(dev_alloc(&g->w, (size_t)nnz + 64, s));
+            CK(cudaMemsetAsync(g->w + nnz, 0, 64, s));
+            if (nnz) CK(cudaMemcpyAsync(g->w, weights, (size_t)nnz, kind, s));
+        }
     }
     g->v.rp = g->rp;
     g->v.col = g->col;
     g->v.w = g->w;
+    unsigned long long *dscr = nullptr;
+    CK(cudaMalloc(&dscr, 48));
+    CK(cudaMemsetAsync(dscr, 0, 48, s));
+    // structure first (the derived arrays below index with row_ptr / col_idx)
+    launch_validate_csr(g->v, dscr, s);
+    unsigned long long hv[6] = {0, 0, 0, 0, 0, 0};
+    CK(cudaMemcpyAsync(hv, dscr, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (hv[0]) {
+        cudaFree(dscr);
+        graph_free(g);
+        return fail(SG_ERR_INVALID, "CSR validation failed (%llu malformed row_ptr / col_idx entries)", hv[0]);
+    }
+    launch_row_check(g->v, dscr + 3, s);                           // [3] unsorted pairs, [4] self-loops
+    if (flags & SG_F_VALIDATE) launch_symmetry(g->v, dscr + 5, s); // [5] arcs without reverse
     CK(dev_alloc(&g->deg8, (size_t)g->v.nw1 * 64, s));
     launch_deg8(g->rp, n, g->v.nw1 * 64, g->deg8, s);
     g->v.deg8 = g->deg8;
@@ -323,29 +384,27 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     CK(dev_alloc(&g->fnbr, sizeof(int32_t) * (size_t)(g->v.nw1 ? g->v.nw1 * 64 : 1), s));   // padded: 16-B quad loads
     launch_first_nbr(g->rp, g->col, g->deg8, n, g->v.nw1 * 64, g->fnbr, s);
     g->v.fnbr = g->fnbr;
-    unsigned long long *dscr = nullptr;
-    CK(cudaMalloc(&dscr, 24));
-    CK(cudaMemsetAsync(dscr, 0, 24, s));
-    if (flags & SG_F_VALIDATE) launch_validate_csr(g->v, dscr, s);
     if (g->w) launch_max_weight(g->w, nnz, reinterpret_cast<unsigned int *>(dscr + 1), s);
     // hubs of the destination-segmented BFS tier (deg >= SEG_MIN): index map + vertex list
     const int64_t max_hubs = nnz / SEG_MIN + 1;
     CK(dev_alloc(&g->hub_idx, sizeof(int32_t) * (size_t)n, s));
     CK(dev_alloc(&g->hub_vertex, sizeof(int32_t) * (size_t)max_hubs, s));
     launch_hub_mark(g->rp, n, g->hub_idx, g->hub_vertex, reinterpret_cast<unsigned int *>(dscr + 2), s);
-    unsigned long long h[3] = {0, 0, 0};
-    CK(cudaMemcpyAsync(h, dscr, 24, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(hv, dscr, 48, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     CK(cudaGetLastError());
     cudaFree(dscr);
-    g->max_w = (uint32_t)(h[1] & 0xffffffffu);
-    if (h[0]) {
+    g->max_w = (uint32_t)(hv[1] & 0xffffffffu);
+    if ((flags & SG_F_VALIDATE) && (hv[3] || hv[4] || hv[5])) {
         graph_free(g);
-        return fail(SG_ERR_INVALID, "CSR validation failed (%llu bad entries)", h[0]);
+        return fail(SG_ERR_INVALID, "CSR validation failed: %llu unsorted/duplicate pairs, %llu self-loops, %llu arcs "
+                    "without their reverse (rows must be strictly ascending, simple, symmetric)", hv[3], hv[4], hv[5]);
     }
-    g->nhubs = (int64_t)(h[2] & 0xffffffffu);
+    g->sorted = hv[3] == 0;
+    if (!g->sorted) g->scsr_state = -1;   // the segment-major copy needs sorted rows
+    g->nhubs = (int64_t)(hv[2] & 0xffffffffu);
     g->v.nseg = (int32_t)((n + SEG_V - 1) / SEG_V);
-    if (g->nhubs > 0) {
+    if (g->nhubs > 0 && g->sorted) {   // hub segment offsets binary-search sorted rows
         CK(dev_alloc(&g->hub_off, sizeof(uint32_t) * (size_t)g->nhubs * (size_t)(g->v.nseg + 1), s));
         launch_hub_off(g->rp, g->col, g->hub_vertex, g->nhubs, g->v.nseg, g->hub_off, s);
         CK(cudaStreamSynchronize(s));
@@ -361,9 +420,11 @@ SG_API int graph_free(sg_graph *g) {
     if (!g) return SG_OK;
     cudaDeviceSynchronize();   // no pending work may use the buffers (cudaFree did this implicitly)
     free_ws(g->ws);
-    dev_free(g->rp);
-    dev_free(g->col);
-    dev_free(g->w);
+    if (!g->borrowed) {
+        dev_free(g->rp);
+        dev_free(g->col);
+        dev_free(g->w);
+    }
     dev_free(g->deg8);
     dev_free(g->fnbr);
     dev_free(g->isolated);
@@ -373,6 +434,10 @@ SG_API int graph_free(sg_graph *g) {
     dev_free(g->cbo);
     if (g->scsr_state == 1) scsr_free(&g->scsr);
     delete g;
+    if (--g_live_graphs == 0) {   // the last graph: give the pool's memory back to the device
+        cudaDeviceSynchronize();
+        dev_trim(0);
+    }
     return SG_OK;
 }
 
@@ -699,6 +764,8 @@ static void prof_flush(Workspace *ws) {
     P.used = 0;
 }
 
+static unsigned long long *ws_scratch(sg_graph *g) { return g->ws->scratch; }
+
 static cudaStream_t stream_of(const sg_opts *o) { return o ? (cudaStream_t)o->stream : (cudaStream_t)0; }
 
 extern "C" {
@@ -739,9 +806,18 @@ SG_API int advance(const sg_graph *gc, const sg_frontier *in, sg_frontier *out, 
         }
         case SG_FN_BC_SIGMA: {
             const sg_bc_state *st = (const sg_bc_state *)state;
-            if (!st->level || !st->visited || !st->sigma) return fail(SG_ERR_STATE, "BC state needs level, visited, sigma");
+            if (!st->level || !st->visited || !st->sigma || !st->exp2_per_level)
+                return fail(SG_ERR_STATE, "BC state needs level, visited, sigma and exp2_per_level");
             if (!out) return fail(SG_ERR_STATE, "BC sigma advance needs an output frontier");
             launch_push_bc(L, BcArgs{st->visited, st->sigma, st->level, st->depth + 1, ob, os}, s);
+            // finish level depth+1 (reading C20): scale it by 2^-k, k = floor(log2 max sigma), and
+            // record E[depth+1] = E[depth] + k (bc.cu; the output holds exactly the new level)
+            TRY(compact(g, out, false, s));
+            unsigned long long *d_max = ws_scratch(g) + 4;
+            CK(cudaMemsetAsync(d_max, 0, sizeof(unsigned long long), s));
+            launch_bc_level_max(st->sigma, out->bits, out->offsets, out->st, g->v.nw1, d_max, s);
+            launch_bc_level_scale_and_stack(st->sigma, out->bits, out->offsets, out->st, g->v.nw1, d_max,
+                                            st->exp2_per_level, st->depth + 1, nullptr, nullptr, ws_scratch(g) + 5, s);
             break;
         }
         default:
@@ -1224,17 +1300,26 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     int cc_nb = (int)(((long long)G.n * 4 + lblock - 1) / (lblock > 0 ? lblock : 1));
     if (cc_nb < 1 || lblock <= 0) cc_nb = 1;
     if (cc_nb > 64) cc_nb = 64;
+    if (!g->sorted) cc_nb = 1;   // block offsets binary-search sorted rows
     if (cc_nb > 1 && o.direction != SG_DIR_PUSH && (g->cbo_nb != cc_nb)) {
         if (g->cbo) {
             CK(cudaStreamSynchronize(s));
             dev_free(g->cbo);
             g->cbo = nullptr;
+            g->cbo_nb = 0;
         }
+        // n x (nb - 1) block offsets: if they do not fit, pull unblocked (same result, more L2 misses)
         const int64_t S = (G.n + cc_nb - 1) / cc_nb;
-        CK(dev_alloc(&g->cbo, sizeof(uint32_t) * (size_t)G.n * (size_t)(cc_nb - 1), s));
-        launch_cc_block_offsets(G.rp, G.col, G.n, cc_nb, S, g->cbo, s);
-        g->cbo_nb = cc_nb;
+        if (dev_alloc(&g->cbo, sizeof(uint32_t) * (size_t)G.n * (size_t)(cc_nb - 1), s) != cudaSuccess) {
+            cudaGetLastError();
+            g->cbo = nullptr;
+            cc_nb = 1;
+        } else {
+            launch_cc_block_offsets(G.rp, G.col, G.n, cc_nb, S, g->cbo, s);
+            g->cbo_nb = cc_nb;
+        }
     }
+    if (cc_nb > 1 && g->cbo_nb != cc_nb) cc_nb = 1;
     CK(cudaEventRecord(ws->ev0, s));
     launch_iota_i32(label, G.n, s);
     sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];

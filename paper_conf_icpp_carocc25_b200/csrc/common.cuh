@@ -177,23 +177,51 @@ __device__ __forceinline__ void word_bounds(const GraphView &g, int64_t w, uint6
 
 }  // namespace sg
 
-// ---- device memory: one stream-ordered pool per process that keeps freed blocks (release
-// threshold = infinity), so a graph loaded after another one of similar size reuses its memory
-// without new driver mappings (graph_load_csr / graph_free in a loop: the e2e step).
+// ---- host helpers --------------------------------------------------------------------------
 namespace sg {
-inline cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s) {
-    static bool init = false;
-    if (!init) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaMemPool_t pool;
-        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-            uint64_t thr = ~0ull;
-            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-        }
-        init = true;
+// SM count of the current device, queried once per device (grid sizing: multiples of the SM count)
+inline int num_sms() {
+    static int cache[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148;
+    if (!cache[dev]) {
+        int n = 0;
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        cache[dev] = n > 0 ? n : 148;
     }
-    return cudaMallocAsync(p, bytes, s);
+    return cache[dev];
+}
+
+// ---- device memory: one private stream-ordered pool per device (release threshold = infinity),
+// so a graph loaded after another one of similar size reuses its memory without new driver
+// mappings (graph_load_csr / graph_free in a loop: the e2e step).  Private, so the process's
+// default pool (used by NCCL or torch's cudaMallocAsync backend) keeps its own policy; graph_free
+// trims the pool back to what is still allocated once it is idle (dev_trim).
+inline cudaMemPool_t graph_pool() {
+    static cudaMemPool_t pools[64] = {};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+    if (!pools[dev]) {
+        cudaMemPoolProps p = {};
+        p.allocType = cudaMemAllocationTypePinned;
+        p.handleTypes = cudaMemHandleTypeNone;
+        p.location.type = cudaMemLocationTypeDevice;
+        p.location.id = dev;
+        cudaMemPool_t pool;
+        if (cudaMemPoolCreate(&pool, &p) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        uint64_t thr = ~0ull;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[dev] = pool;
+    }
+    return pools[dev];
+}
+inline cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s) {
+    cudaMemPool_t pool = graph_pool();
+    if (!pool) return cudaMallocAsync(p, bytes, s);
+    return cudaMallocFromPoolAsync(p, bytes, pool, s);
 }
 template <class T>
 inline cudaError_t dev_alloc(T **p, size_t bytes, cudaStream_t s) {
@@ -202,5 +230,10 @@ inline cudaError_t dev_alloc(T **p, size_t bytes, cudaStream_t s) {
 // the caller guarantees no pending work uses p (graph_free synchronises the device first)
 inline void dev_free(void *p) {
     if (p) cudaFreeAsync(p, 0);
+}
+// release the pool's unused memory beyond `keep` bytes (graph_free with no other graph alive)
+inline void dev_trim(size_t keep) {
+    cudaMemPool_t pool = graph_pool();
+    if (pool) cudaMemPoolTrimTo(pool, keep);
 }
 }  // namespace sg

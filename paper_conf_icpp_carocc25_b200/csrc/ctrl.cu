@@ -41,7 +41,7 @@ __global__ void k_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *
 }
 void launch_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *st_src, int64_t nw1, cudaStream_t s) {
     int64_t blocks = (nw1 + 255) / 256;
-    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     note_launch();
     k_list_all<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(offsets, st_all, st_src, nw1);
 }
@@ -91,7 +91,7 @@ void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *b
                          unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
                          unsigned long long h_sweep, cudaStream_t s) {
     int64_t blocks = (n / 4 + 255) / 256;
-    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_bfs_prologue<<<(int)blocks, 256, 0, s>>>(c, n, deg8, bits, summ, offsets, st, visited, vis_old, h_loop, h_push,
@@ -101,14 +101,14 @@ void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *b
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s) {
     int64_t blocks = (nw1 + 255) / 256;
-    if (blocks > 148 * 4) blocks = 148 * 4;
+    if (blocks > num_sms() * 4) blocks = num_sms() * 4;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_clear_listed<<<(int)blocks, 256, 0, s>>>(bits, summ, offsets, st, nw2, zero_st);
 }
 void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s) {
     int64_t blocks = (n + 255) / 256;
-    if (blocks > 148 * 4) blocks = 148 * 4;
+    if (blocks > num_sms() * 4) blocks = num_sms() * 4;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_zero_u64<<<(int)blocks, 256, 0, s>>>(p, n);

@@ -114,7 +114,7 @@ __global__ void k_min_over_bits(GraphView g, const uint64_t *__restrict__ bits, 
 
 static int grid_for(int64_t items) {
     int64_t b = (items + 255) / 256;
-    if (b > 148 * 8) b = 148 * 8;
+    if (b > num_sms() * 8) b = num_sms() * 8;
     return (int)(b < 1 ? 1 : b);
 }
 

@@ -191,6 +191,57 @@ __global__ void k_validate_csr(GraphView g, unsigned long long *bad) {
     if (b) atomicAdd(bad, b);
 }
 
+// Row structure (reading C9: rows strictly ascending, no self-loops), warp per row:
+// bad[0] += pairs col[e] >= col[e+1] inside a row (unsorted or duplicate), bad[1] += self-loops.
+// Runs at every load (the segmented tier and the label-blocked CC pull need sorted rows).
+__global__ void k_row_check(GraphView g, unsigned long long *bad) {
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    unsigned long long unsorted = 0, loops = 0;
+    for (int64_t v = gw; v < g.n; v += nwarps) {
+        const int64_t s = g.rp[v], e = g.rp[v + 1];
+        if (e < s || s < 0 || e > g.nnz) continue;   // malformed row_ptr: reported by k_validate_csr
+        for (int64_t i = s + lane; i < e; i += 32) {
+            const int32_t c = g.col[i];
+            if (c == (int32_t)v) loops++;
+            if (i + 1 < e && c >= g.col[i + 1]) unsorted++;
+        }
+    }
+    unsorted = warp_sum(unsorted);
+    loops = warp_sum(loops);
+    if (lane == 0) {
+        if (unsorted) atomicAdd(bad, unsorted);
+        if (loops) atomicAdd(bad + 1, loops);
+    }
+}
+// Symmetry (reading C8), warp per row: every arc (v, u) needs v in row u (binary search; rows
+// sorted).  bad += arcs without their reverse.  SG_F_VALIDATE only (O(nnz log deg)).
+__global__ void k_symmetry(GraphView g, unsigned long long *bad) {
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    unsigned long long miss = 0;
+    for (int64_t v = gw; v < g.n; v += nwarps) {
+        const int64_t s = g.rp[v], e = g.rp[v + 1];
+        if (e < s || s < 0 || e > g.nnz) continue;
+        for (int64_t i = s + lane; i < e; i += 32) {
+            const int32_t u = g.col[i];
+            if (u < 0 || u >= g.n) continue;
+            int64_t lo = g.rp[u], hi = g.rp[u + 1];
+            if (hi < lo || lo < 0 || hi > g.nnz) { miss++; continue; }
+            while (lo < hi) {
+                const int64_t mid = (lo + hi) >> 1;
+                if (g.col[mid] < (int32_t)v) lo = mid + 1;
+                else hi = mid;
+            }
+            if (lo >= g.rp[u + 1] || g.col[lo] != (int32_t)v) miss++;
+        }
+    }
+    miss = warp_sum(miss);
+    if (lane == 0 && miss) atomicAdd(bad, miss);
+}
+
 __global__ void k_max_u8(const uint8_t *w, int64_t nnz, unsigned int *out) {
     unsigned int m = 0;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -240,26 +291,26 @@ static int grid_for(int64_t items, int threads, int max_blocks) {
 
 void launch_fill_all(uint64_t *bits, uint64_t *summ, int64_t n, int64_t nw1, int64_t nw2, cudaStream_t s) {
     note_launch();
-    k_fill_all<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(bits, summ, n, nw1, nw2);
+    k_fill_all<<<grid_for(nw1, 256, num_sms() * 8), 256, 0, s>>>(bits, summ, n, nw1, nw2);
 }
 void launch_insert(uint64_t *bits, uint64_t *summ, const int32_t *v, int64_t k, int64_t n, cudaStream_t s) {
-    if (k > 0) { note_launch(); k_insert<<<grid_for(k, 256, 148 * 8), 256, 0, s>>>(bits, summ, v, k, n); }
+    if (k > 0) { note_launch(); k_insert<<<grid_for(k, 256, num_sms() * 8), 256, 0, s>>>(bits, summ, v, k, n); }
 }
 void launch_setop(uint64_t *dst, const uint64_t *src, int64_t nw1, int op, cudaStream_t s) {
     note_launch();
-    k_setop<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(dst, src, nw1, op);
+    k_setop<<<grid_for(nw1, 256, num_sms() * 8), 256, 0, s>>>(dst, src, nw1, op);
 }
 void launch_rebuild_summary(const uint64_t *bits, uint64_t *summ, int64_t nw1, int64_t nw2, cudaStream_t s) {
     note_launch();
-    k_rebuild_summary<<<grid_for(nw2 * 32, 256, 148 * 8), 256, 0, s>>>(bits, summ, nw1, nw2);
+    k_rebuild_summary<<<grid_for(nw2 * 32, 256, num_sms() * 8), 256, 0, s>>>(bits, summ, nw1, nw2);
 }
 void launch_compact(const uint64_t *summ, int64_t nw2, uint32_t *offsets, DevStats *st, cudaStream_t s) {
     note_launch();
-    k_compact<<<grid_for(nw2, COMPACT_WARPS, 148 * 2), COMPACT_THREADS, 0, s>>>(summ, nw2, offsets, st);
+    k_compact<<<grid_for(nw2, COMPACT_WARPS, num_sms() * 2), COMPACT_THREADS, 0, s>>>(summ, nw2, offsets, st);
 }
 void launch_frontier_stats(const GraphView &g, const uint64_t *bits, DevStats *st, cudaStream_t s) {
     note_launch();
-    k_frontier_stats<<<grid_for(g.nw1, 256, 148 * 8), 256, 0, s>>>(bits, g.nw1, g.deg8, st);
+    k_frontier_stats<<<grid_for(g.nw1, 256, num_sms() * 8), 256, 0, s>>>(bits, g.nw1, g.deg8, st);
 }
 // 8-bit log code of each vertex degree (exact below 32, 3 mantissa bits above); padded to 64 B
 // per layer-1 word so k_frontier_stats can read whole words.
@@ -315,28 +366,28 @@ void launch_first_nbr(const int64_t *rp, const int32_t *col, const uint8_t *deg8
                       int32_t *fn, cudaStream_t s) {
     if (npad <= 0) return;
     note_launch();
-    k_first_nbr<<<grid_for(npad, 256, 148 * 8), 256, 0, s>>>(rp, col, deg8, n, npad, fn);
+    k_first_nbr<<<grid_for(npad, 256, num_sms() * 8), 256, 0, s>>>(rp, col, deg8, n, npad, fn);
 }
 void launch_isolated(const uint8_t *deg8, int64_t n, int64_t nw1, uint64_t *iso, cudaStream_t s) {
     note_launch();
-    k_isolated<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(deg8, n, nw1, iso);
+    k_isolated<<<grid_for(nw1, 256, num_sms() * 8), 256, 0, s>>>(deg8, n, nw1, iso);
 }
 void launch_deg8(const int64_t *rp, int64_t n, int64_t npad, uint8_t *deg8, cudaStream_t s) {
     note_launch();
-    k_deg8<<<grid_for(npad, 256, 148 * 8), 256, 0, s>>>(rp, n, npad, deg8);
+    k_deg8<<<grid_for(npad, 256, num_sms() * 8), 256, 0, s>>>(rp, n, npad, deg8);
 }
 void launch_popcount(const uint64_t *bits, int64_t nw1, unsigned long long *out, cudaStream_t s) {
     note_launch();
-    k_popcount<<<grid_for(nw1, 256, 148 * 4), 256, 0, s>>>(bits, nw1, out);
+    k_popcount<<<grid_for(nw1, 256, num_sms() * 4), 256, 0, s>>>(bits, nw1, out);
 }
 void launch_or_listed(const uint64_t *bits, const uint32_t *offsets, const DevStats *st, uint64_t *dst,
                       int64_t max_words, cudaStream_t s) {
     note_launch();
-    k_or_listed<<<grid_for(max_words, 256, 148 * 8), 256, 0, s>>>(bits, offsets, st, dst);
+    k_or_listed<<<grid_for(max_words, 256, num_sms() * 8), 256, 0, s>>>(bits, offsets, st, dst);
 }
 void launch_or_all(const uint64_t *bits, int64_t nw1, uint64_t *dst, cudaStream_t s) {
     note_launch();
-    k_or_all<<<grid_for(nw1, 256, 148 * 8), 256, 0, s>>>(bits, nw1, dst);
+    k_or_all<<<grid_for(nw1, 256, num_sms() * 8), 256, 0, s>>>(bits, nw1, dst);
 }
 void launch_set_u32(uint32_t *p, int64_t i, uint32_t v, cudaStream_t s) { note_launch(); k_set_one<uint32_t><<<1, 1, 0, s>>>(p, i, v); }
 void launch_set_i32(int32_t *p, int64_t i, int32_t v, cudaStream_t s) { note_launch(); k_set_one<int32_t><<<1, 1, 0, s>>>(p, i, v); }
@@ -358,7 +409,7 @@ void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src,
 // costs one memory latency) and stores the levels of vertices lane16 + 16 i (whole 64-B runs of
 // level[] per store instruction).  The last CTA decides the next superstep (graph mode).
 #ifndef SG_DIFF_BLOCKS
-#define SG_DIFF_BLOCKS (148 * 4)   // grid cap (CTAs)
+#define SG_DIFF_BLOCKS (num_sms() * 4)   // grid cap (CTAs)
 #endif
 #ifndef SG_DIFF_WPR
 #define SG_DIFF_WPR 8
@@ -504,18 +555,26 @@ void launch_sssp_diff(const GraphView &g, const uint32_t *dist, uint32_t *dist_o
     o.out_offsets = out_offsets;
     o.st = st;
     int64_t blocks = g.nw2;
-    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (blocks > num_sms() * 16) blocks = num_sms() * 16;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_sssp_diff<<<(int)blocks, 256, 0, s>>>(g, dist, dist_old, o);
 }
-void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(p, n); }
+void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, num_sms() * 8), 256, 0, s>>>(p, n); }
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s) {
     note_launch();
-    k_validate_csr<<<grid_for(g.nnz > g.n ? g.nnz : g.n, 256, 148 * 8), 256, 0, s>>>(g, bad);
+    k_validate_csr<<<grid_for(g.nnz > g.n ? g.nnz : g.n, 256, num_sms() * 8), 256, 0, s>>>(g, bad);
+}
+void launch_row_check(const GraphView &g, unsigned long long *bad, cudaStream_t s) {
+    note_launch();
+    k_row_check<<<grid_for(g.n * 32, 256, num_sms() * 8), 256, 0, s>>>(g, bad);
+}
+void launch_symmetry(const GraphView &g, unsigned long long *bad, cudaStream_t s) {
+    note_launch();
+    k_symmetry<<<grid_for(g.n * 32, 256, num_sms() * 8), 256, 0, s>>>(g, bad);
 }
 void launch_max_weight(const uint8_t *w, int64_t nnz, unsigned int *out, cudaStream_t s) {
-    if (nnz > 0) { note_launch(); k_max_u8<<<grid_for(nnz, 256, 148 * 8), 256, 0, s>>>(w, nnz, out); }
+    if (nnz > 0) { note_launch(); k_max_u8<<<grid_for(nnz, 256, num_sms() * 8), 256, 0, s>>>(w, nnz, out); }
 }
 
 }  // namespace sg

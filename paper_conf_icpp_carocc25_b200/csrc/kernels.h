@@ -33,6 +33,10 @@ void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s);
 void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src, cudaStream_t s,
                  uint64_t *vis_old = nullptr);
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s);
+// bad[0] += unsorted / duplicate pairs inside rows, bad[1] += self-loops (warp per row)
+void launch_row_check(const GraphView &g, unsigned long long *bad, cudaStream_t s);
+// bad[0] += arcs (v, u) whose reverse (u, v) is missing (rows must be sorted)
+void launch_symmetry(const GraphView &g, unsigned long long *bad, cudaStream_t s);
 void launch_max_weight(const uint8_t *w, int64_t nnz, unsigned int *out, cudaStream_t s);
 
 // push.cu — one push advance = k_push_words (+ k_push_heavy), functor selected by `fn`.

@@ -295,7 +295,7 @@ void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visi
                      cudaStream_t s) {
     // one CTA per layer-2 word in a grid-stride loop over SG_PULL_WAVES CTAs per SM
     int64_t blocks = g.nw2;
-    if (blocks > 148 * SG_PULL_WAVES) blocks = 148 * SG_PULL_WAVES;
+    if (blocks > num_sms() * SG_PULL_WAVES) blocks = num_sms() * SG_PULL_WAVES;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);

@@ -129,7 +129,7 @@ __global__ void k_cc_block_offsets(const int64_t *__restrict__ rp, const int32_t
 void launch_cc_block_offsets(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, uint32_t *cbo,
                              cudaStream_t s) {
     int64_t blocks = (n + 255) / 256;
-    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (blocks > num_sms() * 16) blocks = num_sms() * 16;
     note_launch();
     k_cc_block_offsets<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(rp, col, n, nb, S, cbo);
 }
@@ -202,7 +202,7 @@ k_pull_cc_block(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__
 void launch_pull_cc_block(const GraphView &g, int32_t *label, uint64_t *out_bits, DevStats *st, const uint32_t *cbo,
                           int nb, int b, cudaStream_t s) {
     int64_t blocks = (g.nw1 * 32 + CCP_THREADS - 1) / CCP_THREADS;
-    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_pull_cc_block<<<(int)blocks, CCP_THREADS, 0, s>>>(g, label, out_bits, st, cbo, nb, b);
@@ -211,7 +211,7 @@ void launch_pull_cc_block(const GraphView &g, int32_t *label, uint64_t *out_bits
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,
                     cudaStream_t s) {
     int64_t blocks = (g.nw1 * 32 + CCP_THREADS - 1) / CCP_THREADS;
-    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_pull_cc<<<(int)blocks, CCP_THREADS, 0, s>>>(g, label, out_bits, out_summ, st);

@@ -44,13 +44,13 @@ static void launch_push(const PushLaunch &L, const F &f, cudaStream_t s) {
         if (p.seg && p.seg_mode && L.g.hub_idx) {
             note_launch();
             // one CTA per SM (192 KB slice); at least one per destination segment (SG_SEG_OWNER)
-            k_push_seg<<<L.g.nseg > 148 ? L.g.nseg : 148, SEG_THREADS, SEG_SMEM, s>>>(p, f);
+            k_push_seg<<<L.g.nseg > num_sms() ? L.g.nseg : num_sms(), SEG_THREADS, SEG_SMEM, s>>>(p, f);
         }
     }
 }
 
-int push_max_grid_words() { return 148 * 4; }   // 64 regs x 256 threads: 4 CTAs per SM resident
-int push_max_grid_heavy() { return 148 * 3; }
+int push_max_grid_words() { return num_sms() * 4; }   // 64 regs x 256 threads: 4 CTAs per SM resident
+int push_max_grid_heavy() { return num_sms() * 3; }
 
 void launch_push_bfs(const PushLaunch &L, const BfsArgs &a, cudaStream_t s) {
     FnBfs f;
@@ -124,7 +124,7 @@ __global__ void k_hub_off(const int64_t *__restrict__ rp, const int32_t *__restr
 void launch_hub_mark(const int64_t *rp, int64_t n, int32_t *hub_idx, int32_t *hub_vertex, unsigned int *count,
                      cudaStream_t s) {
     int64_t blocks = (n + 255) / 256;
-    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     note_launch();
     k_hub_mark<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(rp, n, hub_idx, hub_vertex, count);
 }
@@ -132,7 +132,7 @@ void launch_hub_off(const int64_t *rp, const int32_t *col, const int32_t *hub_ve
                     uint32_t *off, cudaStream_t s) {
     const int64_t items = nh * (nseg + 1);
     int64_t blocks = (items + 255) / 256;
-    if (blocks > 148 * 8) blocks = 148 * 8;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     note_launch();
     k_hub_off<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(rp, col, hub_vertex, nh, nseg, off);
 }

@@ -595,16 +595,7 @@ __global__ void __launch_bounds__(256) k_frontier_arcs(const int64_t *__restrict
 // ---------------------------------------------------------------------------------------
 // host side
 
-static int sm_count() {
-    static int n = 0;
-    if (!n) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-        if (n <= 0) n = 148;
-    }
-    return n;
-}
+static int sm_count() { return num_sms(); }
 
 cudaError_t scsr_build(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int32_t sw, ScsrStore *out,
                        cudaStream_t s) {

@@ -64,12 +64,16 @@ class Layout:
     def nw2(self):
         return (self.nw1 + 63) // 64
 
-    def word_range(self, r):      # owned layer-1 words
+    def word_range(self, r):      # owned layer-1 words (empty vertex range -> empty word range)
         lo, hi = self.ranges[r]
+        if hi <= lo:
+            return lo // 64, lo // 64
         return lo // 64, min((hi + 63) // 64, self.nw1)
 
     def summ_range(self, r):      # owned layer-2 words
         a, b = self.word_range(r)
+        if b <= a:
+            return a // 64, a // 64
         return a // 64, min((b + 63) // 64, self.nw2)
 
 
@@ -97,7 +101,7 @@ class SliceExchange:
         torch.distributed.all_gather_into_tensor(recv, send, group=self.group)
         self.collectives += 1
         for r, (ra, rb) in enumerate(ranges):
-            if r != self.rank and rb > ra:
+            if r != self.rank and rb > ra:   # empty ranks own nothing (never overwrite a real slice)
                 full[ra:rb] = recv[r * chunk: r * chunk + (rb - ra)]
         return full
 

@@ -46,6 +46,21 @@ def test_lattice_degree_and_sources():
     assert len(set(s.tolist())) == 64 and (g.degrees()[s] > 0).all()
 
 
+def test_c5_sources_in_largest_component():
+    """Reading C15: config-5 sources come from the largest component (checked with the oracle's
+    union-find labels, independent of the scipy routine that builds the mask)."""
+    g = gen.lattice(120, 180, 0.6)
+    lab = oracle.cc(g)
+    big = np.bincount(lab).argmax()
+    mask = gen.largest_component_mask(g)
+    assert np.array_equal(mask.astype(bool), lab == big)
+    s = gen.sources(g, 64, stream=6, eligible=mask)
+    assert len(set(s.tolist())) == 64 and (lab[s] == big).all()
+    # the unrestricted draw on the same stream hits small clusters (so the restriction matters)
+    s_any = gen.sources(g, 64, stream=6)
+    assert (lab[s_any] != big).any()
+
+
 def test_weights_symmetric():
     g = gen.with_weights(gen.rmat(11, 16), seed=5)
     rows = np.repeat(np.arange(g.n), g.degrees())

@@ -136,3 +136,28 @@ def test_jacobi_step_bounds_final_values():
         front = new < lab
         lab = new
     assert np.array_equal(lab.astype(np.int32), oracle.cc(g))
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_jacobi_single_step_vs_brute_force(seed):
+    """One Jacobi step, pinned on its own (not through the fixed point): for every v,
+    new[v] = min(value[v], min over frontier neighbours u of value[u] + w(u,v)), computed here by a
+    pure-Python pull over v's row (the oracle pushes over source rows).  A step that ignored the
+    frontier restriction, dropped the weight, or took max instead of min fails."""
+    g = gen.with_weights(gen.rmat(7, 6, seed=seed, permute=True), seed=seed)
+    rng = np.random.default_rng(seed)
+    value = rng.integers(0, 500, g.n).astype(np.int64)
+    value[rng.random(g.n) < 0.2] = INF
+    front = rng.random(g.n) < 0.3
+    for weights in (g.weights, None):
+        got = oracle.jacobi_relax_step(g, front, value, weights)
+        for v in range(g.n):
+            best = int(value[v])
+            for e in range(int(g.row_ptr[v]), int(g.row_ptr[v + 1])):
+                u = int(g.col_idx[e])
+                if front[u]:
+                    c = int(value[u]) + (int(weights[e]) if weights is not None else 0)
+                    best = min(best, c)
+            assert got[v] == best, (v, got[v], best)
+        # the frontier restriction matters on this input
+        assert not np.array_equal(got, oracle.jacobi_relax_step(g, np.ones(g.n, bool), value, weights))

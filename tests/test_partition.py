@@ -135,3 +135,18 @@ def test_two_rank_gloo_protocol_reproduces_bfs_and_cc(world):
         assert ok_bfs, f"rank {rank}: distributed BFS differs from the oracle"
         assert ok_cc, f"rank {rank}: distributed CC differs from the oracle"
         assert ncoll > 0
+
+
+@pytest.mark.parametrize("n,P", [(3000, 4), (4097, 3), (70000, 8), (1, 2), (8191, 8)])
+def test_owned_slices_disjoint_and_covering(n, P):
+    """Empty ranks (n not a multiple of the alignment, P large) own no layer-1 / layer-2 word:
+    the owned word and summary slices are disjoint and cover the bitmap exactly."""
+    rp = np.arange(n + 1, dtype=np.int64) * 3      # uniform degrees (values irrelevant to ownership)
+    L = Layout(n, partition_ranges(rp, P))
+    for get, total in ((L.word_range, L.nw1), (L.summ_range, L.nw2)):
+        cover = np.zeros(total, np.int32)
+        for r in range(P):
+            a, b = get(r)
+            assert 0 <= a <= b <= total
+            cover[a:b] += 1
+        assert (cover == 1).all(), (get.__name__, cover)
