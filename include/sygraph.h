@@ -33,7 +33,7 @@ enum sg_status {
     SG_ERR_INVALID = -1,      /* bad argument (range, NULL, malformed CSR under SG_F_VALIDATE) */
     SG_ERR_OOM = -2,          /* device allocation failed */
     SG_ERR_CUDA = -3,         /* CUDA runtime/launch error (message in sg_last_error) */
-    SG_ERR_NCCL = -4,         /* reserved: collective failure */
+    SG_ERR_NCCL = -4,         /* partition exchange failure (bootstrap socket, IPC mapping, peer timeout) */
     SG_ERR_UNSUPPORTED = -5,  /* valid request outside the implemented envelope */
     SG_ERR_STATE = -6         /* missing functor state / iteration cap hit / handle misuse */
 };
@@ -58,6 +58,7 @@ enum { SG_DIR_AUTO = 0, SG_DIR_PUSH = 1, SG_DIR_PULL = 2 };                 /* B
 
 typedef struct sg_graph sg_graph;
 typedef struct sg_frontier sg_frontier;
+typedef struct sg_comm sg_comm;         /* ranks of a 1-D destination partition (one process per GPU) */
 
 /* Functor states for advance(): device pointers + scalars (Table 2: an advance functor
  * (src, dst, edge, weight) -> bool decides whether dst enters the output frontier). */
@@ -103,7 +104,10 @@ typedef struct {
     int32_t scsr;             /* run_bfs: heavy push supersteps over the destination-segmented arc copy
                                  (visited slice in shared memory, built at the first run_bfs that can use
                                  it, nnz x 4 B extra): 0 = auto (frontier arcs >= 4 Mi), 1 = off, 2 = always */
-    int32_t reserved[2];
+    int32_t owned_only;       /* partitioned graphs: 1 = run_bfs leaves level[] valid on this rank's owned
+                                 range only (no result gather; each rank holds its part, as in Graph500);
+                                 0 = level[] complete on every rank (default) */
+    int32_t reserved[1];
 } sg_opts;
 
 typedef struct {
@@ -115,14 +119,36 @@ typedef struct {
     double device_ms;         /* CUDA-event time of the call on its stream */
 } sg_stats;
 
+/* ---- communicator (§6 "static graph partitioning") ------------ */
+/* The ranks of a 1-D destination partition: one process per GPU on one node.  The communicator
+ * is a host-side bootstrap (TCP on 127.0.0.1, or SG_COMM_ADDR) used at graph-load time to agree
+ * on the partition and to exchange the CUDA IPC handles of each rank's exchange arena; every
+ * per-superstep exchange then runs inside the kernels over peer memory (NVLink P2P; two ranks
+ * may share one GPU, e.g. for tests).  Usage: rank 0 calls comm_unique_id, the caller broadcasts
+ * the 128 bytes (e.g. torch.distributed.broadcast_object_list), every rank calls comm_init with
+ * its rank and the CUDA device it uses.  Blocking; 120 s connect timeout -> SG_ERR_NCCL. */
+SG_API int comm_unique_id(uint8_t id[128]);
+SG_API int comm_init(const uint8_t id[128], int nranks, int rank, int device, sg_comm **out);
+SG_API int comm_free(sg_comm *c);
+SG_API int comm_info(const sg_comm *c, int *nranks, int *rank);
+
 /* ---- graph ---------------------------------------------------------------------------- */
 /* Copy a symmetric CSR to device memory owned by the returned handle (§3.1; timing of
  * the paper excludes this transfer).  mem = SG_MEM_HOST | SG_MEM_DEVICE says where the
  * three input arrays live; weights may be NULL.  n in [1, 2^31-1], nnz in [0, 2^40].
- * SG_F_VALIDATE checks row_ptr monotone, row_ptr[0] = 0, row_ptr[n] = nnz and 0 <= col < n on
- * the device (SG_ERR_INVALID on failure).  Synchronises `stream` before returning. */
+ * flags: SG_F_BORROW / SG_F_VALIDATE (above).  Synchronises `stream` before returning.
+ * comm (nullable; nranks == 1 behaves as NULL): collective over the communicator's ranks, which
+ * all pass the same full CSR (SG_ERR_INVALID if their partitions disagree).  Rank r keeps only
+ * its partition: owned destinations [lo_r, hi_r) (4,096-aligned, arc-balanced;
+ * graph_partition), the push block (arcs of every source into the owned range) and the pull
+ * block (the owned rows).  Rows must be sorted (SG_ERR_UNSUPPORTED otherwise).  run_bfs /
+ * run_sssp / run_cc on such a graph are collective (every rank calls them with the same
+ * arguments, in the same order); advance / run_bc return SG_ERR_UNSUPPORTED (BC shards sources
+ * over full replicas instead). */
 SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const int32_t *col_idx,
-                          const uint8_t *weights, int mem, int flags, void *stream, sg_graph **out);
+                          const uint8_t *weights, int mem, int flags, void *stream, sg_comm *comm, sg_graph **out);
+/* Owned destination range of a partitioned graph ([0, n) for a single-GPU graph). */
+SG_API int graph_partition(const sg_graph *g, int64_t *lo, int64_t *hi);
 SG_API int graph_free(sg_graph *g);
 SG_API int graph_info(const sg_graph *g, int64_t *n, int64_t *nnz, const int64_t **row_ptr,
                       const int32_t **col_idx, const uint8_t **weights);

@@ -35,7 +35,7 @@ class SgOpts(ctypes.Structure):
                 ("beta", ctypes.c_double), ("max_iters", ctypes.c_int64), ("heavy_degree", ctypes.c_int32),
                 ("small_degree", ctypes.c_int32), ("host_loop", ctypes.c_int32), ("segmented", ctypes.c_int32),
                 ("one_layer", ctypes.c_int32), ("coarsening", ctypes.c_int32), ("sssp_delta", ctypes.c_int32),
-                ("scsr", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2)]
+                ("scsr", ctypes.c_int32), ("owned_only", ctypes.c_int32), ("reserved", ctypes.c_int32 * 1)]
 
 
 class SgStats(ctypes.Structure):
@@ -76,7 +76,7 @@ EXPORTS = ["graph_load_csr", "graph_free", "graph_info", "frontier_init", "front
            "frontier_fill_all", "frontier_clear", "frontier_count", "frontier_view", "frontier_op",
            "frontier_or_into", "advance", "run_bfs", "run_sssp", "run_cc", "run_bc", "sg_opts_default",
            "sg_last_error", "sg_version", "sg_profile", "sg_profile_read", "sg_launch_count", "frontier_filter",
-           "compute_execute"]
+           "compute_execute", "comm_unique_id", "comm_init", "comm_free", "comm_info", "graph_partition"]
 SG_PRED_DEGREE_RANGE, SG_PRED_U32_RANGE, SG_PRED_I32_RANGE, SG_PRED_F64_RANGE, SG_PRED_IN_BITMAP = 0, 1, 2, 3, 4
 SG_OP_SET_U32, SG_OP_SET_I32, SG_OP_SET_F64, SG_OP_ADD_U32, SG_OP_ADD_F64 = 0, 1, 2, 3, 4
 
@@ -94,7 +94,12 @@ def load():
     vp, i64, i32, c_int = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_int
     pp = ctypes.POINTER(ctypes.c_void_p)
     sig = {
-        "graph_load_csr": (c_int, [i64, i64, vp, vp, vp, c_int, c_int, vp, pp]),
+        "graph_load_csr": (c_int, [i64, i64, vp, vp, vp, c_int, c_int, vp, vp, pp]),
+        "graph_partition": (c_int, [vp, ctypes.POINTER(i64), ctypes.POINTER(i64)]),
+        "comm_unique_id": (c_int, [ctypes.c_char_p]),
+        "comm_init": (c_int, [ctypes.c_char_p, c_int, c_int, c_int, pp]),
+        "comm_free": (c_int, [vp]),
+        "comm_info": (c_int, [vp, ctypes.POINTER(c_int), ctypes.POINTER(c_int)]),
         "graph_free": (c_int, [vp]),
         "graph_info": (c_int, [vp, vp, vp, vp, vp, vp]),
         "frontier_init": (c_int, [vp, pp]),
@@ -155,7 +160,7 @@ def _ptr_mem(a):
 
 
 def opts(stream=None, direction=SG_DIR_AUTO, alpha=14.0, beta=24.0, max_iters=0, heavy_degree=0, small_degree=0,
-         host_loop=False, segmented=0, one_layer=False, coarsening=0, sssp_delta=0, scsr=0):
+         host_loop=False, segmented=0, one_layer=False, coarsening=0, sssp_delta=0, scsr=0, owned_only=False):
     """segmented: BFS hub tier with the visited slice in shared memory (0 auto, 1 off, 2 always);
     one_layer: ablation without the summary layer; coarsening: words per warp grab (0 auto);
     scsr: BFS heavy push over the destination-segmented arc copy (0 auto, 1 off, 2 always)."""
@@ -166,6 +171,7 @@ def opts(stream=None, direction=SG_DIR_AUTO, alpha=14.0, beta=24.0, max_iters=0,
     o.heavy_degree, o.small_degree, o.host_loop = heavy_degree, small_degree, int(host_loop)
     o.segmented, o.one_layer, o.coarsening, o.sssp_delta = segmented, int(one_layer), coarsening, sssp_delta
     o.scsr = scsr
+    o.owned_only = int(owned_only)
     return o
 
 
@@ -185,10 +191,11 @@ class Graph:
             pass
 
 
-def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None, borrow=False) -> Graph:
+def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None, borrow=False, comm=None) -> Graph:
     """row_ptr int64[n+1], col_idx int32[nnz], weights uint8[nnz] (numpy/host tensors or CUDA tensors).
     borrow (CUDA tensors only): keep the tensors' memory instead of copying (SG_F_BORROW); the
-    returned Graph holds references to them."""
+    returned Graph holds references to them.  comm (a Comm): collective partitioned load — this
+    rank keeps its owned destination range (graph_partition) and run_* become collective."""
     rp, m1 = _ptr_mem(row_ptr)
     ci, m2 = _ptr_mem(col_idx)
     w, m3 = _ptr_mem(weights)
@@ -199,11 +206,65 @@ def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None, 
         raise ValueError("row_ptr, col_idx and weights must all be host or all be device arrays")
     h = ctypes.c_void_p()
     flags = (SG_F_VALIDATE if validate else 0) | (SG_F_BORROW if borrow else 0)
-    _check(load().graph_load_csr(n, nnz, rp, ci if nnz else None, w, m1, flags, _stream_ptr(stream), ctypes.byref(h)))
+    _check(load().graph_load_csr(n, nnz, rp, ci if nnz else None, w, m1, flags, _stream_ptr(stream),
+                                 comm.handle if comm is not None else None, ctypes.byref(h)))
     G = Graph(h.value, n, nnz, weights is not None)
+    G.comm = comm
     if borrow:
         G._borrowed = (row_ptr, col_idx, weights)
     return G
+
+
+def graph_partition(g: Graph):
+    """(lo, hi): the destination range this rank owns ([0, n) for a single-GPU graph)."""
+    lo, hi = ctypes.c_int64(), ctypes.c_int64()
+    _check(load().graph_partition(g.handle, ctypes.byref(lo), ctypes.byref(hi)))
+    return lo.value, hi.value
+
+
+# ------------------------------------------------------------------------ communicator
+class Comm:
+    """Ranks of a 1-D destination partition (include/sygraph.h comm_*); free after its graphs."""
+
+    def __init__(self, handle, nranks, rank):
+        self.handle, self.nranks, self.rank = handle, nranks, rank
+
+    def free(self):
+        if self.handle:
+            _check(load().comm_free(self.handle))
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def comm_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(load().comm_unique_id(buf))
+    return buf.raw
+
+
+def comm_init(uid: bytes, nranks: int, rank: int, device: int = 0) -> Comm:
+    h = ctypes.c_void_p()
+    _check(load().comm_init(ctypes.create_string_buffer(uid, 128), int(nranks), int(rank), int(device),
+                            ctypes.byref(h)))
+    return Comm(h.value, nranks, rank)
+
+
+def comm_from_torch(group=None, device: int | None = None) -> Comm:
+    """Bootstrap a Comm over an initialised torch.distributed process group (gloo or nccl): rank 0
+    creates the id, torch broadcasts it (plumbing only)."""
+    import torch
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    obj = [comm_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    if device is None:
+        device = torch.cuda.current_device() if torch.cuda.is_available() else 0
+    return comm_init(obj[0], world, rank, device)
 
 
 def graph_info(g: Graph):

@@ -5,6 +5,7 @@
 #pragma once
 #include "common.cuh"
 #include "kernels.h"
+#include "xchg.cuh"
 
 namespace sg {
 
@@ -27,18 +28,17 @@ __device__ __forceinline__ void bfs_set_cond(unsigned long long h, unsigned v) {
 }
 
 // Beamer direction policy (R2) + loop control, from the freshly built output frontier's
-// control block `st`; `prev` (nullable) = the control block of the frontier just advanced: its
-// arcs counter is folded into the per-direction totals, then it is zeroed (it is the next
-// superstep's output).  One thread.
-__device__ __forceinline__ void bfs_decide(BfsCtrl *c, const DevStats *st, DevStats *prev, unsigned long long h_loop,
-                                           unsigned long long h_push, unsigned long long h_pull,
-                                           unsigned long long h_sweep, int first) {
+// control block `st`; `prev_arcs` = arcs inspected by the superstep just run (folded into the
+// per-direction totals); `zero_prev` (nullable) = the control block of the frontier just advanced,
+// zeroed here (it is the next superstep's output).  One thread.
+__device__ __forceinline__ void bfs_decide(BfsCtrl *c, const DevStats *st, unsigned long long prev_arcs,
+                                           DevStats *zero_prev, unsigned long long h_loop, unsigned long long h_push,
+                                           unsigned long long h_pull, unsigned long long h_sweep, int first) {
     // control blocks were filled by atomics of other CTAs / kernels: volatile (L2) reads
     const volatile DevStats *vst = st;
-    if (prev) {
-        const unsigned long long pa = reinterpret_cast<const volatile DevStats *>(prev)->arcs;
-        if (c->pull) c->arcs_pulled += pa;
-        else c->arcs_pushed += pa;
+    if (!first) {
+        if (c->pull) c->arcs_pulled += prev_arcs;
+        else c->arcs_pushed += prev_arcs;
     }
     const unsigned long long count = vst->count;
     bool go = count > 0;
@@ -67,41 +67,62 @@ __device__ __forceinline__ void bfs_decide(BfsCtrl *c, const DevStats *st, DevSt
     bfs_set_cond(h_sweep, sweep);
     bfs_set_cond(h_pull, go && c->pull);
     bfs_set_cond(h_loop, go);
-    if (prev) *prev = DevStats{};
+    if (zero_prev) *zero_prev = DevStats{};
 }
 
 // Emit a block's slice of the output frontier: `S` = the block's layer-2 words (in shared
-// memory, nS of them, the first = layer-2 word sw0), written as is; their set bits are appended
-// to the word list with one atomic per block (ascending within the block).  Call with the whole
-// block; ends with __syncthreads.
-__device__ __forceinline__ void bfs_emit_words(const BfsOut &o, int64_t nw2, int64_t sw0, const uint64_t *S, int nS,
+// memory, nS of them, the first = layer-2 word sw0; words at or past w2_hi are not this rank's
+// and are skipped), written as is; their set bits are appended to the word list with one atomic
+// per block (ascending within the block).  Partitioned: the same layer-2 words and list entries
+// go to every peer's replica (one remote atomic per block and peer).  Call with the whole block;
+// ends with __syncthreads.
+__device__ __forceinline__ void bfs_emit_words(const BfsOut &o, int64_t w2_hi, int64_t sw0, const uint64_t *S, int nS,
                                                uint32_t *s_base) {
-    if ((int)threadIdx.x < nS && sw0 + threadIdx.x < nw2) o.out_summ[sw0 + threadIdx.x] = S[threadIdx.x];
+    const Xchg &x = o.x;
+    if ((int)threadIdx.x < nS && sw0 + threadIdx.x < w2_hi) xstore(x, o.out_summ + sw0 + threadIdx.x, S[threadIdx.x]);
     if (threadIdx.x == 0) {
         uint32_t tot = 0;
         for (int i = 0; i < nS; i++) tot += (uint32_t)__popcll(S[i]);
-        *s_base = tot ? (uint32_t)atomicAdd(&o.st->count, (unsigned long long)tot) : 0u;
+        s_base[0] = tot ? (uint32_t)atomicAdd(&o.st->count, (unsigned long long)tot) : 0u;
+        if (x.nranks > 1 && tot) {
+            unsigned long long b[SG_MAX_RANKS];
+#pragma unroll
+            for (int j = 0; j < SG_MAX_RANKS; j++)   // all remote atomics in flight together
+                b[j] = (j < x.nranks && j != x.rank) ? atomicAdd(&xpeer(x, o.st, j)->count, (unsigned long long)tot)
+                                                       : 0ull;
+#pragma unroll
+            for (int j = 0; j < SG_MAX_RANKS; j++) s_base[1 + j] = (uint32_t)b[j];
+        }
     }
     __syncthreads();
     for (int t = threadIdx.x; t < nS * 64; t += blockDim.x) {
         const int i = t >> 6, b = t & 63;
-        const uint64_t x = S[i];
-        if ((x >> b) & 1ull) {
-            uint32_t pos = *s_base + (uint32_t)__popcll(x & ((1ull << b) - 1ull));
+        const uint64_t xw = S[i];
+        if ((xw >> b) & 1ull) {
+            uint32_t pos = (uint32_t)__popcll(xw & ((1ull << b) - 1ull));
             for (int j = 0; j < i; j++) pos += (uint32_t)__popcll(S[j]);
-            o.out_offsets[pos] = (uint32_t)((sw0 + i) * 64 + b);
+            const uint32_t val = (uint32_t)((sw0 + i) * 64 + b);
+            o.out_offsets[s_base[0] + pos] = val;
+            if (x.nranks > 1) {
+                for (int j = 0; j < x.nranks; j++)
+                    if (j != x.rank) xpeer(x, o.out_offsets, j)[s_base[1 + j] + pos] = val;
+            }
         }
     }
     __syncthreads();
 }
 
 // End of the output kernel: block sums of n_f / m_f (and `arcs` into the input's control block),
-// then the last CTA to finish takes the direction decision (graph mode).  Whole block.
+// then the last CTA to finish takes the direction decision (graph mode).  Partitioned: the last
+// CTA first runs the superstep barrier (xchg.cuh) and replaces st's n_f / m_f by the global sums;
+// it zeroes the input's control block BEFORE publishing (peers add their word-list counts into it
+// as soon as they pass this barrier: it is the next superstep's output).  Whole block.
 __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long nf, unsigned long long mf,
                                            unsigned long long arcs, DevStats *in_st) {
     __shared__ unsigned long long s_r[3][32];
     __shared__ bool s_last;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const bool part = o.x.nranks > 1;
     nf = warp_sum(nf);
     mf = warp_sum(mf);
     arcs = warp_sum(arcs);
@@ -124,16 +145,32 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
         }
         if (c && in_st) atomicAdd(&in_st->arcs, c);
         s_last = false;
-        if (o.ctrl) {
-            __threadfence();
+        if (o.ctrl || part) {
+            if (part) __threadfence_system();   // this CTA's peer stores before the barrier's epoch
+            else __threadfence();
             s_last = atomicAdd(o.done, 1u) == gridDim.x - 1;
         }
     }
     __syncthreads();
     if (s_last && threadIdx.x == 0) {
-        __threadfence();
+        __threadfence_system();
         *o.done = 0u;
-        bfs_decide(o.ctrl, o.st, o.prev, o.h_loop, o.h_push, o.h_pull, o.h_sweep, 0);
+        DevStats *prev = o.prev ? o.prev : in_st;
+        unsigned long long prev_arcs = prev ? reinterpret_cast<const volatile DevStats *>(prev)->arcs : 0ull;
+        if (part) {
+            volatile DevStats *vst = o.st;
+            const unsigned long long my_nf = vst->nf, my_mf = vst->mf;
+            if (o.prev) *o.prev = DevStats{};   // zero before peers may add into it (next output)
+            XSlot tot;
+            xbarrier(o.x, my_nf, my_mf, prev_arcs, &tot);
+            vst->nf = tot.nf;
+            vst->mf = tot.mf;
+            prev_arcs = tot.arcs;
+            vst->pad = tot.arcs;   // host loops read the superstep's global arcs here
+            if (o.ctrl) bfs_decide(o.ctrl, o.st, prev_arcs, nullptr, o.h_loop, o.h_push, o.h_pull, o.h_sweep, 0);
+        } else if (o.ctrl) {
+            bfs_decide(o.ctrl, o.st, prev_arcs, o.prev, o.h_loop, o.h_push, o.h_pull, o.h_sweep, 0);
+        }
     }
 }
 

@@ -16,6 +16,7 @@
 
 #include "sygraph.h"
 #include "kernels.h"
+#include "comm.h"
 
 using namespace sg;
 
@@ -59,6 +60,25 @@ struct sg_frontier {
     uint32_t *offsets = nullptr;   // nw1 entries
     DevStats *st = nullptr;        // control block (device)
     bool owns_st = true;
+    bool in_arena = false;         // buffers carved from a partitioned graph's exchange arena
+};
+
+struct sg_comm {
+    Comm c;
+};
+
+// IPC-shared exchange memory of a partitioned graph (xchg.cuh): same layout on every rank, so a
+// local pointer p has the peer replica p + x.delta[j].
+struct Arena {
+    void *base = nullptr;
+    size_t bytes = 0;
+    XCtl *ctl = nullptr;
+    uint64_t *bits[2] = {}, *summ[2] = {};
+    uint32_t *offsets[2] = {};
+    DevStats *st = nullptr;        // 3 control blocks (fr[0], fr[1], spare)
+    uint32_t *vals = nullptr;      // n (+ pad) u32: SSSP dist / CC labels / BFS level gather, replicated
+    void *peer[SG_MAX_RANKS] = {};
+    Xchg x;
 };
 
 // Optional per-kernel-class timing (CUDA events on the launching stream) + algorithmic bytes
@@ -136,6 +156,15 @@ struct sg_graph {
     bool borrowed = false;          // SG_F_BORROW: rp / col / w are the caller's
     bool sorted = true;             // every row strictly ascending (checked at load)
     Workspace *ws = nullptr;
+    // 1-D destination partition: v = push block, vl = pull block (owned rows);
+    // single GPU: vl = v
+    GraphView vl;
+    int64_t nnz_global = 0;         // arcs of the whole graph (Beamer m_u, CC direction)
+    int64_t *rpl = nullptr;         // pull block buffers (partitioned only)
+    int32_t *coll = nullptr;
+    Arena *ar = nullptr;            // exchange arena (partitioned only)
+    int nranks = 1, rank = 0;
+    sg_comm *comm = nullptr;        // partitioned: graph_free is collective over it
 };
 static std::atomic<int> g_live_graphs{0};
 
@@ -156,6 +185,12 @@ static int alloc_frontier_bufs(sg_frontier *f, const sg_graph *g, bool own_st) {
 }
 
 static void free_frontier_bufs(sg_frontier *f) {
+    if (f->in_arena) {
+        f->bits = f->summ = nullptr;
+        f->offsets = nullptr;
+        f->st = nullptr;
+        return;
+    }
     cudaFree(f->bits);
     cudaFree(f->summ);
     cudaFree(f->offsets);
@@ -169,13 +204,29 @@ static int ensure_ws(sg_graph *g) {
     if (g->ws) return SG_OK;
     Workspace *ws = new Workspace();
     g->ws = ws;
-    CK(cudaMalloc(&ws->st, 3 * sizeof(DevStats)));   // fr[0], fr[1], one-layer ablation list
-    CK(cudaMemset(ws->st, 0, 3 * sizeof(DevStats)));
     CK(cudaMallocHost(&ws->h_st, 3 * sizeof(DevStats)));
-    for (int i = 0; i < 2; i++) {
-        TRY(alloc_frontier_bufs(&ws->fr[i], g, false));
-        ws->fr[i].st = ws->st + i;
+    if (g->ar) {   // partitioned: the two frontiers and their control blocks live in the arena
+        ws->st = g->ar->st;
+        for (int i = 0; i < 2; i++) {
+            sg_frontier &f = ws->fr[i];
+            f.g = g;
+            f.bits = g->ar->bits[i];
+            f.summ = g->ar->summ[i];
+            f.offsets = g->ar->offsets[i];
+            f.st = ws->st + i;
+            f.owns_st = false;
+            f.in_arena = true;
+        }
+    } else {
+        CK(cudaMalloc(&ws->st, 3 * sizeof(DevStats)));   // fr[0], fr[1], one-layer ablation list
+        CK(cudaMemset(ws->st, 0, 3 * sizeof(DevStats)));
+        for (int i = 0; i < 2; i++) {
+            TRY(alloc_frontier_bufs(&ws->fr[i], g, false));
+            ws->fr[i].st = ws->st + i;
+        }
     }
+    CK(cudaMalloc(&ws->bfs_done, sizeof(unsigned int)));
+    CK(cudaMemset(ws->bfs_done, 0, sizeof(unsigned int)));
     CK(cudaMalloc(&ws->visited, sizeof(uint64_t) * (size_t)g->v.nw1));
     CK(cudaMalloc(&ws->vis_old, sizeof(uint64_t) * (size_t)g->v.nw1));
     CK(cudaMalloc(&ws->scratch, 8 * sizeof(unsigned long long)));
@@ -208,8 +259,9 @@ static int ensure_heavy(sg_graph *g, int32_t heavy_deg) {
 
 static void free_ws(Workspace *ws) {
     if (!ws) return;
+    const bool arena = ws->fr[0].in_arena;
     for (int i = 0; i < 2; i++) free_frontier_bufs(&ws->fr[i]);
-    cudaFree(ws->st);
+    if (!arena) cudaFree(ws->st);
     cudaFreeHost(ws->h_st);
     cudaFree(ws->visited);
     cudaFree(ws->vis_old);
@@ -282,6 +334,163 @@ SG_API void sg_opts_default(sg_opts *o) {
     o->beta = 24.0;
 }
 
+// ---- 1-D destination partition: bounds, blocks, exchange arena -------------------------------
+static size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+// Allocate the IPC-shared arena, exchange handles over the communicator, map every peer's arena.
+static int arena_create(sg_graph *g, cudaStream_t s) {
+    Comm &C = g->comm->c;
+    const GraphView &G = g->v;
+    Arena *A = new Arena();
+    g->ar = A;
+    size_t off = 0;
+    const size_t o_ctl = off;
+    off += al256(sizeof(XCtl));
+    size_t o_bits[2], o_summ[2], o_off[2];
+    for (int i = 0; i < 2; i++) {
+        o_bits[i] = off;
+        off += al256(sizeof(uint64_t) * (size_t)(G.nw1 + 8));
+        o_summ[i] = off;
+        off += al256(sizeof(uint64_t) * (size_t)G.nw2);
+        o_off[i] = off;
+        off += al256(sizeof(uint32_t) * (size_t)G.nw1);
+    }
+    const size_t o_st = off;
+    off += al256(3 * sizeof(DevStats));
+    const size_t o_vals = off;
+    off += al256(sizeof(uint32_t) * (size_t)(G.n + 4));
+    A->bytes = off;
+    CK(cudaMalloc(&A->base, A->bytes));   // plain cudaMalloc: exportable through cudaIpcGetMemHandle
+    CK(cudaMemsetAsync(A->base, 0, A->bytes, s));
+    CK(cudaStreamSynchronize(s));
+    char *b = static_cast<char *>(A->base);
+    A->ctl = reinterpret_cast<XCtl *>(b + o_ctl);
+    for (int i = 0; i < 2; i++) {
+        A->bits[i] = reinterpret_cast<uint64_t *>(b + o_bits[i]);
+        A->summ[i] = reinterpret_cast<uint64_t *>(b + o_summ[i]);
+        A->offsets[i] = reinterpret_cast<uint32_t *>(b + o_off[i]);
+    }
+    A->st = reinterpret_cast<DevStats *>(b + o_st);
+    A->vals = reinterpret_cast<uint32_t *>(b + o_vals);
+    struct Hello {
+        cudaIpcMemHandle_t h;
+        unsigned long long bytes;
+        int device;
+        int pad;
+    } me{}, all[SG_MAX_RANKS];
+    CK(cudaIpcGetMemHandle(&me.h, A->base));
+    me.bytes = A->bytes;
+    me.device = g->device;
+    std::string err;
+    if (comm_allgather(&C, &me, all, sizeof me, err) != 0) return fail(SG_ERR_NCCL, "arena handle exchange: %s", err.c_str());
+    A->x.nranks = C.nranks;
+    A->x.rank = C.rank;
+    A->x.ctl = A->ctl;
+    for (int j = 0; j < C.nranks; j++) {
+        if (all[j].bytes != A->bytes) return fail(SG_ERR_INVALID, "ranks disagree on the graph size (arena %llu vs %llu B)",
+                                                  (unsigned long long)all[j].bytes, (unsigned long long)A->bytes);
+        if (j == C.rank) continue;
+        void *p = nullptr;
+        const cudaError_t e = cudaIpcOpenMemHandle(&p, all[j].h, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(SG_ERR_NCCL, "cudaIpcOpenMemHandle of rank %d's arena (device %d) failed: %s", j, all[j].device,
+                        cudaGetErrorString(e));
+        }
+        A->peer[j] = p;
+        A->x.delta[j] = (long long)((char *)p - (char *)A->base);
+    }
+    // every rank has mapped every peer before any kernel may store into a peer's arena
+    int one = 1, ones[SG_MAX_RANKS];
+    if (comm_allgather(&C, &one, ones, sizeof one, err) != 0) return fail(SG_ERR_NCCL, "barrier: %s", err.c_str());
+    return SG_OK;
+}
+
+static void arena_free(sg_graph *g) {
+    Arena *A = g->ar;
+    if (!A) return;
+    for (int j = 0; j < SG_MAX_RANKS; j++)
+        if (A->peer[j]) cudaIpcCloseMemHandle(A->peer[j]);
+    // no rank frees its arena while a peer still maps it
+    if (g->comm) {
+        std::string err;
+        int one = 1, ones[SG_MAX_RANKS];
+        comm_allgather(&g->comm->c, &one, ones, sizeof one, err);
+    }
+    cudaFree(A->base);
+    delete A;
+    g->ar = nullptr;
+}
+
+// Partition the loaded full CSR (g->rp / col / w) across the communicator: bounds (agreed by
+// all ranks), push block + pull block of this rank, exchange arena.
+static int partition_graph(sg_graph *g, cudaStream_t s) {
+    Comm &C = g->comm->c;
+    const int P = C.nranks;
+    const int64_t n = g->v.n, nnz = g->v.nnz;
+    if (!g->sorted) return fail(SG_ERR_UNSUPPORTED, "a partitioned graph needs sorted rows (binary-searched row parts)");
+    int64_t q[SG_MAX_RANKS] = {0};
+    CK(part_quantiles(g->rp, n, nnz, P, q, s));
+    int64_t bounds[SG_MAX_RANKS + 1];
+    bounds[0] = 0;
+    for (int r = 1; r < P; r++) {   // partition.py: partition_ranges (ALIGN = 4096)
+        int64_t v = (q[r - 1] + 2048) / 4096 * 4096;
+        if (v < bounds[r - 1]) v = bounds[r - 1];
+        if (v > n) v = n;
+        bounds[r] = v;
+    }
+    bounds[P] = n;
+    struct Agree {
+        int64_t n, nnz, bounds[SG_MAX_RANKS + 1];
+    } me{}, all[SG_MAX_RANKS];
+    me.n = n;
+    me.nnz = nnz;
+    for (int r = 0; r <= P; r++) me.bounds[r] = bounds[r];
+    std::string err;
+    if (comm_allgather(&C, &me, all, sizeof me, err) != 0) return fail(SG_ERR_NCCL, "partition exchange: %s", err.c_str());
+    for (int j = 0; j < P; j++)
+        if (memcmp(&all[j], &me, sizeof me) != 0)
+            return fail(SG_ERR_INVALID, "rank %d loaded a different graph (n / nnz / partition bounds differ)", j);
+    const int64_t lo = bounds[C.rank], hi = bounds[C.rank + 1];
+    int64_t *rpp = nullptr, *rpl = nullptr;
+    int32_t *colp = nullptr, *coll = nullptr;
+    uint8_t *wp = nullptr;
+    int64_t nnzp = 0, nnzl = 0;
+    CK(part_push_block(g->rp, g->col, g->w, n, lo, hi, &rpp, &colp, &wp, &nnzp, s));
+    CK(part_pull_block(g->rp, g->col, n, lo, hi, &rpl, &coll, &nnzl, s));
+    if (!g->borrowed) {
+        dev_free(g->rp);
+        dev_free(g->col);
+        dev_free(g->w);
+    }
+    g->borrowed = false;   // the blocks are the graph's own
+    g->rp = rpp;
+    g->col = colp;
+    g->w = wp;
+    g->rpl = rpl;
+    g->coll = coll;
+    GraphView &V = g->v;
+    V.rp = rpp;
+    V.col = colp;
+    V.w = wp;
+    V.nnz = nnzp;
+    V.hub_idx = nullptr;   // the hub-segmented tier and the sweep are single-GPU structures
+    V.hub_off = nullptr;
+    g->scsr_state = -1;
+    V.own_lo = lo;
+    V.own_hi = hi;
+    V.w1_lo = lo / 64;
+    V.w1_hi = hi > lo ? (hi + 63) / 64 : lo / 64;
+    V.w2_lo = V.w1_lo / 64;
+    V.w2_hi = hi > lo ? (V.w1_hi + 63) / 64 : V.w1_lo / 64;
+    g->vl = V;
+    g->vl.rp = rpl;
+    g->vl.col = coll;
+    g->vl.w = nullptr;
+    g->vl.nnz = nnzl;
+    return arena_create(g, s);
+}
+
 // bytes readable from p to the end of its allocation (driver allocation range), -1 if unknown
 // (cuMemGetAddressRange through cudaGetDriverEntryPoint: the library does not link libcuda)
 static long long bytes_to_alloc_end(const void *p) {
@@ -304,7 +513,7 @@ static long long bytes_to_alloc_end(const void *p) {
 }
 
 SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const int32_t *col_idx,
-                          const uint8_t *weights, int mem, int flags, void *stream, sg_graph **out) {
+                          const uint8_t *weights, int mem, int flags, void *stream, sg_comm *comm, sg_graph **out) {
     t_err.clear();
     if (!out) return fail(SG_ERR_INVALID, "out is NULL");
     *out = nullptr;
@@ -339,7 +548,20 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     g->v.nnz = nnz;
     g->v.nw1 = (n + 63) / 64;
     g->v.nw2 = (g->v.nw1 + 63) / 64;
+    g->v.own_lo = 0;
+    g->v.own_hi = n;
+    g->v.w1_lo = 0;
+    g->v.w1_hi = g->v.nw1;
+    g->v.w2_lo = 0;
+    g->v.w2_hi = g->v.nw2;
+    g->nnz_global = nnz;
     g->borrowed = borrow;
+    const bool part = comm && comm->c.nranks > 1;
+    if (part) {
+        g->comm = comm;
+        g->nranks = comm->c.nranks;
+        g->rank = comm->c.rank;
+    }
     if (borrow) {
         g->rp = const_cast<int64_t *>(row_ptr);
         g->col = const_cast<int32_t *>(col_idx);
@@ -404,6 +626,16 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     if (!g->sorted) g->scsr_state = -1;   // the segment-major copy needs sorted rows
     g->nhubs = (int64_t)(hv[2] & 0xffffffffu);
     g->v.nseg = (int32_t)((n + SEG_V - 1) / SEG_V);
+    if (part) {
+        g->nhubs = 0;
+        const int r = partition_graph(g, s);
+        if (r != SG_OK) {
+            const std::string msg = t_err;
+            graph_free(g);
+            t_err = msg;
+            return r;
+        }
+    }
     if (g->nhubs > 0 && g->sorted) {   // hub segment offsets binary-search sorted rows
         CK(dev_alloc(&g->hub_off, sizeof(uint32_t) * (size_t)g->nhubs * (size_t)(g->v.nseg + 1), s));
         launch_hub_off(g->rp, g->col, g->hub_vertex, g->nhubs, g->v.nseg, g->hub_off, s);
@@ -412,6 +644,7 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
         g->v.hub_idx = g->hub_idx;
         g->v.hub_off = g->hub_off;
     }
+    if (!part) g->vl = g->v;
     *out = g;
     return SG_OK;
 }
@@ -420,6 +653,10 @@ SG_API int graph_free(sg_graph *g) {
     if (!g) return SG_OK;
     cudaDeviceSynchronize();   // no pending work may use the buffers (cudaFree did this implicitly)
     free_ws(g->ws);
+    g->ws = nullptr;
+    arena_free(g);
+    dev_free(g->rpl);
+    dev_free(g->coll);
     if (!g->borrowed) {
         dev_free(g->rp);
         dev_free(g->col);
@@ -449,6 +686,56 @@ SG_API int graph_info(const sg_graph *g, int64_t *n, int64_t *nnz, const int64_t
     if (row_ptr) *row_ptr = g->rp;
     if (col_idx) *col_idx = g->col;
     if (weights) *weights = g->w;
+    return SG_OK;
+}
+
+SG_API int graph_partition(const sg_graph *g, int64_t *lo, int64_t *hi) {
+    if (!g) return fail(SG_ERR_INVALID, "graph is NULL");
+    if (lo) *lo = g->v.own_lo;
+    if (hi) *hi = g->v.own_hi;
+    return SG_OK;
+}
+
+// ---- communicator ---------------------------------------------------------------------------
+SG_API int comm_unique_id(uint8_t id[128]) {
+    t_err.clear();
+    if (!id) return fail(SG_ERR_INVALID, "id is NULL");
+    std::string err;
+    if (comm_create_id(id, err) != 0) return fail(SG_ERR_NCCL, "comm_unique_id: %s", err.c_str());
+    return SG_OK;
+}
+
+SG_API int comm_init(const uint8_t id[128], int nranks, int rank, int device, sg_comm **out) {
+    t_err.clear();
+    if (!id || !out) return fail(SG_ERR_INVALID, "NULL argument");
+    *out = nullptr;
+    if (nranks < 1 || nranks > SG_MAX_RANKS || rank < 0 || rank >= nranks)
+        return fail(SG_ERR_INVALID, "nranks %d / rank %d outside [1, %d] / [0, nranks)", nranks, rank, SG_MAX_RANKS);
+    sg_comm *c = new sg_comm();
+    c->c.device = device;
+    std::string err;
+    if (nranks > 1 && comm_connect(&c->c, id, nranks, rank, err) != 0) {
+        comm_close(&c->c);
+        delete c;
+        return fail(SG_ERR_NCCL, "comm_init: %s", err.c_str());
+    }
+    c->c.nranks = nranks;
+    c->c.rank = rank;
+    *out = c;
+    return SG_OK;
+}
+
+SG_API int comm_free(sg_comm *c) {
+    if (!c) return SG_OK;
+    comm_close(&c->c);
+    delete c;
+    return SG_OK;
+}
+
+SG_API int comm_info(const sg_comm *c, int *nranks, int *rank) {
+    if (!c) return fail(SG_ERR_INVALID, "comm is NULL");
+    if (nranks) *nranks = c->c.nranks;
+    if (rank) *rank = c->c.rank;
     return SG_OK;
 }
 
@@ -775,6 +1062,7 @@ SG_API int advance(const sg_graph *gc, const sg_frontier *in, sg_frontier *out, 
                    void *stream) {
     t_err.clear();
     if (!gc || !in || !state) return fail(SG_ERR_INVALID, "NULL argument");
+    if (gc->ar) return fail(SG_ERR_UNSUPPORTED, "advance on a partitioned graph: use run_bfs / run_sssp / run_cc");
     if (in->g != gc || (out && out->g != gc)) return fail(SG_ERR_INVALID, "frontier belongs to another graph");
     sg_graph *g = const_cast<sg_graph *>(gc);
     cudaStream_t s = (cudaStream_t)stream;
@@ -893,10 +1181,6 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     ws->bfs_exec = nullptr;
     ws->bfs_graph = nullptr;
     if (!ws->cap_stream) CK(cudaStreamCreateWithFlags(&ws->cap_stream, cudaStreamNonBlocking));
-    if (!ws->bfs_done) {
-        CK(cudaMalloc(&ws->bfs_done, sizeof(unsigned int)));
-        CK(cudaMemset(ws->bfs_done, 0, sizeof(unsigned int)));
-    }
     if (!ws->ctrl) {
         CK(cudaMalloc(&ws->ctrl, sizeof(BfsCtrl)));
         CK(cudaMallocHost(&ws->h_ctrl, sizeof(BfsCtrl)));
@@ -925,7 +1209,8 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
     launch_bfs_prologue(ws->ctrl, G.n, G.deg8, F[0]->bits, F[0]->summ, F[0]->offsets, F[0]->st, ws->visited,
                         ws->vis_old, (unsigned long long)h_loop, (unsigned long long)h_push[0],
-                        (unsigned long long)h_pull[0], sc ? (unsigned long long)h_sweep[0] : 0ull, cs);
+                        (unsigned long long)h_pull[0], sc ? (unsigned long long)h_sweep[0] : 0ull,
+                        g->ar ? g->ar->x : Xchg{}, cs);
     TRY(capture_end(cs, leaves));
     cudaGraphNode_t wnode;
     cudaGraph_t body;
@@ -947,10 +1232,11 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         BfsArgs a{ws->visited, nullptr, 0u, nullptr, nullptr, &ws->ctrl->next, &ws->ctrl->level, 1u};
         // output of the superstep (out->st was zeroed by the previous decision / the prologue);
         // the output kernel's last CTA decides the next superstep (handles of the other half)
-        const BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, nullptr, 0u, &ws->ctrl->next,
-                        &ws->ctrl->level, out->st, ws->ctrl, in->st, ws->bfs_done, (unsigned long long)h_loop,
-                        (unsigned long long)h_push[half ^ 1], (unsigned long long)h_pull[half ^ 1],
-                        sc ? (unsigned long long)h_sweep[half ^ 1] : 0ull};
+        BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, nullptr, 0u, &ws->ctrl->next,
+                  &ws->ctrl->level, out->st, ws->ctrl, in->st, ws->bfs_done, (unsigned long long)h_loop,
+                  (unsigned long long)h_push[half ^ 1], (unsigned long long)h_pull[half ^ 1],
+                  sc ? (unsigned long long)h_sweep[half ^ 1] : 0ull};
+        if (g->ar) bo.x = g->ar->x;   // partitioned: owned slice replicated to the peers + barrier
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
         launch_bfs_diff(G, ws->visited, bo, cs);
@@ -962,7 +1248,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
             TRY(capture_end(cs, leaves));
         }
         TRY(capture_begin(cs, b_pull, {}));
-        launch_pull_bfs(G, in->bits, ws->visited, in->st, bo, cs);   // writes its output itself
+        launch_pull_bfs(g->vl, in->bits, ws->visited, in->st, bo, cs);   // writes its output itself
         TRY(capture_end(cs, leaves));
         deps = {n_push, n_pull};
         if (n_sweep) deps.push_back(n_sweep);
@@ -973,6 +1259,15 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     ws->bfs_seg = t.seg;
     ws->bfs_cf = t.cf;
     ws->bfs_scsr = t.scsr != 0 && g->scsr_state == 1 ? t.scsr : 0;
+    return SG_OK;
+}
+
+// partitioned runs: a peer that missed a superstep barrier (timeout) poisons the run
+static int check_peers(sg_graph *g) {
+    if (!g->ar) return SG_OK;
+    unsigned long long err = 0;
+    CK(cudaMemcpy(&err, &g->ar->ctl->error, sizeof err, cudaMemcpyDeviceToHost));
+    if (err) return fail(SG_ERR_NCCL, "a peer rank did not reach a superstep barrier within the timeout");
     return SG_OK;
 }
 
@@ -987,7 +1282,7 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     BfsCtrl &c = *ws->h_ctrl;
     memset(&c, 0, sizeof c);
     c.level = level;
-    c.mu = g->v.nnz;
+    c.mu = g->nnz_global;
     c.n = g->v.n;
     c.max_iters = max_iters;
     c.alpha = o.alpha;
@@ -1001,12 +1296,19 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     CK(cudaEventRecord(ws->ev0, s));
     CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, sizeof(BfsCtrl), cudaMemcpyHostToDevice, s));
     CK(cudaGraphLaunch(ws->bfs_exec, s));
+    if (g->ar && !o.owned_only) {   // result gather: owned level slices into every rank's replica
+        const Arena *A = g->ar;
+        launch_publish_owned(level, A->vals, g->v.own_lo, g->v.own_hi, A->x, s);
+        launch_xbarrier(A->x, s);
+        CK(cudaMemcpyAsync(level, A->vals, sizeof(uint32_t) * (size_t)g->v.n, cudaMemcpyDeviceToDevice, s));
+    }
     CK(cudaMemcpyAsync(ws->h_ctrl, ws->ctrl, sizeof(BfsCtrl), cudaMemcpyDeviceToHost, s));
     CK(cudaEventRecord(ws->ev1, s));
     CK(cudaEventSynchronize(ws->ev1));
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
     CK(cudaGetLastError());
+    TRY(check_peers(g));
     if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
     {
         // kernels the graph executed: the prologue kernel + the
@@ -1045,9 +1347,16 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
     cudaStream_t s = stream_of(&o);
     TRY(ensure_ws(g));
-    const Tiers t = tiers_from(&o);
+    Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
+    if (g->ar) {   // partitioned: the device-driven loop (every superstep ends in the peer barrier)
+        if (o.host_loop || o.one_layer)
+            return fail(SG_ERR_UNSUPPORTED, "a partitioned BFS runs device-driven only (no host_loop / one_layer)");
+        t.seg = 0;
+        t.scsr = 0;
+        return run_bfs_graph(g, src, level, o, t, max_iters, stats);
+    }
     const bool scsr_on =
         !o.one_layer && scsr_ready(g, t, o.direction == SG_DIR_PUSH || env_or("SG_SCSR_EAGER", 0) != 0, s);
     if (!ws->prof.on && !o.host_loop && !o.one_layer) return run_bfs_graph(g, src, level, o, t, max_iters, stats);
@@ -1166,6 +1475,131 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     return SG_OK;
 }
 
+}  // extern "C"
+
+// ---- SSSP / CC over the 1-D destination partition (xchg.cuh) ------------------
+// Every rank holds the replicated value array (arena vals) and frontier; a superstep = the local
+// advance over the push block (SSSP relax / CC push: atomicMin on owned destinations only) or the
+// pull over the owned rows (CC), then k_value_diff over the owned words: the vertices whose value
+// decreased form the owned slice of the next frontier, and it stores the changed values, the
+// output words and the word list into every peer's replica and runs the superstep barrier.  The
+// host reads one control block per superstep (global count / n_f / m_f / arcs), as the single-GPU
+// SSSP / CC loops do.  A peer's values of superstep e may land while this rank still relaxes
+// superstep e: asynchronous relaxation (reading C12), same fixed point.
+static int run_value_part(sg_graph *g, bool cc, int32_t src, uint32_t *result, const sg_opts &o, sg_stats *stats) {
+    Workspace *ws = g->ws;
+    Arena *A = g->ar;
+    const GraphView &G = g->v;
+    cudaStream_t s = stream_of(&o);
+    Tiers t = tiers_from(&o);
+    t.seg = 0;
+    t.scsr = 0;
+    TRY(ensure_heavy(g, t.heavy));
+    const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
+    uint32_t *vals = A->vals;
+    if (!ws->dist_old) CK(cudaMalloc(&ws->dist_old, sizeof(uint32_t) * (size_t)(G.n + 4)));
+    // label-blocked pull over the owned rows (CC, as run_cc)
+    int cc_nb = 1;
+    if (cc && o.direction != SG_DIR_PUSH) {
+        const long long lblock = (long long)env_or("SG_CC_LBLOCK_KB", 32768) << 10;
+        cc_nb = (int)(((long long)G.n * 4 + lblock - 1) / (lblock > 0 ? lblock : 1));
+        if (cc_nb < 1 || lblock <= 0) cc_nb = 1;
+        if (cc_nb > 64) cc_nb = 64;
+        if (cc_nb > 1 && g->cbo_nb != cc_nb) {
+            if (g->cbo) {
+                CK(cudaStreamSynchronize(s));
+                dev_free(g->cbo);
+                g->cbo = nullptr;
+                g->cbo_nb = 0;
+            }
+            if (dev_alloc(&g->cbo, sizeof(uint32_t) * (size_t)G.n * (size_t)(cc_nb - 1), s) != cudaSuccess) {
+                cudaGetLastError();
+                g->cbo = nullptr;
+            } else {
+                launch_cc_block_offsets(g->vl.rp, g->vl.col, G.n, cc_nb, (G.n + cc_nb - 1) / cc_nb, g->cbo, s);
+                g->cbo_nb = cc_nb;
+            }
+        }
+        if (g->cbo_nb != cc_nb) cc_nb = 1;
+    }
+    CK(cudaEventRecord(ws->ev0, s));
+    if (cc) {
+        launch_iota_i32(reinterpret_cast<int32_t *>(vals), G.n, s);
+    } else {
+        CK(cudaMemsetAsync(vals, 0xFF, sizeof(uint32_t) * (size_t)G.n, s));
+        launch_set_u32(vals, src, 0u, s);
+    }
+    CK(cudaMemcpyAsync(ws->dist_old, vals, sizeof(uint32_t) * (size_t)G.n, cudaMemcpyDeviceToDevice, s));
+    sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
+    TRY(clear_frontier(in, s));
+    TRY(clear_frontier(out, s));
+    CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), s));
+    if (cc) launch_fill_all(in->bits, in->summ, G.n, G.nw1, G.nw2, s);   // advance::vertices
+    else launch_seed(in->bits, in->summ, nullptr, src, s);
+    TRY(compact(g, in, cc, s));          // identical on every rank (replicated input)
+    launch_xbarrier(A->x, s);            // every rank initialised before any peer writes into it
+    TRY(read_stats(ws, s));
+    int64_t iters = 0, push_steps = 0, pull_steps = 0, arcs_pushed = 0, arcs_pulled = 0;
+    int in_idx = 0;
+    for (;;) {
+        const int64_t count = (int64_t)ws->h_st[in_idx].count;
+        if (count == 0) break;
+        if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
+        const bool pull = cc && (o.direction == SG_DIR_PULL ||
+                                 (o.direction == SG_DIR_AUTO && (double)ws->h_st[in_idx].mf * 4.0 > (double)g->nnz_global));
+        if (pull && cc_nb > 1) {
+            for (int b = 0; b < cc_nb; b++)
+                launch_pull_cc_block(g->vl, reinterpret_cast<int32_t *>(vals), out->bits, in->st, g->cbo, cc_nb, b, s);
+        } else if (pull) {
+            launch_pull_cc(g->vl, reinterpret_cast<int32_t *>(vals), out->bits, out->summ, in->st, s);
+        } else {
+            const PushLaunch L = push_launch(g, in, t, count);
+            if (cc) {
+                launch_push_cc(L, CcArgs{reinterpret_cast<int32_t *>(vals), nullptr, nullptr}, s);
+            } else {
+                SsspArgs sa{vals, nullptr, nullptr};
+                sa.diff = 1;
+                launch_push_sssp(L, sa, s);
+            }
+        }
+        (pull ? pull_steps : push_steps)++;
+        BfsOut bo{};
+        bo.out_bits = out->bits;
+        bo.out_summ = out->summ;
+        bo.out_offsets = out->offsets;
+        bo.st = out->st;
+        bo.prev = in->st;      // zeroed by the last CTA before it publishes (the next output)
+        bo.done = ws->bfs_done;
+        bo.x = A->x;
+        launch_value_diff(G, vals, ws->dist_old, bo, cc ? 1 : 0, s);
+        TRY(read_stats(ws, s));
+        (pull ? arcs_pulled : arcs_pushed) += (int64_t)ws->h_st[in_idx ^ 1].pad;   // global arcs of the step
+        std::swap(in, out);
+        in_idx ^= 1;
+        iters++;
+    }
+    CK(cudaMemcpyAsync(result, vals, sizeof(uint32_t) * (size_t)G.n, cudaMemcpyDeviceToDevice, s));
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    TRY(check_peers(g));
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->iterations = iters;
+        stats->push_steps = push_steps;
+        stats->pull_steps = pull_steps;
+        stats->arcs_pushed = arcs_pushed;
+        stats->arcs_pulled = arcs_pulled;
+        stats->reached = cc ? G.n : -1;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
+extern "C" {
+
 // ---- SSSP (frontier Bellman-Ford) --------------------------------------------------
 SG_API int run_sssp(const sg_graph *gc, int32_t src, uint32_t *dist, const sg_opts *opts, sg_stats *stats) {
     t_err.clear();
@@ -1181,6 +1615,10 @@ SG_API int run_sssp(const sg_graph *gc, int32_t src, uint32_t *dist, const sg_op
     const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
     cudaStream_t s = stream_of(&o);
     TRY(ensure_ws(g));
+    if (g->ar) {
+        if (o.sssp_delta > 0) return fail(SG_ERR_UNSUPPORTED, "delta-stepping runs on single-GPU graphs only");
+        return run_value_part(g, false, src, dist, o, stats);
+    }
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
@@ -1291,6 +1729,7 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
     cudaStream_t s = stream_of(&o);
     TRY(ensure_ws(g));
+    if (g->ar) return run_value_part(g, true, 0, reinterpret_cast<uint32_t *>(label), o, stats);
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
@@ -1468,6 +1907,7 @@ SG_API int run_bc(const sg_graph *gc, const int32_t *sources, int32_t k, double 
                   sg_stats *stats) {
     t_err.clear();
     if (!gc || !bc || (k > 0 && !sources) || k < 0) return fail(SG_ERR_INVALID, "bad run_bc arguments");
+    if (gc->ar) return fail(SG_ERR_UNSUPPORTED, "BC shards sources over full replicas (SURVEY 8(e)), not a partitioned graph");
     sg_graph *g = const_cast<sg_graph *>(gc);
     const GraphView &G = g->v;
     for (int32_t i = 0; i < k; i++)

@@ -11,6 +11,30 @@ namespace sg {
 constexpr uint32_t INF32 = 0xFFFFFFFFu;
 constexpr int WARP = 32;
 
+// ---- 1-D destination partition over peer memory (xchg.cuh, comm.cu) ----------
+constexpr int SG_MAX_RANKS = 8;
+// One rank's contribution to a superstep's statistics, published into every peer's control
+// block (double-buffered by epoch parity).
+struct XSlot {
+    unsigned long long epoch;   // barrier number this slot belongs to (written last, release)
+    unsigned long long nf, mf, arcs;
+};
+// Exchange control block: lives at the start of each rank's IPC-shared arena.
+struct XCtl {
+    unsigned long long epoch;   // barriers passed by this rank (local)
+    unsigned long long error;   // a peer did not arrive within the timeout (host reports SG_ERR_NCCL)
+    unsigned long long pad[6];
+    XSlot slots[2][SG_MAX_RANKS];
+};
+// Kernel-visible exchange descriptor (by value).  nranks <= 1: single GPU, every helper is local.
+// Every rank's arena has the same layout, so the peer copy of a local arena pointer p is
+// p + delta[j] (bytes; delta[rank] = 0).
+struct Xchg {
+    int32_t nranks = 0, rank = 0;
+    long long delta[SG_MAX_RANKS] = {};
+    XCtl *ctl = nullptr;
+};
+
 // Graph as the kernels see it (device pointers).
 struct GraphView {
     const int64_t *__restrict__ rp;    // row_ptr[n+1]
@@ -23,6 +47,11 @@ struct GraphView {
     const int32_t *__restrict__ hub_idx;   // hub index of u (deg >= SEG_MIN) or -1; nullptr: no segmentation
     const uint32_t *__restrict__ hub_off;  // [nhubs][nseg+1] neighbours of the hub with id < b*SEG_V
     int32_t nseg;                          // ceil(n / SEG_V)
+    // owned destination range (1-D partition); single GPU: everything.  Ranges are
+    // 4,096-vertex aligned (except hi = n), so owned layer-1 and layer-2 words are whole.
+    int64_t own_lo = 0, own_hi = 0;        // vertices
+    int64_t w1_lo = 0, w1_hi = 0;          // layer-1 words
+    int64_t w2_lo = 0, w2_hi = 0;          // layer-2 words
 };
 
 // Destination-segmented copy of the arcs (scsr.cu): segment b = vertices [b*sv, (b+1)*sv), sv =

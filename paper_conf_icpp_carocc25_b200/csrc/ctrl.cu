@@ -10,6 +10,7 @@
 #include "common.cuh"
 #include "kernels.h"
 #include "bfsstep.cuh"
+#include "xchg.cuh"
 
 namespace sg {
 
@@ -58,7 +59,7 @@ __global__ void k_zero_u64(unsigned long long *p, int64_t n) {
 __global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                                uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
                                unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
-                               unsigned long long h_sweep) {
+                               unsigned long long h_sweep, Xchg x) {
     uint32_t *level = c->level;
     const int32_t src = c->src;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -83,19 +84,44 @@ __global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint6
         st->count = 1ull;
         st->nf = 1ull;
         st->mf = deg8_decode(deg8[src]);
-        bfs_decide(c, st, nullptr, h_loop, h_push, h_pull, h_sweep, 1);
+        if (x.nranks > 1) xbarrier(x, 0ull, 0ull, 0ull, nullptr);   // every rank's prologue memsets done
+        bfs_decide(c, st, 0ull, nullptr, h_loop, h_push, h_pull, h_sweep, 1);
     }
 }
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                          uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
                          unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
-                         unsigned long long h_sweep, cudaStream_t s) {
+                         unsigned long long h_sweep, const Xchg &x, cudaStream_t s) {
     int64_t blocks = (n / 4 + 255) / 256;
     if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_bfs_prologue<<<(int)blocks, 256, 0, s>>>(c, n, deg8, bits, summ, offsets, st, visited, vis_old, h_loop, h_push,
-                                               h_pull, h_sweep);
+                                               h_pull, h_sweep, x);
+}
+
+// Barrier across the ranks of a partition (one thread; xchg.cuh)
+__global__ void k_xbarrier(Xchg x) { xbarrier(x, 0ull, 0ull, 0ull, nullptr); }
+void launch_xbarrier(const Xchg &x, cudaStream_t s) {
+    if (x.nranks <= 1) return;
+    note_launch();
+    k_xbarrier<<<1, 1, 0, s>>>(x);
+}
+// The owned slice [lo, hi) of `src` into every rank's replica `vals` (own included): the result
+// gather of a partitioned BFS (level), 16-B stores when aligned
+__global__ void k_publish_owned(const uint32_t *__restrict__ src, uint32_t *vals, int64_t lo, int64_t hi, Xchg x) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = lo + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < hi; v += stride) {
+        const uint32_t a = src[v];
+        for (int j = 0; j < x.nranks; j++) *xpeer(x, vals + v, j) = a;
+    }
+}
+void launch_publish_owned(const uint32_t *src, uint32_t *vals, int64_t lo, int64_t hi, const Xchg &x, cudaStream_t s) {
+    int64_t blocks = (hi - lo + 255) / 256;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_publish_owned<<<(int)blocks, 256, 0, s>>>(src, vals, lo, hi, x);
 }
 
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,

@@ -419,7 +419,7 @@ constexpr int DIFF_THREADS = 256;
 __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited, BfsOut o) {
     __shared__ uint64_t s_S[DIFF_THREADS / 64];
     __shared__ uint32_t s_ch[DIFF_THREADS / 32];
-    __shared__ uint32_t s_base, s_lut[256];
+    __shared__ uint32_t s_base[1 + SG_MAX_RANKS], s_lut[256];
     deg8_lut_init(s_lut);   // visible after the loop's first __syncthreads
     const int lane = lane_id(), wid = threadIdx.x >> 5;
     const int half = lane >> 4;
@@ -427,24 +427,27 @@ __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const ui
     unsigned long long nf = 0, mf = 0;
     uint32_t *lvl = nullptr;
     uint32_t nx = 0;
-    for (int64_t base = blockIdx.x * (int64_t)DIFF_THREADS; base < g.nw1; base += (int64_t)gridDim.x * DIFF_THREADS) {
+    // owned layer-1 words only (partitioned: w1_lo is a multiple of 64, so CTA slices start on
+    // layer-2 word boundaries); every output word is also stored into the peers' replicas
+    for (int64_t base = g.w1_lo + blockIdx.x * (int64_t)DIFF_THREADS; base < g.w1_hi;
+         base += (int64_t)gridDim.x * DIFF_THREADS) {
         const int64_t w0 = base + wid * 32;
         const int64_t wa = w0 + lane;
         uint64_t na = 0, oa = 0;
-        if (wa < g.nw1) {
+        if (wa < g.w1_hi) {
             na = visited[wa];
             oa = o.vis_old[wa];
         }
         const uint64_t da = na & ~oa;
         uint32_t ch = __ballot_sync(0xffffffffu, da != 0);
         if (lane == 0) s_ch[wid] = ch;
-        if (wa < g.nw1) o.out_bits[wa] = da;
+        if (wa < g.w1_hi) xstore(o.x, o.out_bits + wa, da);
         if (da) o.vis_old[wa] = na;
         __syncthreads();
         if (threadIdx.x < DIFF_THREADS / 64)
             s_S[threadIdx.x] = (uint64_t)s_ch[2 * threadIdx.x] | ((uint64_t)s_ch[2 * threadIdx.x + 1] << 32);
         __syncthreads();
-        bfs_emit_words(o, g.nw2, base >> 6, s_S, DIFF_THREADS / 64, &s_base);
+        bfs_emit_words(o, g.w2_hi, base >> 6, s_S, DIFF_THREADS / 64, s_base);
         if (ch && !lvl) {
             lvl = o.level_pp ? *o.level_pp : o.level;
             nx = o.next_ptr ? *o.next_ptr : o.next;
@@ -491,24 +494,31 @@ __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const ui
     bfs_finish(o, nf, mf, 0ull, nullptr);
 }
 void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s) {
-    int64_t blocks = (g.nw1 + DIFF_THREADS - 1) / DIFF_THREADS;   // 256 layer-1 words per CTA
+    int64_t blocks = (g.w1_hi - g.w1_lo + DIFF_THREADS - 1) / DIFF_THREADS;   // 256 layer-1 words per CTA
     if (blocks > SG_DIFF_BLOCKS) blocks = SG_DIFF_BLOCKS;
     if (blocks < 1) blocks = 1;
     note_launch();
     k_bfs_diff<<<(int)blocks, DIFF_THREADS, 0, s>>>(g, visited, o);
 }
-// Output of a diff-mode SSSP superstep (FnSssp::diff): the vertices whose distance decreased.
-// A CTA of 256 threads takes 64 layer-1 words (4,096 vertices, one layer-2 word): a thread
-// compares 4 x 4 distances (16-B loads of dist and dist_old), the half-warp ORs the word's
-// bits, every output word is written, and the CTA emits its layer-2 word and word list.
-__global__ void __launch_bounds__(256) k_sssp_diff(GraphView g, const uint32_t *__restrict__ dist,
-                                                   uint32_t *__restrict__ dist_old, BfsOut o) {
+// Output of a diff-mode SSSP / CC superstep (FnSssp::diff; CC pulls and pushes in place): the
+// vertices whose value decreased (value < old, unsigned; CC labels are >= 0).  A CTA of 256
+// threads takes 64 layer-1 words (4,096 vertices, one layer-2 word): a thread compares 4 x 4
+// values (16-B loads of value and old), the half-warp ORs the word's bits, every output word is
+// written, and the CTA emits its layer-2 word and word list; n_f (and m_f from the degree codes
+// when want_mf, CC's direction policy) go to o.st.  Partitioned (xchg.cuh): owned layer-2 words
+// only; the changed quads' new values and the output words are stored into every peer's replica
+// (a value that did not change needs no exchange: peers already hold it), and the last CTA runs
+// the superstep barrier.
+__global__ void __launch_bounds__(256) k_value_diff(GraphView g, uint32_t *__restrict__ dist,
+                                                    uint32_t *__restrict__ dist_old, BfsOut o, int want_mf) {
     __shared__ uint64_t s_S[1];
-    __shared__ uint32_t s_base;
+    __shared__ uint32_t s_base[1 + SG_MAX_RANKS], s_lut[256];
+    deg8_lut_init(s_lut);
     const int lane = lane_id();
     const uint32_t half = (lane < 16) ? 0x0000ffffu : 0xffff0000u;
     const bool vec = (((uintptr_t)dist | (uintptr_t)dist_old) & 15) == 0;
-    for (int64_t sw = blockIdx.x; sw < g.nw2; sw += gridDim.x) {
+    unsigned long long nf = 0, mf = 0;
+    for (int64_t sw = g.w2_lo + blockIdx.x; sw < g.w2_hi; sw += gridDim.x) {
         if (threadIdx.x == 0) s_S[0] = 0ull;
         __syncthreads();
 #pragma unroll 1
@@ -517,13 +527,18 @@ __global__ void __launch_bounds__(256) k_sssp_diff(GraphView g, const uint32_t *
             const int64_t w = qd >> 4;
             const int sh = (int)(qd & 15) * 4;
             uint32_t m = 0;
-            if (w < g.nw1) {
+            if (w < g.w1_hi) {
                 const int64_t v0 = w * 64 + sh;
                 if (vec && v0 + 4 <= g.n) {
                     const uint4 a = *reinterpret_cast<const uint4 *>(dist + v0);
                     const uint4 b = *reinterpret_cast<const uint4 *>(dist_old + v0);
                     m = (a.x < b.x ? 1u : 0u) | (a.y < b.y ? 2u : 0u) | (a.z < b.z ? 4u : 0u) | (a.w < b.w ? 8u : 0u);
-                    if (m) *reinterpret_cast<uint4 *>(dist_old + v0) = a;
+                    if (m) {
+                        *reinterpret_cast<uint4 *>(dist_old + v0) = a;
+                        if (o.x.nranks > 1)
+                            for (int j = 0; j < o.x.nranks; j++)
+                                if (j != o.x.rank) *reinterpret_cast<uint4 *>(xpeer(o.x, dist + v0, j)) = a;
+                    }
                 } else {
                     for (int k = 0; k < 4; k++) {
                         if (v0 + k >= g.n) break;
@@ -531,21 +546,37 @@ __global__ void __launch_bounds__(256) k_sssp_diff(GraphView g, const uint32_t *
                         if (a < dist_old[v0 + k]) {
                             m |= 1u << k;
                             dist_old[v0 + k] = a;
+                            if (o.x.nranks > 1)
+                                for (int j = 0; j < o.x.nranks; j++)
+                                    if (j != o.x.rank) *xpeer(o.x, dist + v0 + k, j) = a;
                         }
                     }
+                }
+                if (m) {
+                    nf += __popc(m);
+                    if (want_mf) mf += quad_mf(s_lut, __ldg(reinterpret_cast<const uint32_t *>(g.deg8 + v0)), m);
                 }
             }
             const uint64_t mine = (uint64_t)m << sh;
             const uint64_t nb = (uint64_t)__reduce_or_sync(half, (uint32_t)mine) |
                                 ((uint64_t)__reduce_or_sync(half, (uint32_t)(mine >> 32)) << 32);
-            if ((lane & 15) == 0 && w < g.nw1) {
-                o.out_bits[w] = nb;
+            if ((lane & 15) == 0 && w < g.w1_hi) {
+                xstore(o.x, o.out_bits + w, nb);
                 if (nb) atomicOr(reinterpret_cast<unsigned long long *>(s_S), 1ull << (w & 63));
             }
         }
         __syncthreads();
-        bfs_emit_words(o, g.nw2, sw, s_S, 1, &s_base);
+        bfs_emit_words(o, g.w2_hi, sw, s_S, 1, s_base);
     }
+    bfs_finish(o, nf, mf, 0ull, nullptr);
+}
+void launch_value_diff(const GraphView &g, uint32_t *value, uint32_t *old, const BfsOut &o, int want_mf,
+                       cudaStream_t s) {
+    int64_t blocks = g.w2_hi - g.w2_lo;
+    if (blocks > num_sms() * 16) blocks = num_sms() * 16;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_value_diff<<<(int)blocks, 256, 0, s>>>(g, value, old, o, want_mf);
 }
 void launch_sssp_diff(const GraphView &g, const uint32_t *dist, uint32_t *dist_old, uint64_t *out_bits,
                       uint64_t *out_summ, uint32_t *out_offsets, DevStats *st, cudaStream_t s) {
@@ -554,11 +585,7 @@ void launch_sssp_diff(const GraphView &g, const uint32_t *dist, uint32_t *dist_o
     o.out_summ = out_summ;
     o.out_offsets = out_offsets;
     o.st = st;
-    int64_t blocks = g.nw2;
-    if (blocks > num_sms() * 16) blocks = num_sms() * 16;
-    if (blocks < 1) blocks = 1;
-    note_launch();
-    k_sssp_diff<<<(int)blocks, 256, 0, s>>>(g, dist, dist_old, o);
+    launch_value_diff(g, const_cast<uint32_t *>(dist), dist_old, o, 0, s);
 }
 void launch_iota_i32(int32_t *p, int64_t n, cudaStream_t s) { note_launch(); k_iota_i32<<<grid_for(n, 256, num_sms() * 8), 256, 0, s>>>(p, n); }
 void launch_validate_csr(const GraphView &g, unsigned long long *bad, cudaStream_t s) {

@@ -100,6 +100,7 @@ struct BfsOut {
     DevStats *prev;
     unsigned int *done;               // CTA completion counter (self-resetting)
     unsigned long long h_loop, h_push, h_pull, h_sweep;
+    Xchg x;                           // partitioned: peers' replicas of the output (xchg.cuh)
 };
 // pull.cu — bottom-up BFS step (direction-optimising, Beamer): writes its output `o`
 // itself (no k_bfs_diff after it); o.out_bits == NULL: marks visited only (k_bfs_diff after it)
@@ -113,6 +114,11 @@ void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &
 // dist_old = dist
 void launch_sssp_diff(const GraphView &g, const uint32_t *dist, uint32_t *dist_old, uint64_t *out_bits,
                       uint64_t *out_summ, uint32_t *out_offsets, DevStats *st, cudaStream_t s);
+// the general form (SSSP dist / CC labels): output o (out_bits / out_summ / out_offsets / st,
+// prev = the input's control block, x = peers), n_f (+ m_f when want_mf) into o.st; partitioned:
+// owned words only, changed values + output replicated to the peers, superstep barrier at the end
+void launch_value_diff(const GraphView &g, uint32_t *value, uint32_t *old, const BfsOut &o, int want_mf,
+                       cudaStream_t s);
 
 // filter.cu — filter::inplace / external, compute::execute (Table 2)
 void launch_filter(const GraphView &g, const uint64_t *in_bits, uint64_t *out_bits, uint64_t *out_summ, int pred,
@@ -157,10 +163,24 @@ void launch_push_sweep(const ScsrView &v, const int64_t *rp, const uint64_t *in_
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                          uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
                          unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
-                         unsigned long long h_sweep, cudaStream_t s);
+                         unsigned long long h_sweep, const Xchg &x, cudaStream_t s);
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s);
 void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s);
+// partition (xchg.cuh): barrier across ranks (one thread); owned slice [lo, hi) of src into
+// every rank's replica vals
+void launch_xbarrier(const Xchg &x, cudaStream_t s);
+void launch_publish_owned(const uint32_t *src, uint32_t *vals, int64_t lo, int64_t hi, const Xchg &x, cudaStream_t s);
+
+// partition.cu — graph-load side of the 1-D destination partition
+// h_out[r-1] = first vertex whose row starts at or after nnz*r/P (r = 1..P-1); synchronises s
+cudaError_t part_quantiles(const int64_t *rp, int64_t n, int64_t nnz, int P, int64_t *h_out, cudaStream_t s);
+// push block: the arcs of every row into [lo, hi) (CSR over all n rows; +64 B padding)
+cudaError_t part_push_block(const int64_t *rp, const int32_t *col, const uint8_t *w, int64_t n, int64_t lo, int64_t hi,
+                            int64_t **rpp, int32_t **colp, uint8_t **wp, int64_t *nnz, cudaStream_t s);
+// pull block: rows [lo, hi) (CSR over all n rows, rows outside empty)
+cudaError_t part_pull_block(const int64_t *rp, const int32_t *col, int64_t n, int64_t lo, int64_t hi, int64_t **rpl,
+                            int32_t **coll, int64_t *nnz, cudaStream_t s);
 void launch_list_all(uint32_t *offsets, DevStats *st_all, const DevStats *st_src, int64_t nw1, cudaStream_t s);
 
 // bcb.cu — source-batched BC (32 sources per batch): init, cooperative forward and backward

@@ -94,7 +94,7 @@ __global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
            BfsOut o) {
     __shared__ uint64_t s_wm[PULL_THREADS / 32], s_S[1];
-    __shared__ uint32_t s_base, s_lut[256];
+    __shared__ uint32_t s_base[1 + SG_MAX_RANKS], s_lut[256];
 #if SG_PULL_WSKIP
     __shared__ uint32_t s_full[2][2], s_mx[2][2];   // double-buffered by iteration parity (no barrier at reuse)
     int par = 0;
@@ -114,7 +114,8 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
 #if SG_PULL_PF
     uint64_t vis_next = vis_at((int64_t)blockIdx.x * 1024 + threadIdx.x);
 #endif
-    for (int64_t sw = blockIdx.x; sw < g.nw2; sw += gridDim.x) {
+    // owned layer-2 words only (1-D partition; single GPU: all of them)
+    for (int64_t sw = g.w2_lo + blockIdx.x; sw < g.w2_hi; sw += gridDim.x) {
         uint64_t wm = 0;   // the warp's changed words within the layer-2 word
 #if SG_PULL_WSKIP
         // bit i of `full`: layer-1 word sw*64+i has no unvisited vertex (or lies past the end).
@@ -141,8 +142,8 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
         const uint32_t mxw = max(s_mx[par][0], s_mx[par][1]);
         par ^= 1;
         if (full == ~0ull) {
-            if (threadIdx.x < 64 && sw * 64 + threadIdx.x < g.nw1) o.out_bits[sw * 64 + threadIdx.x] = 0ull;
-            if (threadIdx.x == 0) o.out_summ[sw] = 0ull;
+            if (threadIdx.x < 64 && sw * 64 + threadIdx.x < g.nw1) xstore(o.x, o.out_bits + sw * 64 + threadIdx.x, 0ull);
+            if (threadIdx.x == 0) xstore(o.x, o.out_summ + sw, 0ull);
             continue;
         }
 #if SG_PULL_WORD_MAX > 0
@@ -181,7 +182,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                     }
                 }
                 if (w < g.nw1) {
-                    o.out_bits[w] = nbw;
+                    xstore(o.x, o.out_bits + w, nbw);
                     if (nbw) {
                         visited[w] = my_vis | nbw;
                         o.vis_old[w] = my_vis | nbw;
@@ -199,7 +200,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             __syncthreads();
             if (threadIdx.x == 0) s_S[0] = s_wm[0] | (s_wm[1] << 32);
             __syncthreads();
-            bfs_emit_words(o, g.nw2, sw, s_S, 1, &s_base);
+            bfs_emit_words(o, g.w2_hi, sw, s_S, 1, s_base);
             continue;
         }
 #endif
@@ -211,7 +212,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             const int64_t w = qd >> 4;
 #if SG_PULL_WSKIP
             if (((full >> (r * (PULL_THREADS / 16) + wid * 2)) & 3ull) == 3ull) {
-                if ((lane & 15) == 0 && ok) o.out_bits[w] = 0ull;
+                if ((lane & 15) == 0 && ok) xstore(o.x, o.out_bits + w, 0ull);
                 continue;
             }
 #endif
@@ -227,7 +228,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             const uint32_t valid = !ok ? 0u : rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
             const uint32_t unv = (uint32_t)(~vis >> sh) & valid;
             if (__all_sync(0xffffffffu, unv == 0u)) {   // the warp's two words are fully visited:
-                if ((lane & 15) == 0 && ok) o.out_bits[w] = 0ull;   // no new vertices, no work
+                if ((lane & 15) == 0 && ok) xstore(o.x, o.out_bits + w, 0ull);   // no new vertices, no work
                 continue;
             }
             uint32_t found = 0, codes = 0;
@@ -269,7 +270,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                     if ((t >> (16 * i)) & 1u) lw[16 * i] = nx;
             }
             if ((lane & 15) == 0 && ok) {
-                o.out_bits[w] = nb;   // every output word is written
+                xstore(o.x, o.out_bits + w, nb);   // every output word is written
                 if (nb) {
                     visited[w] = vis | nb;
                     o.vis_old[w] = vis | nb;
@@ -286,7 +287,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             s_S[0] = S;
         }
         __syncthreads();
-        bfs_emit_words(o, g.nw2, sw, s_S, 1, &s_base);
+        bfs_emit_words(o, g.w2_hi, sw, s_S, 1, s_base);
     }
     bfs_finish(o, nf, mf, arcs, st);
 }
@@ -294,7 +295,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,
                      cudaStream_t s) {
     // one CTA per layer-2 word in a grid-stride loop over SG_PULL_WAVES CTAs per SM
-    int64_t blocks = g.nw2;
+    int64_t blocks = g.w2_hi - g.w2_lo;
     if (blocks > num_sms() * SG_PULL_WAVES) blocks = num_sms() * SG_PULL_WAVES;
     if (blocks < 1) blocks = 1;
     note_launch();

@@ -56,7 +56,7 @@ k_pull_cc(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__ out_b
 #if SG_CC_HINTS & 2
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_last));
 #endif
-    for (int64_t w = gw; w < g.nw1; w += nwarps) {
+    for (int64_t w = g.w1_lo + gw; w < g.w1_hi; w += nwarps) {   // owned words (1-D partition)
         const int64_t rem = g.n - w * 64;
         const uint64_t valid = rem >= 64 ? ~0ull : ((1ull << rem) - 1ull);
         int64_t sa, ea, sb, eb;
@@ -156,7 +156,7 @@ k_pull_cc_block(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__
         s0 = b == 0 ? r0 : r0 + __ldg(cbo + v * (nb - 1) + (b - 1));
         e0 = b == nb - 1 ? r1 : r0 + __ldg(cbo + v * (nb - 1) + b);
     };
-    for (int64_t w = gw; w < g.nw1; w += nwarps) {
+    for (int64_t w = g.w1_lo + gw; w < g.w1_hi; w += nwarps) {   // owned words (1-D partition)
         const int64_t va = w * 64 + lane, vb = va + 32;
         const bool act_a = va < g.n, act_b = vb < g.n;
         int64_t sa = 0, ea = 0, sb = 0, eb = 0;
@@ -201,7 +201,7 @@ k_pull_cc_block(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__
 }
 void launch_pull_cc_block(const GraphView &g, int32_t *label, uint64_t *out_bits, DevStats *st, const uint32_t *cbo,
                           int nb, int b, cudaStream_t s) {
-    int64_t blocks = (g.nw1 * 32 + CCP_THREADS - 1) / CCP_THREADS;
+    int64_t blocks = ((g.w1_hi - g.w1_lo) * 32 + CCP_THREADS - 1) / CCP_THREADS;
     if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
     note_launch();
@@ -210,7 +210,7 @@ void launch_pull_cc_block(const GraphView &g, int32_t *label, uint64_t *out_bits
 
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,
                     cudaStream_t s) {
-    int64_t blocks = (g.nw1 * 32 + CCP_THREADS - 1) / CCP_THREADS;
+    int64_t blocks = ((g.w1_hi - g.w1_lo) * 32 + CCP_THREADS - 1) / CCP_THREADS;
     if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
     note_launch();

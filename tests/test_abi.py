@@ -65,6 +65,51 @@ def test_error_paths_without_gpu():
     import paper_conf_icpp_carocc25_b200 as sg
     L = sg.load()
     h = ctypes.c_void_p()
-    assert L.graph_load_csr(0, 0, None, None, None, 0, 0, None, ctypes.byref(h)) == sg.SG_ERR_INVALID
+    assert L.graph_load_csr(0, 0, None, None, None, 0, 0, None, None, ctypes.byref(h)) == sg.SG_ERR_INVALID
     assert b"outside" in L.sg_last_error()
     assert L.run_bfs(None, 0, None, None, None) == sg.SG_ERR_INVALID
+
+
+def _comm_worker(rank, world, q_id, q_out):
+    import paper_conf_icpp_carocc25_b200 as sg
+    if rank == 0:
+        uid = sg.comm_unique_id()
+        for _ in range(world - 1):
+            q_id.put(uid)
+    else:
+        uid = q_id.get(timeout=60)
+    c = sg.comm_init(uid, world, rank, 0)
+    import ctypes
+    nr, rk = ctypes.c_int(), ctypes.c_int()
+    assert sg.load().comm_info(c.handle, ctypes.byref(nr), ctypes.byref(rk)) == 0
+    q_out.put((rank, nr.value, rk.value))
+    c.free()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_comm_bootstrap_multiprocess(world):
+    """The partition communicator's TCP bootstrap (comm_unique_id / comm_init, no GPU needed):
+    world processes join through rank 0's id; each sees (nranks, rank)."""
+    import multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q_id, q_out = ctx.Queue(), ctx.Queue()
+    ps = [ctx.Process(target=_comm_worker, args=(r, world, q_id, q_out)) for r in range(world)]
+    for p in ps:
+        p.start()
+    got = sorted(q_out.get(timeout=120) for _ in range(world))
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert got == [(r, world, r) for r in range(world)]
+
+
+def test_comm_rejects_bad_arguments():
+    import paper_conf_icpp_carocc25_b200 as sg
+    with pytest.raises(sg.SgError) as e:
+        sg.comm_init(b"\0" * 128, 2, 1, 0)          # not an id made by comm_unique_id
+    assert e.value.code == sg.SG_ERR_NCCL
+    with pytest.raises(sg.SgError) as e:
+        sg.comm_init(sg.comm_unique_id(), 9, 0, 0)   # more ranks than SG_MAX_RANKS
+    assert e.value.code == sg.SG_ERR_INVALID
+    c = sg.comm_init(b"\0" * 128, 1, 0, 0)           # a single rank needs no bootstrap
+    c.free()

@@ -1,6 +1,13 @@
-"""The 1-D partitioned BFS on one GPU: P simulated ranks, each a push block loaded through the
-C ABI, advanced with the real kernels over the replicated frontier; the all-gather is emulated
-by OR-ing the disjoint owned slices (what ncclAllGather delivers).  Must equal the oracle."""
+"""The 1-D destination partition end to end on the GPU: world = 2 or 3 processes (ranks) share
+this box's one B200, each with its own CUDA context, a communicator (comm_unique_id / comm_init)
+and its partition of the graph (graph_load_csr(..., comm)).  Every superstep runs the real
+kernels and the real exchange: the output kernels store each rank's owned slice into its peers'
+replicas through CUDA IPC peer memory and meet at the in-kernel superstep barrier (xchg.cuh) —
+the same code path as one rank per GPU over NVLink, where time-slicing of the shared GPU is the
+only difference.  Results must equal the oracle; statistics must equal the single-GPU run's
+(every rank takes the same direction decisions from the global sums)."""
+import os
+
 import numpy as np
 import pytest
 
@@ -11,136 +18,107 @@ pytestmark = pytest.mark.gpu
 INF = 0xFFFFFFFF
 
 
-@pytest.mark.parametrize("P", [1, 2, 3, 4])
-def test_partitioned_bfs_equals_oracle(P):
+def _check(name, ok, errs):
+    if not ok:
+        errs.append(name)
+
+
+def _worker(rank, world, q_id, q_out, case):
     import torch
     import paper_conf_icpp_carocc25_b200 as sg
-    from paper_conf_icpp_carocc25_b200.partition import partition_ranges, push_block
-
-    g = gen.rmat(15, 16, permute=True)
-    s = int(gen.sources(g, 1)[0])
-    ranges = partition_ranges(g.row_ptr, P)
-    ranks = []
-    for lo, hi in ranges:
-        rp, ci, _ = push_block(g.row_ptr, g.col_idx, None, lo, hi)
-        G = sg.graph_load_csr(rp, ci)
-        fi, fo = sg.frontier_init(G), sg.frontier_init(G)
-        sg.frontier_insert(fi, np.array([s], np.int32))
-        ranks.append(dict(G=G, fi=fi, fo=fo, lo=lo, hi=hi,
-                          level=torch.full((g.n,), -1, dtype=torch.int32, device="cuda"),
-                          visited=torch.zeros((g.n + 63) // 64, dtype=torch.int64, device="cuda")))
-    bit = 1 << (s & 63)
-    for r in ranks:
-        r["visited"][s >> 6] = bit - (1 << 64) if bit >= 1 << 63 else bit
-        if r["lo"] <= s < r["hi"]:
-            r["level"][s] = 0
-    depth = 0
-    while True:
-        for r in ranks:
-            sg.advance(r["G"], r["fi"], r["fo"], sg.SG_FN_BFS, dict(level=r["level"], visited=r["visited"], depth=depth))
-        views = [sg.frontier_view(r["fo"]) for r in ranks]
-        bits = views[0][0].view(torch.int64).clone()
-        summ = views[0][1].view(torch.int64).clone()
-        for b, sm in views[1:]:
-            bits |= b.view(torch.int64)
-            summ |= sm.view(torch.int64)
-        for (b, sm), r in zip(views, ranks):           # "all-gather": every rank sees every slice
-            b.view(torch.int64).copy_(bits)
-            sm.view(torch.int64).copy_(summ)
-            sg.frontier_or_into(r["fo"], r["visited"])
-        if int(torch.count_nonzero(bits)) == 0:
-            break
-        depth += 1
-        for r in ranks:
-            sg.frontier_clear(r["fi"])
-            r["fi"], r["fo"] = r["fo"], r["fi"]
-    level = np.full(g.n, INF, np.uint32)
-    for r in ranks:
-        lv = sg.as_u32(r["level"])
-        level[r["lo"]:r["hi"]] = lv[r["lo"]:r["hi"]]
-    assert np.array_equal(level, oracle.bfs(g, s))
-
-
-def test_dist_bfs_world1():
-    """The production driver (partition.dist_bfs) at world size 1 through the C ABI."""
-    import torch
-    import paper_conf_icpp_carocc25_b200 as sg
-    from paper_conf_icpp_carocc25_b200.partition import DistGraph, SliceExchange, dist_bfs
-
-    g = gen.rmat(14, 16, permute=True)
-    dg = DistGraph(g.row_ptr, g.col_idx, None, 0, 1)
-    ex = SliceExchange(dg.layout, 0, 1, torch.device("cuda"))
-    for s in gen.sources(g, 3):
-        lv = dist_bfs(dg, int(s), ex)
-        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s)))
-
-
-def test_dist_sssp_and_cc_world1():
-    """The production SSSP / CC drivers (partition.dist_sssp / dist_cc) at world size 1."""
-    import torch
-    import paper_conf_icpp_carocc25_b200 as sg
-    from paper_conf_icpp_carocc25_b200.partition import DistGraph, SliceExchange, dist_cc, dist_sssp
-
-    g = gen.with_weights(gen.rmat(14, 16, permute=True), seed=5)
-    dg = DistGraph(g.row_ptr, g.col_idx, g.weights, 0, 1)
-    ex = SliceExchange(dg.layout, 0, 1, torch.device("cuda"))
-    for s in gen.sources(g, 3):
-        d = dist_sssp(dg, int(s), ex)
-        assert np.array_equal(sg.as_u32(d), oracle.sssp(g, int(s)))
-    lab = dist_cc(dg, ex)
-    assert np.array_equal(lab.cpu().numpy(), oracle.cc(g))
+    from paper_conf_icpp_carocc25_b200.partition import partition_ranges
+    torch.cuda.set_device(0)
+    errs = []
+    try:
+        if rank == 0:
+            uid = sg.comm_unique_id()
+            for _ in range(world - 1):
+                q_id.put(uid)
+        else:
+            uid = q_id.get(timeout=120)
+        comm = sg.comm_init(uid, world, rank, 0)
+        if case == "bfs":
+            g = gen.rmat(14, 16, permute=True)
+            G = sg.graph_load_csr(g.row_ptr, g.col_idx, comm=comm)
+            Gs = sg.graph_load_csr(g.row_ptr, g.col_idx)                 # single-GPU reference run
+            lo, hi = sg.graph_partition(G)
+            _check("partition bounds", (lo, hi) == partition_ranges(g.row_ptr, world)[rank], errs)
+            roots = list(gen.sources(g, 3)) + [int(np.argmax(g.degrees()))]
+            for s in roots:
+                ref = oracle.bfs(g, int(s))
+                for d in (sg.SG_DIR_AUTO, sg.SG_DIR_PUSH, sg.SG_DIR_PULL):
+                    lv, st = sg.run_bfs(G, int(s), direction=d)
+                    _check(f"bfs root {s} dir {d}", np.array_equal(sg.as_u32(lv), ref), errs)
+                    _, st1 = sg.run_bfs(Gs, int(s), direction=d)
+                    _check(f"bfs stats root {s} dir {d}",
+                           (st.iterations, st.push_steps, st.pull_steps, st.reached) ==
+                           (st1.iterations, st1.push_steps, st1.pull_steps, st1.reached), errs)
+                lv, _ = sg.run_bfs(G, int(s), owned_only=True)
+                _check(f"bfs owned_only root {s}", np.array_equal(sg.as_u32(lv)[lo:hi], ref[lo:hi]), errs)
+            with pytest.raises(sg.SgError):
+                sg.run_bfs(G, 0, host_loop=True)
+        elif case == "sssp":
+            g = gen.with_weights(gen.rmat(13, 16, permute=True), seed=5)
+            G = sg.graph_load_csr(g.row_ptr, g.col_idx, g.weights, comm=comm)
+            for s in gen.sources(g, 3):
+                d, _ = sg.run_sssp(G, int(s))
+                _check(f"sssp {s}", np.array_equal(sg.as_u32(d), oracle.sssp(g, int(s))), errs)
+        elif case == "cc":
+            for name, g in (("gnm", gen.gnm(60_000, 45_000, seed=3)), ("rmat", gen.rmat(13, 8, permute=True)),
+                            ("lattice", gen.lattice(120, 150, 0.55, seed=2))):
+                G = sg.graph_load_csr(g.row_ptr, g.col_idx, comm=comm)
+                ref = oracle.cc(g)
+                for d in (sg.SG_DIR_AUTO, sg.SG_DIR_PUSH, sg.SG_DIR_PULL):
+                    lab, _ = sg.run_cc(G, direction=d)
+                    _check(f"cc {name} dir {d}", np.array_equal(lab.cpu().numpy(), ref), errs)
+                os.environ["SG_CC_LBLOCK_KB"] = "16"                      # label-blocked pull, several blocks
+                lab, _ = sg.run_cc(G, direction=sg.SG_DIR_PULL)
+                del os.environ["SG_CC_LBLOCK_KB"]
+                _check(f"cc {name} blocked", np.array_equal(lab.cpu().numpy(), ref), errs)
+                G.free()
+        elif case == "tiny":
+            # n = 3000 < 4096: one rank owns every vertex, the others own nothing (empty ranges)
+            g = gen.rmat(11, 8, permute=True)
+            g = gen.from_edges(3000, *[np.asarray(a) for a in _edges_below(g, 3000)])
+            G = sg.graph_load_csr(g.row_ptr, g.col_idx, comm=comm)
+            lo, hi = sg.graph_partition(G)
+            _check("tiny bounds", (lo, hi) == partition_ranges(g.row_ptr, world)[rank], errs)
+            for s in gen.sources(g, 2):
+                lv, _ = sg.run_bfs(G, int(s))
+                _check(f"tiny bfs {s}", np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), errs)
+            lab, _ = sg.run_cc(G)
+            _check("tiny cc", np.array_equal(lab.cpu().numpy(), oracle.cc(g)), errs)
+        torch.cuda.synchronize()
+        q_out.put((rank, errs, None))
+    except Exception as e:   # report instead of hanging the parent
+        import traceback
+        q_out.put((rank, errs, traceback.format_exc()[-1500:]))
 
 
-@pytest.mark.parametrize("P", [2, 3])
-def test_partitioned_sssp_and_cc_equal_oracle(P):
-    """P simulated ranks on one GPU through the real kernels: each rank advances its push block
-    over the replicated frontier and values; the all-gathers are emulated by copying each rank's
-    owned slices into every rank's replicas (what ncclAllGather delivers)."""
-    import torch
-    import paper_conf_icpp_carocc25_b200 as sg
-    from paper_conf_icpp_carocc25_b200.partition import partition_ranges, push_block
+def _edges_below(g, n):
+    rows = np.repeat(np.arange(g.n), g.degrees())
+    keep = (rows < n) & (g.col_idx < n) & (rows < g.col_idx)
+    return rows[keep], g.col_idx[keep].astype(np.int64)
 
-    g = gen.with_weights(gen.rmat(14, 16, permute=True), seed=7)
-    ranges = partition_ranges(g.row_ptr, P)
-    Gs = [sg.graph_load_csr(*push_block(g.row_ptr, g.col_idx, g.weights, lo, hi)) for lo, hi in ranges]
 
-    def run(functor, key, init, seed_frontier):
-        vals = [init() for _ in Gs]
-        fr = [(sg.frontier_init(G), sg.frontier_init(G)) for G in Gs]
-        for fi, _ in fr:
-            seed_frontier(fi)
-        for _ in range(g.n + 1):
-            for G, (fi, fo), v in zip(Gs, fr, vals):
-                sg.advance(G, fi, fo, functor, {key: v})
-            views = [sg.frontier_view(fo) for _, fo in fr]
-            bits = sum_or = views[0][0].view(torch.int64).clone()
-            summ = views[0][1].view(torch.int64).clone()
-            for b, sm in views[1:]:
-                bits |= b.view(torch.int64)
-                summ |= sm.view(torch.int64)
-            full = vals[0].clone()
-            for (lo, hi), v in zip(ranges, vals):
-                full[lo:hi] = v[lo:hi]
-            for (b, sm), v in zip(views, vals):
-                b.view(torch.int64).copy_(bits)
-                sm.view(torch.int64).copy_(summ)
-                v.copy_(full)
-            if int(torch.count_nonzero(sum_or)) == 0:
-                return full
-            for (fi, fo), i in zip(fr, range(len(fr))):
-                sg.frontier_clear(fi)
-                fr[i] = (fo, fi)
-        raise AssertionError("no fixed point")
-
-    s = int(gen.sources(g, 1)[0])
-
-    def init_dist():
-        d = torch.full((g.n,), -1, dtype=torch.int32, device="cuda")
-        d[s] = 0
-        return d
-
-    dist = run(sg.SG_FN_SSSP, "dist", init_dist, lambda f: sg.frontier_insert(f, np.array([s], np.int32)))
-    assert np.array_equal(sg.as_u32(dist), oracle.sssp(g, s))
-    lab = run(sg.SG_FN_CC, "label", lambda: torch.arange(g.n, dtype=torch.int32, device="cuda"),
-              lambda f: sg.frontier_fill_all(f))
-    assert np.array_equal(lab.cpu().numpy(), oracle.cc(g))
+@pytest.mark.parametrize("world,case", [(2, "bfs"), (3, "bfs"), (2, "sssp"), (3, "sssp"), (2, "cc"), (3, "cc"),
+                                        (2, "tiny"), (4, "tiny")])
+def test_partitioned_ranks_on_one_gpu(world, case):
+    import multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q_id, q_out = ctx.Queue(), ctx.Queue()
+    ps = [ctx.Process(target=_worker, args=(r, world, q_id, q_out, case)) for r in range(world)]
+    for p in ps:
+        p.start()
+    res = []
+    try:
+        for _ in ps:
+            res.append(q_out.get(timeout=600))
+    finally:
+        for p in ps:
+            p.join(timeout=120)
+            if p.exitcode is None:
+                p.kill()
+    for rank, errs, tb in sorted(res, key=lambda r: r[0]):
+        assert tb is None, f"rank {rank} raised:\n{tb}"
+        assert not errs, f"rank {rank}: {errs}"
