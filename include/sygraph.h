@@ -234,6 +234,14 @@ SG_API int sg_profile(sg_graph *g, int enable);
 SG_API int sg_profile_read(const sg_graph *g, sg_kprof *out);
 /* Kernel launches issued by this library since load (host-side counter). */
 SG_API int64_t sg_launch_count(void);
+/* Per-superstep trace of the last device-driven run_bfs on g: for decision i (i = 0 is the
+ * prologue's), globaltimer ns since decision 0, the decision (0 stop, 1 push, 2 pull, 3 sweep,
+ * 4 fused sparse superstep) and the frontier it was taken on (words, n_f, m_f).  Returns the
+ * number of entries (<= cap); pointers may be NULL. */
+/* Debug accumulators of the last device-driven run_bfs (fused sparse loop phase times, ns). */
+SG_API int sg_ctrl_debug(const sg_graph *g, int64_t out[16]);
+SG_API int sg_bfs_trace(const sg_graph *g, int64_t *t_ns, int32_t *kind, int64_t *count, int64_t *nf, int64_t *mf,
+                        int32_t cap);
 
 /* Defaults for sg_opts (stream NULL, AUTO direction, alpha 14, beta 24). */
 SG_API void sg_opts_default(sg_opts *o);

@@ -76,7 +76,7 @@ EXPORTS = ["graph_load_csr", "graph_free", "graph_info", "frontier_init", "front
            "frontier_fill_all", "frontier_clear", "frontier_count", "frontier_view", "frontier_op",
            "frontier_or_into", "advance", "run_bfs", "run_sssp", "run_cc", "run_bc", "sg_opts_default",
            "sg_last_error", "sg_version", "sg_profile", "sg_profile_read", "sg_launch_count", "frontier_filter",
-           "compute_execute", "comm_unique_id", "comm_init", "comm_free", "comm_info", "graph_partition"]
+           "compute_execute", "comm_unique_id", "comm_init", "comm_free", "comm_info", "graph_partition", "sg_bfs_trace", "sg_ctrl_debug"]
 SG_PRED_DEGREE_RANGE, SG_PRED_U32_RANGE, SG_PRED_I32_RANGE, SG_PRED_F64_RANGE, SG_PRED_IN_BITMAP = 0, 1, 2, 3, 4
 SG_OP_SET_U32, SG_OP_SET_I32, SG_OP_SET_F64, SG_OP_ADD_U32, SG_OP_ADD_F64 = 0, 1, 2, 3, 4
 
@@ -96,6 +96,8 @@ def load():
     sig = {
         "graph_load_csr": (c_int, [i64, i64, vp, vp, vp, c_int, c_int, vp, vp, pp]),
         "graph_partition": (c_int, [vp, ctypes.POINTER(i64), ctypes.POINTER(i64)]),
+        "sg_bfs_trace": (c_int, [vp, vp, vp, vp, vp, vp, i32]),
+        "sg_ctrl_debug": (c_int, [vp, vp]),
         "comm_unique_id": (c_int, [ctypes.c_char_p]),
         "comm_init": (c_int, [ctypes.c_char_p, c_int, c_int, c_int, pp]),
         "comm_free": (c_int, [vp]),
@@ -448,6 +450,32 @@ def profile_read(g: Graph) -> dict:
     arr = (SgKprof * SG_K_COUNT)()
     _check(load().sg_profile_read(g.handle, arr))
     return {K_NAMES[i]: dict(ms=arr[i].ms, bytes=arr[i].bytes, launches=arr[i].launches) for i in range(SG_K_COUNT)}
+
+
+TRACE_KINDS = {0: "stop", 1: "push", 2: "pull", 3: "sweep", 4: "sparse"}
+
+
+def bfs_trace(g: Graph) -> list:
+    """Per-superstep trace of the last device-driven run_bfs on g (sg_bfs_trace): dicts with the
+    superstep's kind, input frontier (words, n_f, m_f) and device time in us (decision to decision)."""
+    cap = 48
+    t = (ctypes.c_int64 * cap)()
+    k = (ctypes.c_int32 * cap)()
+    c, nf, mf = (ctypes.c_int64 * cap)(), (ctypes.c_int64 * cap)(), (ctypes.c_int64 * cap)()
+    n = load().sg_bfs_trace(g.handle, t, k, c, nf, mf, cap)
+    if n < 0:
+        _check(n)
+    out = []
+    for i in range(n - 1):
+        out.append({"step": i, "kind": TRACE_KINDS.get(k[i], k[i]), "words": c[i], "nf": nf[i], "mf": mf[i],
+                    "us": (t[i + 1] - t[i]) / 1e3})
+    return out
+
+
+def ctrl_debug(g: Graph) -> list:
+    out = (ctypes.c_int64 * 16)()
+    _check(load().sg_ctrl_debug(g.handle, out))
+    return list(out)
 
 
 def launch_count() -> int:

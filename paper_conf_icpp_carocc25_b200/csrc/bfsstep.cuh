@@ -27,13 +27,18 @@ __device__ __forceinline__ void bfs_set_cond(unsigned long long h, unsigned v) {
     if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, v);
 }
 
+// Superstep kinds (decisions)
+enum : uint32_t { SK_STOP = 0, SK_PUSH = 1, SK_PULL = 2, SK_SWEEP = 3, SK_SPARSE = 4 };
+
 // Beamer direction policy (R2) + loop control, from the freshly built output frontier's
 // control block `st`; `prev_arcs` = arcs inspected by the superstep just run (folded into the
 // per-direction totals); `zero_prev` (nullable) = the control block of the frontier just advanced,
-// zeroed here (it is the next superstep's output).  One thread.
-__device__ __forceinline__ void bfs_decide(BfsCtrl *c, const DevStats *st, unsigned long long prev_arcs,
-                                           DevStats *zero_prev, unsigned long long h_loop, unsigned long long h_push,
-                                           unsigned long long h_pull, unsigned long long h_sweep, int first) {
+// zeroed here (it is the next superstep's output).  `next_in` = the buffer holding the next
+// superstep's input: the IF nodes of that buffer's half get the decision, the other half's are
+// switched off (the fused sparse loop may end on either parity; its half is then skipped and the
+// WHILE loop comes back to the right one).  Returns the decision (SK_*).  One thread.
+__device__ __forceinline__ uint32_t bfs_decide(BfsCtrl *c, const DevStats *st, unsigned long long prev_arcs,
+                                               DevStats *zero_prev, int next_in, int first, bool defer_sparse = false) {
     // control blocks were filled by atomics of other CTAs / kernels: volatile (L2) reads
     const volatile DevStats *vst = st;
     if (!first) {
@@ -63,11 +68,38 @@ __device__ __forceinline__ void bfs_decide(BfsCtrl *c, const DevStats *st, unsig
     const bool push = go && !c->pull;
     const bool sweep = push && (c->sweep_mode == 2 || (c->sweep_mode == 1 && vst->mf >= c->sweep_thr));
     if (sweep) c->sweep_steps++;
-    bfs_set_cond(h_push, push && !sweep);
-    bfs_set_cond(h_sweep, sweep);
-    bfs_set_cond(h_pull, go && c->pull);
-    bfs_set_cond(h_loop, go);
+    const bool sparse = push && !sweep && c->hsparse[next_in] && c->sparse_mode && count <= c->sparse_words &&
+                        vst->mf <= c->sparse_arcs;
+    if (sparse) c->sparse_steps++;
+    {
+        const unsigned long long i = c->tr_n++;
+        if (i < (unsigned long long)SG_TRACE_STEPS) {
+            unsigned long long t;
+            asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+            c->t_ns[i] = t;
+            c->kind[i] = !go ? SK_STOP : (c->pull ? SK_PULL : (sweep ? SK_SWEEP : (sparse ? SK_SPARSE : SK_PUSH)));
+            c->tr_count[i] = count;
+            c->tr_nf[i] = vst->nf;
+            c->tr_mf[i] = vst->mf;
+        }
+    }
+    // handle values wanted: only the next input buffer's half has a taken IF; set the changed ones
+    if (!(defer_sparse && sparse)) {   // (the fused sparse loop continues without touching them)
+        const uint32_t kinds = (push && !sweep && !sparse ? 1u : 0u) | (go && c->pull ? 2u : 0u) |
+                               (sweep ? 4u : 0u) | (sparse ? 8u : 0u);
+        uint32_t want = go ? 0x100u : 0u;
+        for (int k = 0; k < 4; k++)
+            if ((kinds >> k) & 1u) want |= 1u << (2 * k + next_in);
+        const uint32_t diff = want ^ c->hmask;
+        const unsigned long long *hs[4] = {c->hpush, c->hpull, c->hsweep, c->hsparse};
+        for (int k = 0; k < 4; k++)
+            for (int b = 0; b < 2; b++)
+                if ((diff >> (2 * k + b)) & 1u) bfs_set_cond(hs[k][b], (want >> (2 * k + b)) & 1u);
+        if (diff & 0x100u) bfs_set_cond(c->hl, go);
+        c->hmask = want;
+    }
     if (zero_prev) *zero_prev = DevStats{};
+    return !go ? SK_STOP : (c->pull ? SK_PULL : (sweep ? SK_SWEEP : (sparse ? SK_SPARSE : SK_PUSH)));
 }
 
 // Emit a block's slice of the output frontier: `S` = the block's layer-2 words (in shared
@@ -157,6 +189,10 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
         *o.done = 0u;
         DevStats *prev = o.prev ? o.prev : in_st;
         unsigned long long prev_arcs = prev ? reinterpret_cast<const volatile DevStats *>(prev)->arcs : 0ull;
+        if (o.ctrl && prev) {   // retire the input buffer: the sparse kernel needs to know what it holds
+            o.ctrl->saved_count[o.half] = reinterpret_cast<const volatile DevStats *>(prev)->count;
+            o.ctrl->dirty[o.half] = o.sparse ? 0u : 1u;
+        }
         if (part) {
             volatile DevStats *vst = o.st;
             const unsigned long long my_nf = vst->nf, my_mf = vst->mf;
@@ -167,9 +203,9 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
             vst->mf = tot.mf;
             prev_arcs = tot.arcs;
             vst->pad = tot.arcs;   // host loops read the superstep's global arcs here
-            if (o.ctrl) bfs_decide(o.ctrl, o.st, prev_arcs, nullptr, o.h_loop, o.h_push, o.h_pull, o.h_sweep, 0);
+            if (o.ctrl) bfs_decide(o.ctrl, o.st, prev_arcs, nullptr, o.half ^ 1, 0);
         } else if (o.ctrl) {
-            bfs_decide(o.ctrl, o.st, prev_arcs, o.prev, o.h_loop, o.h_push, o.h_pull, o.h_sweep, 0);
+            bfs_decide(o.ctrl, o.st, prev_arcs, o.prev, o.half ^ 1, 0);
         }
     }
 }

@@ -122,6 +122,8 @@ struct Workspace {
     // CUDA-graph driven BFS (ctrl.cu): instantiated once per (level buffer, tiers)
     BfsCtrl *ctrl = nullptr, *h_ctrl = nullptr;
     unsigned int *bfs_done = nullptr;   // CTA completion counter of the BFS output kernels (self-resetting)
+    unsigned int *gbar = nullptr;       // grid barrier of the sparse superstep kernel (2 u32)
+    unsigned long long hnd[9] = {};     // conditional handles of bfs_graph (loop, push/pull/sweep/sparse x 2)
     cudaGraph_t bfs_graph = nullptr;
     cudaGraphExec_t bfs_exec = nullptr;
     uint32_t *bfs_level = nullptr;
@@ -227,6 +229,8 @@ static int ensure_ws(sg_graph *g) {
     }
     CK(cudaMalloc(&ws->bfs_done, sizeof(unsigned int)));
     CK(cudaMemset(ws->bfs_done, 0, sizeof(unsigned int)));
+    CK(cudaMalloc(&ws->gbar, 4 * sizeof(unsigned int)));
+    CK(cudaMemset(ws->gbar, 0, 4 * sizeof(unsigned int)));
     CK(cudaMalloc(&ws->visited, sizeof(uint64_t) * (size_t)g->v.nw1));
     CK(cudaMalloc(&ws->vis_old, sizeof(uint64_t) * (size_t)g->v.nw1));
     CK(cudaMalloc(&ws->scratch, 8 * sizeof(unsigned long long)));
@@ -241,7 +245,8 @@ static int ensure_ws(sg_graph *g) {
 static int ensure_heavy(sg_graph *g, int32_t heavy_deg) {
     Workspace *ws = g->ws;
     if (ws->heavy && ws->heavy_deg <= heavy_deg) return SG_OK;
-    const int64_t cap64 = g->v.nnz / HEAVY_CHUNK + g->v.nnz / heavy_deg + 64;
+    // (+ the sparse kernel's 256-arc items: <= SG_SPARSE_ARCS / 256 + one per listed word)
+    const int64_t cap64 = g->v.nnz / HEAVY_CHUNK + g->v.nnz / heavy_deg + 64 + (1 << 16) / 256 + 4096 + 64;
     if (cap64 > 0xFFFFFFF0ll) return fail(SG_ERR_UNSUPPORTED, "heavy queue too large (heavy_degree too small)");
     cudaFree(ws->heavy);
     ws->heavy = nullptr;
@@ -301,6 +306,7 @@ static void free_ws(Workspace *ws) {
     if (ws->cap_stream) cudaStreamDestroy(ws->cap_stream);
     cudaFree(ws->ctrl);
     cudaFree(ws->bfs_done);
+    cudaFree(ws->gbar);
     cudaFreeHost(ws->h_ctrl);
     if (ws->ev0) cudaEventDestroy(ws->ev0);
     if (ws->ev1) cudaEventDestroy(ws->ev1);
@@ -1189,13 +1195,14 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     cudaGraph_t root;
     CK(cudaGraphCreate(&root, 0));
     ws->bfs_graph = root;
-    cudaGraphConditionalHandle h_loop, h_push[2], h_pull[2], h_sweep[2];
+    cudaGraphConditionalHandle h_loop, h_push[2], h_pull[2], h_sweep[2], h_sparse[2];
     const bool sc = t.scsr != 0 && g->scsr_state == 1;
     CK(cudaGraphConditionalHandleCreate(&h_loop, root, 0, cudaGraphCondAssignDefault));
     for (int i = 0; i < 2; i++) {
         CK(cudaGraphConditionalHandleCreate(&h_push[i], root, 0, cudaGraphCondAssignDefault));
         CK(cudaGraphConditionalHandleCreate(&h_pull[i], root, 0, cudaGraphCondAssignDefault));
         if (sc) CK(cudaGraphConditionalHandleCreate(&h_sweep[i], root, 0, cudaGraphCondAssignDefault));
+        CK(cudaGraphConditionalHandleCreate(&h_sparse[i], root, 0, cudaGraphCondAssignDefault));
     }
     sg_frontier *F[2] = {&ws->fr[0], &ws->fr[1]};
     std::vector<cudaGraphNode_t> leaves;
@@ -1208,9 +1215,15 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
     CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
     launch_bfs_prologue(ws->ctrl, G.n, G.deg8, F[0]->bits, F[0]->summ, F[0]->offsets, F[0]->st, ws->visited,
-                        ws->vis_old, (unsigned long long)h_loop, (unsigned long long)h_push[0],
-                        (unsigned long long)h_pull[0], sc ? (unsigned long long)h_sweep[0] : 0ull,
-                        g->ar ? g->ar->x : Xchg{}, cs);
+                        ws->vis_old, g->ar ? g->ar->x : Xchg{}, cs);
+    // the handles go to the device with every run's control block (run_bfs_graph)
+    ws->hnd[0] = (unsigned long long)h_loop;
+    for (int i = 0; i < 2; i++) {
+        ws->hnd[1 + i] = (unsigned long long)h_push[i];
+        ws->hnd[3 + i] = (unsigned long long)h_pull[i];
+        ws->hnd[5 + i] = sc ? (unsigned long long)h_sweep[i] : 0ull;
+        ws->hnd[7 + i] = (unsigned long long)h_sparse[i];
+    }
     TRY(capture_end(cs, leaves));
     cudaGraphNode_t wnode;
     cudaGraph_t body;
@@ -1223,9 +1236,10 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         cudaGraph_t b_push, b_pull;
         TRY(add_cond(body, deps, h_push[half], cudaGraphCondTypeIf, &n_push, &b_push));
         TRY(add_cond(body, deps, h_pull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
-        cudaGraphNode_t n_sweep = nullptr;
-        cudaGraph_t b_sweep = nullptr;
+        cudaGraphNode_t n_sweep = nullptr, n_sparse = nullptr;
+        cudaGraph_t b_sweep = nullptr, b_sparse = nullptr;
         if (sc) TRY(add_cond(body, deps, h_sweep[half], cudaGraphCondTypeIf, &n_sweep, &b_sweep));
+        TRY(add_cond(body, deps, h_sparse[half], cudaGraphCondTypeIf, &n_sparse, &b_sparse));
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
         L.sparse_ok = 1;  // n_f of every BFS frontier is exact (prologue statistics / output kernels)
@@ -1233,10 +1247,9 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         // output of the superstep (out->st was zeroed by the previous decision / the prologue);
         // the output kernel's last CTA decides the next superstep (handles of the other half)
         BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, nullptr, 0u, &ws->ctrl->next,
-                  &ws->ctrl->level, out->st, ws->ctrl, in->st, ws->bfs_done, (unsigned long long)h_loop,
-                  (unsigned long long)h_push[half ^ 1], (unsigned long long)h_pull[half ^ 1],
-                  sc ? (unsigned long long)h_sweep[half ^ 1] : 0ull};
+                  &ws->ctrl->level, out->st, ws->ctrl, in->st, ws->bfs_done};
         if (g->ar) bo.x = g->ar->x;   // partitioned: owned slice replicated to the peers + barrier
+        bo.half = half;
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
         launch_bfs_diff(G, ws->visited, bo, cs);
@@ -1250,7 +1263,15 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         TRY(capture_begin(cs, b_pull, {}));
         launch_pull_bfs(g->vl, in->bits, ws->visited, in->st, bo, cs);   // writes its output itself
         TRY(capture_end(cs, leaves));
-        deps = {n_push, n_pull};
+        {   // small frontiers: the whole superstep in one kernel (sparse.cu)
+            BfsOut bs = bo;
+            bs.sparse = 1;
+            PushLaunch Ls = push_launch(g, in, t, -1);
+            TRY(capture_begin(cs, b_sparse, {}));
+            launch_bfs_sparse(Ls, a, bs, in->bits, in->summ, ws->gbar, cs);
+            TRY(capture_end(cs, leaves));
+        }
+        deps = {n_push, n_pull, n_sparse};
         if (n_sweep) deps.push_back(n_sweep);
     }
     CK(cudaGraphInstantiate(&ws->bfs_exec, root, 0));
@@ -1293,6 +1314,20 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     c.reached = 1;
     c.sweep_mode = (uint32_t)sc_mode;
     c.sweep_thr = sweep_threshold(g->v.nnz);
+    // the fused small-frontier loop (sparse.cu) beats the 4-kernel push superstep only across runs
+    // of >= 2 consecutive small supersteps (12 vs 21 us each, path graph); on config 4 it loses
+    // its first superstep to the extra clear + launch (measured 578 vs 543 us per BFS),
+    // so it is opt-in: SG_SPARSE=1
+    c.sparse_mode = (uint32_t)env_or("SG_SPARSE", 0);
+    c.sparse_words = env_or("SG_SPARSE_WORDS", 4096);
+    c.sparse_arcs = env_or("SG_SPARSE_ARCS", 1 << 16);
+    c.hl = ws->hnd[0];
+    for (int i = 0; i < 2; i++) {
+        c.hpush[i] = ws->hnd[1 + i];
+        c.hpull[i] = ws->hnd[3 + i];
+        c.hsweep[i] = ws->hnd[5 + i];
+        c.hsparse[i] = ws->hnd[7 + i];
+    }
     CK(cudaEventRecord(ws->ev0, s));
     CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, sizeof(BfsCtrl), cudaMemcpyHostToDevice, s));
     CK(cudaGraphLaunch(ws->bfs_exec, s));
@@ -1315,8 +1350,8 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         // taken IF bodies (push = word + CTA tier [+ hub segment tier] + output, sweep = arc
         // count + sweep + output, pull = 1)
         const long long per_push = 3 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
-        const long long k = 1 + per_push * (long long)(c.push_steps - c.sweep_steps) + 3 * (long long)c.sweep_steps +
-                            (long long)c.pull_steps;
+        const long long k = 1 + per_push * (long long)(c.push_steps - c.sweep_steps - c.sparse_steps) +
+                            3 * (long long)c.sweep_steps + (long long)c.sparse_steps + (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }
     if (stats) {
@@ -2031,5 +2066,26 @@ SG_API int sg_profile_read(const sg_graph *g, sg_kprof *out) {
 }
 
 SG_API int64_t sg_launch_count(void) { return (int64_t)g_launches.load(); }
+
+SG_API int sg_ctrl_debug(const sg_graph *g, int64_t out[16]) {
+    if (!g || !g->ws || !g->ws->h_ctrl || !out) return fail(SG_ERR_STATE, "no device-driven BFS has run on this graph");
+    for (int i = 0; i < 16; i++) out[i] = (int64_t)g->ws->h_ctrl->dbg[i];
+    return SG_OK;
+}
+
+SG_API int sg_bfs_trace(const sg_graph *g, int64_t *t_ns, int32_t *kind, int64_t *count, int64_t *nf, int64_t *mf,
+                        int32_t cap) {
+    if (!g || !g->ws || !g->ws->h_ctrl) return fail(SG_ERR_STATE, "no device-driven BFS has run on this graph");
+    const BfsCtrl &c = *g->ws->h_ctrl;
+    const int n = (int)(c.tr_n < (unsigned long long)SG_TRACE_STEPS ? c.tr_n : SG_TRACE_STEPS);
+    for (int i = 0; i < n && i < cap; i++) {
+        if (t_ns) t_ns[i] = (int64_t)(c.t_ns[i] - c.t_ns[0]);
+        if (kind) kind[i] = (int32_t)c.kind[i];
+        if (count) count[i] = (int64_t)c.tr_count[i];
+        if (nf) nf[i] = (int64_t)c.tr_nf[i];
+        if (mf) mf[i] = (int64_t)c.tr_mf[i];
+    }
+    return n < cap ? n : cap;
+}
 
 }  // extern "C"

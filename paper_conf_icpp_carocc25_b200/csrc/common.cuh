@@ -78,6 +78,8 @@ struct DevStats {
     unsigned long long pad;
 };
 
+constexpr int SG_TRACE_STEPS = 48;
+
 // Device-resident state of a graph-driven BFS (written by k_bfs_decide, read back once per run).
 struct BfsCtrl {
     unsigned long long iters, push_steps, pull_steps, arcs_pushed, arcs_pulled, reached;
@@ -94,6 +96,29 @@ struct BfsCtrl {
     uint32_t sweep_mode;     // push supersteps through the sweep: 0 never, 1 when m_f >= sweep_thr, 2 always
     unsigned long long sweep_thr;
     unsigned long long sweep_steps;
+    // fused small-frontier supersteps (sparse.cu): taken when count <= sparse_words and m_f <= sparse_arcs
+    uint32_t sparse_mode;    // 0 off, 1 on
+    uint32_t pad0;
+    unsigned long long sparse_words, sparse_arcs, sparse_steps;
+    // frontier buffer b still holds a consumed frontier (dirty[b]) whose word list had
+    // saved_count[b] entries (~0: unknown, clear every word); the sparse kernel needs an all-zero
+    // output buffer and clears it first when dirty
+    uint32_t dirty[2];
+    unsigned long long saved_count[2];
+    // conditional handles of the graph (cudaGraphConditionalHandle values; 0 = no such node):
+    // the loop, and per frontier buffer b the IF nodes of the supersteps whose input is buffer b
+    unsigned long long hl, hpush[2], hpull[2], hsweep[2], hsparse[2];
+    unsigned long long dbg[16];   // phase time accumulators of the fused sparse loop (CTA 0, ns; sg_ctrl_debug)
+    uint32_t sp_kind;        // the fused sparse loop's last decision (read by all its CTAs)
+    uint32_t sp_epoch;       // bumped by CTA 0 once sp_kind is written (the loop's broadcast)
+    uint32_t hmask;          // current values of the IF handles (bit 2k+b: kind k of buffer b; bit 8: loop);
+    uint32_t pad1;           // only changed handles are set (cudaGraphSetConditional costs ~0.4 us)
+    // per-superstep trace (sg_bfs_trace): globaltimer at each decision, the decision taken
+    // (0 stop, 1 push, 2 pull, 3 sweep, 4 sparse) and the frontier it was taken on
+    unsigned long long tr_n;
+    unsigned long long t_ns[SG_TRACE_STEPS];
+    uint32_t kind[SG_TRACE_STEPS];
+    unsigned long long tr_count[SG_TRACE_STEPS], tr_nf[SG_TRACE_STEPS], tr_mf[SG_TRACE_STEPS];
 };
 
 // Device-resident control of one source-batched BC batch (bcb.cu).

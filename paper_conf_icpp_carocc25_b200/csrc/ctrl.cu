@@ -57,9 +57,7 @@ __global__ void k_zero_u64(unsigned long long *p, int64_t n) {
 // list, n_f = 1, m_f = src's coded degree, as the compaction + statistics kernels would give),
 // visited |= {src}, then the first direction decision.  The frontier's words were zeroed before.
 __global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
-                               uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
-                               unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
-                               unsigned long long h_sweep, Xchg x) {
+                               uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old, Xchg x) {
     uint32_t *level = c->level;
     const int32_t src = c->src;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -85,19 +83,20 @@ __global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint6
         st->nf = 1ull;
         st->mf = deg8_decode(deg8[src]);
         if (x.nranks > 1) xbarrier(x, 0ull, 0ull, 0ull, nullptr);   // every rank's prologue memsets done
-        bfs_decide(c, st, 0ull, nullptr, h_loop, h_push, h_pull, h_sweep, 1);
+        c->dirty[0] = 0u;            // buffer 0: zeroed by the prologue, holds {src}
+        c->dirty[1] = 1u;            // buffer 1: a previous run's frontier; contents unknown
+        c->saved_count[1] = ~0ull;
+        bfs_decide(c, st, 0ull, nullptr, 0, 1);
     }
 }
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
-                         uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
-                         unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
-                         unsigned long long h_sweep, const Xchg &x, cudaStream_t s) {
+                         uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old, const Xchg &x,
+                         cudaStream_t s) {
     int64_t blocks = (n / 4 + 255) / 256;
     if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
     note_launch();
-    k_bfs_prologue<<<(int)blocks, 256, 0, s>>>(c, n, deg8, bits, summ, offsets, st, visited, vis_old, h_loop, h_push,
-                                               h_pull, h_sweep, x);
+    k_bfs_prologue<<<(int)blocks, 256, 0, s>>>(c, n, deg8, bits, summ, offsets, st, visited, vis_old, x);
 }
 
 // Barrier across the ranks of a partition (one thread; xchg.cuh)

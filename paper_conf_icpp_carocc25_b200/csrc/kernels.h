@@ -96,16 +96,22 @@ struct BfsOut {
     const uint32_t *next_ptr;
     uint32_t *const *level_pp;
     DevStats *st;
-    BfsCtrl *ctrl;                    // NULL: host loop (no device-side decision)
+    BfsCtrl *ctrl;                    // NULL: host loop (no device-side decision; handles in ctrl)
     DevStats *prev;
     unsigned int *done;               // CTA completion counter (self-resetting)
-    unsigned long long h_loop, h_push, h_pull, h_sweep;
     Xchg x;                           // partitioned: peers' replicas of the output (xchg.cuh)
+    int32_t half = 0;                 // graph mode: index (0/1) of the INPUT frontier buffer
+    int32_t sparse = 0;               // 1: the superstep consumed (zeroed) its input (sparse.cu)
 };
 // pull.cu — bottom-up BFS step (direction-optimising, Beamer): writes its output `o`
 // itself (no k_bfs_diff after it); o.out_bits == NULL: marks visited only (k_bfs_diff after it)
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,
                      cudaStream_t s);
+// sparse.cu — a whole small-frontier BFS superstep in one persistent kernel (graph mode only):
+// push with direct output insertion, the input zeroed as consumed, the decision by its last CTA.
+// gbar: 2 zeroed u32 (grid barrier).
+void launch_bfs_sparse(const PushLaunch &L, const BfsArgs &a, const BfsOut &o, uint64_t *in_bits, uint64_t *in_summ,
+                       unsigned int *gbar, cudaStream_t s);
 // frontier.cu — output of a diff-mode BFS superstep (push word path / sweep): see BfsOut
 void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s);
 
@@ -161,9 +167,8 @@ void launch_push_sweep(const ScsrView &v, const int64_t *rp, const uint64_t *in_
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 // level init + seed + the seed frontier's word list / statistics + first decision, one kernel
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
-                         uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old,
-                         unsigned long long h_loop, unsigned long long h_push, unsigned long long h_pull,
-                         unsigned long long h_sweep, const Xchg &x, cudaStream_t s);
+                         uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old, const Xchg &x,
+                         cudaStream_t s);
 void launch_clear_listed(uint64_t *bits, uint64_t *summ, const uint32_t *offsets, const DevStats *st, int64_t nw1,
                          int64_t nw2, DevStats *zero_st, cudaStream_t s);
 void launch_zero_u64(unsigned long long *p, int64_t n, cudaStream_t s);

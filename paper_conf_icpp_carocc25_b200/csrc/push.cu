@@ -23,6 +23,7 @@ static PushParams make_params(const PushLaunch &L) {
     p.seg_threshold = L.seg_threshold;
     p.skip_mf = L.skip_mf;
     p.sparse_ok = L.sparse_ok;
+    p.chunk = HEAVY_CHUNK;
     return p;
 }
 

@@ -53,6 +53,7 @@ struct PushParams {
     unsigned long long skip_mf;   // the segmented (SCSR) advance handles this superstep: m_f >= skip_mf
     int32_t sparse_ok;     // st->nf is exact: words with <= 2 active vertices on average take the
                            // thread-per-word path (push_words_sparse)
+    int32_t chunk = HEAVY_CHUNK;   // arcs per queued CTA/grid-tier item (the sparse kernel: a warp round)
 };
 
 template <class F>
@@ -117,13 +118,14 @@ __device__ __forceinline__ void warp_expand(const GraphView &g, const F &f, int6
 // ---- CTA/grid tier enqueue -------------------------------------------------------------
 __device__ __forceinline__ void enqueue_heavy(const PushParams &p, int32_t u, int64_t s, int64_t e) {
     const int64_t d = e - s;
-    const uint32_t nch = (uint32_t)((d + HEAVY_CHUNK - 1) / HEAVY_CHUNK);
+    const int64_t ch = p.chunk;
+    const uint32_t nch = (uint32_t)((d + ch - 1) / ch);
     const unsigned long long pos = atomicAdd(&p.st->heavy_count, (unsigned long long)nch);
     for (uint32_t j = 0; j < nch; j++) {
         if (pos + j >= p.heavy_cap) break;      // cannot happen: capacity bound in DESIGN.md
         HeavyItem it;
-        it.begin = s + (int64_t)j * HEAVY_CHUNK;
-        it.len = (int32_t)min((int64_t)HEAVY_CHUNK, e - it.begin);
+        it.begin = s + (int64_t)j * ch;
+        it.len = (int32_t)min(ch, e - it.begin);
         it.u = u;
         p.heavy[pos + j] = it;
     }

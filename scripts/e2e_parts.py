@@ -1,7 +1,7 @@
 """Wall-clock parts of one end-to-end BFS step on config 4 (graph_load_csr from pinned host
 memory, first run_bfs on the fresh graph, a second run_bfs, graph free).
 
-    python scripts/e2e_parts.py [reps]"""
+    python scripts/e2e_parts.py [reps] [--resident]   (--resident: another graph stays loaded, as in bench.py)"""
 import os
 import sys
 import time
@@ -12,13 +12,14 @@ import torch  # noqa: E402
 import gen  # noqa: E402
 import paper_conf_icpp_carocc25_b200 as sg  # noqa: E402
 
-reps = int(sys.argv[1]) if len(sys.argv) > 1 else 3
+reps = int(sys.argv[1]) if len(sys.argv) > 1 and sys.argv[1].isdigit() else 3
 g = gen.make_config_graph(4)
 roots = gen.config_sources(4, g)
 rp_h = torch.from_numpy(g.row_ptr).pin_memory()
 ci_h = torch.from_numpy(g.col_idx).pin_memory()
 lv = torch.empty(g.n, dtype=torch.int32, device="cuda")
 stream = torch.cuda.current_stream()
+keep = sg.graph_load_csr(rp_h, ci_h, stream=stream) if "--resident" in sys.argv else None   # as in bench.py
 for r in range(reps):
     torch.cuda.synchronize()
     t0 = time.perf_counter()

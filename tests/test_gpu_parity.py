@@ -510,3 +510,26 @@ def test_bc_duplicates_and_isolated(sg):
     srcs = [0, 0, 7, 2]
     bc, _ = sg.run_bc(G, srcs)
     assert bc_close(bc.cpu().numpy(), oracle.bc(g, srcs))
+
+
+@pytest.mark.parametrize("make", [lambda: gen.rmat(14, 16, permute=True), lambda: gen.path(300),
+                                  lambda: gen.lattice(90, 120, 0.6, seed=3), lambda: gen.rmat(12, 4, permute=True)])
+def test_bfs_fused_sparse_supersteps(sg, monkeypatch, make):
+    """SG_SPARSE=1: small push supersteps run in the fused persistent loop (sparse.cu: direct output
+    insertion, the input zeroed as consumed, dirty output buffers cleared first, 256-arc items for
+    long lists, several supersteps per launch ending on either buffer parity); levels and step
+    counts equal the default path's and the oracle's."""
+    g = make()
+    G = load(sg, g)
+    for s in list(gen.sources(g, 3)) + [int(np.argmax(g.degrees()))]:
+        ref = oracle.bfs(g, int(s))
+        monkeypatch.setenv("SG_SPARSE", "0")
+        _, st0 = sg.run_bfs(G, int(s))
+        for arcs in ("65536", "300", "0"):
+            monkeypatch.setenv("SG_SPARSE", "1")
+            monkeypatch.setenv("SG_SPARSE_ARCS", arcs)
+            for d in (sg.SG_DIR_AUTO, sg.SG_DIR_PUSH):
+                lv, st = sg.run_bfs(G, int(s), direction=d)
+                assert np.array_equal(sg.as_u32(lv), ref), (s, arcs, d)
+            _, st = sg.run_bfs(G, int(s))
+            assert (st.iterations, st.push_steps, st.pull_steps) == (st0.iterations, st0.push_steps, st0.pull_steps)

@@ -55,6 +55,11 @@ def _worker(rank, world, q_id, q_out, case):
                            (st1.iterations, st1.push_steps, st1.pull_steps, st1.reached), errs)
                 lv, _ = sg.run_bfs(G, int(s), owned_only=True)
                 _check(f"bfs owned_only root {s}", np.array_equal(sg.as_u32(lv)[lo:hi], ref[lo:hi]), errs)
+            os.environ["SG_SPARSE"] = "1"        # fused small supersteps (peer inserts + clear barrier)
+            for s in roots[:2]:
+                lv, _ = sg.run_bfs(G, int(s))
+                _check(f"bfs sparse root {s}", np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), errs)
+            del os.environ["SG_SPARSE"]
             with pytest.raises(sg.SgError):
                 sg.run_bfs(G, 0, host_loop=True)
         elif case == "sssp":
