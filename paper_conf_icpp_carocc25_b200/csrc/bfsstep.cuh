@@ -83,6 +83,10 @@ __device__ __forceinline__ uint32_t bfs_decide(BfsCtrl *c, const DevStats *st, u
             c->tr_mf[i] = vst->mf;
         }
     }
+    // late pulls run warp-owned layer-2 words (pull.cu k_pull_bfs_w): few unvisited vertices left
+    c->pull_warp[next_in] = c->pull_warp_frac &&
+                   (unsigned long long)(c->n - c->n_iso - (long long)c->reached) * c->pull_warp_frac <
+                       (unsigned long long)(c->n - c->n_iso);
     // handle values wanted: only the next input buffer's half has a taken IF; set the changed ones
     if (!(defer_sparse && sparse)) {   // (the fused sparse loop continues without touching them)
         const uint32_t kinds = (push && !sweep && !sparse ? 1u : 0u) | (go && c->pull ? 2u : 0u) |

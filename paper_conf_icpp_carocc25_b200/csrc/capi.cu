@@ -167,6 +167,7 @@ struct sg_graph {
     Arena *ar = nullptr;            // exchange arena (partitioned only)
     int nranks = 1, rank = 0;
     sg_comm *comm = nullptr;        // partitioned: graph_free is collective over it
+    int64_t n_iso = 0;              // isolated vertices (deg 0)
 };
 static std::atomic<int> g_live_graphs{0};
 
@@ -590,11 +591,11 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     g->v.col = g->col;
     g->v.w = g->w;
     unsigned long long *dscr = nullptr;
-    CK(cudaMalloc(&dscr, 48));
-    CK(cudaMemsetAsync(dscr, 0, 48, s));
+    CK(cudaMalloc(&dscr, 64));
+    CK(cudaMemsetAsync(dscr, 0, 64, s));
     // structure first (the derived arrays below index with row_ptr / col_idx)
     launch_validate_csr(g->v, dscr, s);
-    unsigned long long hv[6] = {0, 0, 0, 0, 0, 0};
+    unsigned long long hv[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     CK(cudaMemcpyAsync(hv, dscr, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     if (hv[0]) {
@@ -609,6 +610,7 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     g->v.deg8 = g->deg8;
     CK(dev_alloc(&g->isolated, sizeof(uint64_t) * (size_t)g->v.nw1, s));
     launch_isolated(g->deg8, n, g->v.nw1, g->isolated, s);
+    launch_popcount(g->isolated, g->v.nw1, dscr + 6, s);           // [6] isolated vertices
     CK(dev_alloc(&g->fnbr, sizeof(int32_t) * (size_t)(g->v.nw1 ? g->v.nw1 * 64 : 1), s));   // padded: 16-B quad loads
     launch_first_nbr(g->rp, g->col, g->deg8, n, g->v.nw1 * 64, g->fnbr, s);
     g->v.fnbr = g->fnbr;
@@ -618,11 +620,12 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     CK(dev_alloc(&g->hub_idx, sizeof(int32_t) * (size_t)n, s));
     CK(dev_alloc(&g->hub_vertex, sizeof(int32_t) * (size_t)max_hubs, s));
     launch_hub_mark(g->rp, n, g->hub_idx, g->hub_vertex, reinterpret_cast<unsigned int *>(dscr + 2), s);
-    CK(cudaMemcpyAsync(hv, dscr, 48, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(hv, dscr, 64, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     CK(cudaGetLastError());
     cudaFree(dscr);
     g->max_w = (uint32_t)(hv[1] & 0xffffffffu);
+    g->n_iso = (int64_t)hv[6];
     if ((flags & SG_F_VALIDATE) && (hv[3] || hv[4] || hv[5])) {
         graph_free(g);
         return fail(SG_ERR_INVALID, "CSR validation failed: %llu unsorted/duplicate pairs, %llu self-loops, %llu arcs "
@@ -1321,6 +1324,8 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     c.sparse_mode = (uint32_t)env_or("SG_SPARSE", 0);
     c.sparse_words = env_or("SG_SPARSE_WORDS", 4096);
     c.sparse_arcs = env_or("SG_SPARSE_ARCS", 1 << 16);
+    c.pull_warp_frac = (uint32_t)env_or("SG_PULL_WARP_FRAC", 8);
+    c.n_iso = g->n_iso;
     c.hl = ws->hnd[0];
     for (int i = 0; i < 2; i++) {
         c.hpush[i] = ws->hnd[1 + i];
@@ -1351,7 +1356,7 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         // count + sweep + output, pull = 1)
         const long long per_push = 3 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
         const long long k = 1 + per_push * (long long)(c.push_steps - c.sweep_steps - c.sparse_steps) +
-                            3 * (long long)c.sweep_steps + (long long)c.sparse_steps + (long long)c.pull_steps;
+                            3 * (long long)c.sweep_steps + (long long)c.sparse_steps + 2 * (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }
     if (stats) {
@@ -1432,7 +1437,11 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         const int64_t reached_before = reached;
         const bool sweep = !pull && scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz));
         CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
-        const BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, level, d + 1, nullptr, nullptr, out->st};
+        BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, level, d + 1, nullptr, nullptr, out->st};
+        {   // late pulls: warp-owned layer-2 words (same rule as bfs_decide)
+            const long long frac = (long long)env_or("SG_PULL_WARP_FRAC", 8), live = G.n - g->n_iso;
+            bo.pull_warp = frac > 0 && (live - reached) * frac < live ? 1 : 0;
+        }
         const int pr = prof_begin(ws, pull ? SG_K_PULL : (sweep ? SG_K_SWEEP : SG_K_PUSH), s);
         if (pull) {
             launch_pull_bfs(G, in->bits, ws->visited, in->st, bo, s);   // writes its output itself

@@ -109,6 +109,11 @@ struct BfsCtrl {
     // the loop, and per frontier buffer b the IF nodes of the supersteps whose input is buffer b
     unsigned long long hl, hpush[2], hpull[2], hsweep[2], hsparse[2];
     unsigned long long dbg[16];   // phase time accumulators of the fused sparse loop (CTA 0, ns; sg_ctrl_debug)
+    uint32_t pull_warp[2];   // a pull whose input is buffer b runs warp-owned layer-2 words (late pulls);
+                             // indexed by buffer: the decision writes the next input's entry while
+                             // both pull kernels of the current superstep read the current one
+    uint32_t pull_warp_frac; // ... when unvisited non-isolated vertices < (n - n_iso) / pull_warp_frac
+    long long n_iso;         // isolated vertices (visited from the start, never reached)
     uint32_t sp_kind;        // the fused sparse loop's last decision (read by all its CTAs)
     uint32_t sp_epoch;       // bumped by CTA 0 once sp_kind is written (the loop's broadcast)
     uint32_t hmask;          // current values of the IF handles (bit 2k+b: kind k of buffer b; bit 8: loop);

@@ -102,6 +102,7 @@ struct BfsOut {
     Xchg x;                           // partitioned: peers' replicas of the output (xchg.cuh)
     int32_t half = 0;                 // graph mode: index (0/1) of the INPUT frontier buffer
     int32_t sparse = 0;               // 1: the superstep consumed (zeroed) its input (sparse.cu)
+    int32_t pull_warp = 0;            // host loop: 1 = the pull runs warp-owned layer-2 words (graph mode: ctrl)
 };
 // pull.cu — bottom-up BFS step (direction-optimising, Beamer): writes its output `o`
 // itself (no k_bfs_diff after it); o.out_bits == NULL: marks visited only (k_bfs_diff after it)

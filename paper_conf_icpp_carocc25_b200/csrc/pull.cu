@@ -27,9 +27,12 @@
 // words; at most SG_PULL_WORD_MAX unvisited in every word -> word mode (a thread per layer-1
 // word walks its unvisited vertices, SG_PULL_WORD_BATCH candidate tests in flight); else the
 // quad rounds, where a warp whose two words are fully visited skips without loading them.
+#include <cstdlib>
+
 #include "common.cuh"
 #include "kernels.h"
 #include "bfsstep.cuh"
+#include "pullw.cuh"
 
 namespace sg {
 
@@ -99,6 +102,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
     __shared__ uint32_t s_full[2][2], s_mx[2][2];   // double-buffered by iteration parity (no barrier at reuse)
     int par = 0;
 #endif
+    if (o.ctrl ? o.ctrl->pull_warp[o.half] : o.pull_warp) return;   // late pull: k_pull_bfs_w takes it
     deg8_lut_init(s_lut);
     __syncthreads();
     uint32_t *const lvl = o.level_pp ? *o.level_pp : o.level;
@@ -292,14 +296,47 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
     bfs_finish(o, nf, mf, arcs, st);
 }
 
+// Late pull steps (few unvisited vertices left): one warp per layer-2 word (pullw.cuh), no CTA
+// barrier, misses drained cooperatively.  Runs iff ctrl->pull_warp (graph mode; both kernels are
+// in the pull node and the other one returns at once) or o.pull_warp (host loop).
+__global__ void __launch_bounds__(256, 4)
+k_pull_bfs_w(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
+             BfsOut o) {
+    if (!(o.ctrl ? o.ctrl->pull_warp[o.half] : o.pull_warp)) return;
+    __shared__ P2Warp s_w[8];
+    __shared__ uint32_t s_lut[256];
+    deg8_lut_init(s_lut);
+    __syncthreads();
+    uint32_t *const lvl = o.level_pp ? *o.level_pp : o.level;
+    const uint32_t nx = o.next_ptr ? *o.next_ptr : o.next;
+    const int wid = threadIdx.x >> 5;
+    const uint32_t *in32 = reinterpret_cast<const uint32_t *>(in_bits);
+    unsigned long long nf = 0, mf = 0, arcs = 0;
+    const int64_t gwarp = (int64_t)blockIdx.x * 8 + wid, nwarps = (int64_t)gridDim.x * 8;
+    for (int64_t sw = g.w2_lo + gwarp; sw < g.w2_hi; sw += nwarps)
+        pull_l2_warp(g, sw, in32, visited, o, s_w[wid], s_lut, lvl, nx, nf, mf, arcs);
+    bfs_finish(o, nf, mf, arcs, st);
+}
+
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,
                      cudaStream_t s) {
-    // one CTA per layer-2 word in a grid-stride loop over SG_PULL_WAVES CTAs per SM
-    int64_t blocks = g.w2_hi - g.w2_lo;
-    if (blocks > num_sms() * SG_PULL_WAVES) blocks = num_sms() * SG_PULL_WAVES;
-    if (blocks < 1) blocks = 1;
-    note_launch();
-    k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);
+    // graph mode launches both kernels (the device-side decision picks one); the host loop one
+    const bool both = o.ctrl != nullptr;
+    if (both || !o.pull_warp) {
+        // one CTA per layer-2 word in a grid-stride loop over SG_PULL_WAVES CTAs per SM
+        int64_t blocks = g.w2_hi - g.w2_lo;
+        if (blocks > num_sms() * SG_PULL_WAVES) blocks = num_sms() * SG_PULL_WAVES;
+        if (blocks < 1) blocks = 1;
+        note_launch();
+        k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);
+    }
+    if (both || o.pull_warp) {
+        int64_t blocks = (g.w2_hi - g.w2_lo + 7) / 8;   // one warp per layer-2 word
+        if (blocks > num_sms() * 4) blocks = num_sms() * 4;
+        if (blocks < 1) blocks = 1;
+        note_launch();
+        k_pull_bfs_w<<<(int)blocks, 256, 0, s>>>(g, in_bits, visited, st, o);
+    }
 }
 
 }  // namespace sg

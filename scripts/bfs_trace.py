@@ -26,6 +26,9 @@ def main():
     ap.add_argument("--env", nargs="*", default=[""])
     ap.add_argument("--json", default=None)
     ap.add_argument("--quiet", action="store_true")
+    ap.add_argument("--alpha", type=float, default=14.0)
+    ap.add_argument("--beta", type=float, default=24.0)
+    ap.add_argument("--segmented", type=int, default=0)
     a = ap.parse_args()
     torch.cuda.set_device(0)
     g = gen.make_config_graph(a.config)
@@ -38,11 +41,12 @@ def main():
         for kv in filter(None, env.split(",")):
             k, _, v = kv.partition("=")
             os.environ[k] = v
+        o = sg.opts(alpha=a.alpha, beta=a.beta, segmented=a.segmented)
         for r in roots[:2]:
-            sg.run_bfs(G, r, lv)   # warm-up (graph instantiation)
+            sg.run_bfs(G, r, lv, o)   # warm-up (graph instantiation)
         per_kind, totals = {}, []
         for r in roots:
-            _, st = sg.run_bfs(G, r, lv)
+            _, st = sg.run_bfs(G, r, lv, o)
             tr = sg.bfs_trace(G)
             totals.append(st.device_ms * 1e3)
             dbg = sg.ctrl_debug(G)
