@@ -150,6 +150,8 @@ struct sg_graph {
     uint32_t *hub_off = nullptr;    // [nhubs][nseg+1] segment offsets within the hub's row
     uint32_t *cbo = nullptr;        // [n][cbo_nb-1] first arc of each row into each CC label block (run_cc)
     int cbo_nb = 0;
+    CcBlocks ccb;                   // block-major arc copy for the label-blocked CC pull (built lazily)
+    int ccb_state = 0;              // 0 not built, 1 built (ccb.nb blocks), -1 unavailable (memory)
     int64_t nhubs = 0;
     ScsrStore scsr;                 // destination-segmented copy of the arcs (BFS heavy push), built lazily
     int scsr_state = 0;             // 0 not built, 1 built, -1 unavailable (segment block >= 2^32 arcs, unsorted rows)
@@ -678,6 +680,7 @@ SG_API int graph_free(sg_graph *g) {
     dev_free(g->hub_vertex);
     dev_free(g->hub_off);
     dev_free(g->cbo);
+    ccb_free(&g->ccb);
     if (g->scsr_state == 1) scsr_free(&g->scsr);
     delete g;
     if (--g_live_graphs == 0) {   // the last graph: give the pool's memory back to the device
@@ -1521,6 +1524,67 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
 
 }  // extern "C"
 
+// Label blocks of the CC pull (label block <= SG_CC_LBLOCK_KB stays in L2).  Returns the number
+// of blocks to pull with and sets *ccb: the block-major copy (preferred; SG_CC_CCB=0 disables),
+// else the per-row block offsets (cbo), else 1 block (unblocked; needs no extra memory).
+static int cc_blocks(sg_graph *g, const GraphView &GL, int direction, cudaStream_t s, bool *ccb) {
+    *ccb = false;
+    if (direction == SG_DIR_PUSH || !g->sorted) return 1;
+    const long long lblock = (long long)env_or("SG_CC_LBLOCK_KB", 32768) << 10;
+    int nb = (int)(((long long)GL.n * 4 + lblock - 1) / (lblock > 0 ? lblock : 1));
+    if (nb < 1 || lblock <= 0) nb = 1;
+    if (nb > 64) nb = 64;
+    if (nb == 1) return 1;
+    const int64_t S = (GL.n + nb - 1) / nb;
+    if (env_or("SG_CC_CCB", 1) != 0 && GL.nnz < 0xFFFFFFF0ll) {
+        if (g->ccb_state == 1 && g->ccb.nb == nb && g->ccb.S == S) {
+            *ccb = true;
+            return nb;
+        }
+        if (g->ccb_state != -1) {
+            if (g->ccb_state == 1) {
+                cudaStreamSynchronize(s);
+                ccb_free(&g->ccb);
+                g->ccb_state = 0;
+            }
+            if (ccb_build(GL.rp, GL.col, GL.n, nb, S, &g->ccb, s) == cudaSuccess) {
+                g->ccb_state = 1;
+                *ccb = true;
+                return nb;
+            }
+            cudaGetLastError();
+            g->ccb_state = -1;   // memory short: per-row offsets instead
+        }
+    }
+    if (g->cbo_nb != nb) {
+        if (g->cbo) {
+            cudaStreamSynchronize(s);
+            dev_free(g->cbo);
+            g->cbo = nullptr;
+            g->cbo_nb = 0;
+        }
+        // n x (nb - 1) block offsets: if they do not fit, pull unblocked (same result, more L2 misses)
+        if (dev_alloc(&g->cbo, sizeof(uint32_t) * (size_t)GL.n * (size_t)(nb - 1), s) != cudaSuccess) {
+            cudaGetLastError();
+            g->cbo = nullptr;
+            return 1;
+        }
+        launch_cc_block_offsets(GL.rp, GL.col, GL.n, nb, S, g->cbo, s);
+        g->cbo_nb = nb;
+    }
+    return nb;
+}
+static void cc_pull_blocked(sg_graph *g, const GraphView &GL, int nb, bool ccb, int32_t *label, uint64_t *out_bits,
+                            DevStats *st, cudaStream_t s) {
+    for (int b = 0; b < nb; b++) {
+        if (ccb)
+            launch_pull_ccb(GL, label, out_bits, st, g->ccb.off + (size_t)b * (size_t)(GL.n + 1),
+                            g->ccb.col + g->ccb.h_base[b], b, s);
+        else
+            launch_pull_cc_block(GL, label, out_bits, st, g->cbo, nb, b, s);
+    }
+}
+
 // ---- SSSP / CC over the 1-D destination partition (xchg.cuh) ------------------
 // Every rank holds the replicated value array (arena vals) and frontier; a superstep = the local
 // advance over the push block (SSSP relax / CC push: atomicMin on owned destinations only) or the
@@ -1543,29 +1607,8 @@ static int run_value_part(sg_graph *g, bool cc, int32_t src, uint32_t *result, c
     uint32_t *vals = A->vals;
     if (!ws->dist_old) CK(cudaMalloc(&ws->dist_old, sizeof(uint32_t) * (size_t)(G.n + 4)));
     // label-blocked pull over the owned rows (CC, as run_cc)
-    int cc_nb = 1;
-    if (cc && o.direction != SG_DIR_PUSH) {
-        const long long lblock = (long long)env_or("SG_CC_LBLOCK_KB", 32768) << 10;
-        cc_nb = (int)(((long long)G.n * 4 + lblock - 1) / (lblock > 0 ? lblock : 1));
-        if (cc_nb < 1 || lblock <= 0) cc_nb = 1;
-        if (cc_nb > 64) cc_nb = 64;
-        if (cc_nb > 1 && g->cbo_nb != cc_nb) {
-            if (g->cbo) {
-                CK(cudaStreamSynchronize(s));
-                dev_free(g->cbo);
-                g->cbo = nullptr;
-                g->cbo_nb = 0;
-            }
-            if (dev_alloc(&g->cbo, sizeof(uint32_t) * (size_t)G.n * (size_t)(cc_nb - 1), s) != cudaSuccess) {
-                cudaGetLastError();
-                g->cbo = nullptr;
-            } else {
-                launch_cc_block_offsets(g->vl.rp, g->vl.col, G.n, cc_nb, (G.n + cc_nb - 1) / cc_nb, g->cbo, s);
-                g->cbo_nb = cc_nb;
-            }
-        }
-        if (g->cbo_nb != cc_nb) cc_nb = 1;
-    }
+    bool use_ccb = false;
+    const int cc_nb = cc ? cc_blocks(g, g->vl, o.direction, s, &use_ccb) : 1;
     CK(cudaEventRecord(ws->ev0, s));
     if (cc) {
         launch_iota_i32(reinterpret_cast<int32_t *>(vals), G.n, s);
@@ -1592,8 +1635,7 @@ static int run_value_part(sg_graph *g, bool cc, int32_t src, uint32_t *result, c
         const bool pull = cc && (o.direction == SG_DIR_PULL ||
                                  (o.direction == SG_DIR_AUTO && (double)ws->h_st[in_idx].mf * 4.0 > (double)g->nnz_global));
         if (pull && cc_nb > 1) {
-            for (int b = 0; b < cc_nb; b++)
-                launch_pull_cc_block(g->vl, reinterpret_cast<int32_t *>(vals), out->bits, in->st, g->cbo, cc_nb, b, s);
+            cc_pull_blocked(g, g->vl, cc_nb, use_ccb, reinterpret_cast<int32_t *>(vals), out->bits, in->st, s);
         } else if (pull) {
             launch_pull_cc(g->vl, reinterpret_cast<int32_t *>(vals), out->bits, out->summ, in->st, s);
         } else {
@@ -1779,30 +1821,8 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     Workspace *ws = g->ws;
     L2Pin pin(label, sizeof(int32_t) * (size_t)G.n, s);   // labels are probed once per arc: keep them in L2
     // label blocks for the pull step: labels of one block (<= SG_CC_LBLOCK_KB) stay in L2
-    const long long lblock = (long long)env_or("SG_CC_LBLOCK_KB", 32768) << 10;
-    int cc_nb = (int)(((long long)G.n * 4 + lblock - 1) / (lblock > 0 ? lblock : 1));
-    if (cc_nb < 1 || lblock <= 0) cc_nb = 1;
-    if (cc_nb > 64) cc_nb = 64;
-    if (!g->sorted) cc_nb = 1;   // block offsets binary-search sorted rows
-    if (cc_nb > 1 && o.direction != SG_DIR_PUSH && (g->cbo_nb != cc_nb)) {
-        if (g->cbo) {
-            CK(cudaStreamSynchronize(s));
-            dev_free(g->cbo);
-            g->cbo = nullptr;
-            g->cbo_nb = 0;
-        }
-        // n x (nb - 1) block offsets: if they do not fit, pull unblocked (same result, more L2 misses)
-        const int64_t S = (G.n + cc_nb - 1) / cc_nb;
-        if (dev_alloc(&g->cbo, sizeof(uint32_t) * (size_t)G.n * (size_t)(cc_nb - 1), s) != cudaSuccess) {
-            cudaGetLastError();
-            g->cbo = nullptr;
-            cc_nb = 1;
-        } else {
-            launch_cc_block_offsets(G.rp, G.col, G.n, cc_nb, S, g->cbo, s);
-            g->cbo_nb = cc_nb;
-        }
-    }
-    if (cc_nb > 1 && g->cbo_nb != cc_nb) cc_nb = 1;
+    bool use_ccb = false;
+    const int cc_nb = cc_blocks(g, G, o.direction, s, &use_ccb);
     CK(cudaEventRecord(ws->ev0, s));
     launch_iota_i32(label, G.n, s);
     sg_frontier *in = &ws->fr[0], *out = &ws->fr[1];
@@ -1821,7 +1841,7 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
         const bool pull = o.direction == SG_DIR_PULL ||
                           (o.direction == SG_DIR_AUTO && (double)ws->h_st[in_idx].mf * 4.0 > (double)G.nnz);
         if (pull && cc_nb > 1) {   // label-blocked pull: one pass per L2-sized label block
-            for (int b = 0; b < cc_nb; b++) launch_pull_cc_block(G, label, out->bits, in->st, g->cbo, cc_nb, b, s);
+            cc_pull_blocked(g, G, cc_nb, use_ccb, label, out->bits, in->st, s);
             launch_rebuild_summary(out->bits, out->summ, G.nw1, G.nw2, s);
             pull_steps++;
         } else if (pull) {

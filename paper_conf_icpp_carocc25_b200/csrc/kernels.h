@@ -2,6 +2,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <vector>
 #include "common.cuh"
 
 namespace sg {
@@ -140,6 +141,25 @@ void launch_cc_block_offsets(const int64_t *rp, const int32_t *col, int64_t n, i
                              cudaStream_t s);
 void launch_pull_cc_block(const GraphView &g, int32_t *label, uint64_t *out_bits, DevStats *st, const uint32_t *cbo,
                           int nb, int b, cudaStream_t s);
+// pull_cc.cu — block-major arc copy for the label-blocked CC pull: block b holds, for every v,
+// v's neighbours in [b*S, (b+1)*S) contiguously at col[h_base[b] + off[b*(n+1) + v] ..)
+struct CcBlocks {
+    int nb = 0;
+    int64_t S = 0;
+    uint32_t *off = nullptr;       // [nb][n+1] offsets relative to the block's base
+    int64_t *base = nullptr;       // [nb+1] device copy of h_base
+    int32_t *col = nullptr;        // block-major arcs (+64 B padding)
+    int64_t total = 0;
+    std::vector<int64_t> h_base;
+};
+cudaError_t ccb_build(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, CcBlocks *out, cudaStream_t s);
+void ccb_free(CcBlocks *B);
+void launch_ccb_count(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, uint32_t *cnt, cudaStream_t s);
+void launch_ccb_fill(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, const uint32_t *off,
+                     const int64_t *base, int32_t *out, cudaStream_t s);
+// one label-blocked pull pass over block b (off = off[b], bcol = col + h_base[b])
+void launch_pull_ccb(const GraphView &g, int32_t *label, uint64_t *out_bits, DevStats *st, const uint32_t *off,
+                     const int32_t *bcol, int b, cudaStream_t s);
 // pull_cc.cu — pull label-propagation step (dense CC supersteps)
 void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint64_t *out_summ, DevStats *st,
                     cudaStream_t s);

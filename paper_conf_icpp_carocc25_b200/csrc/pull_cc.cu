@@ -8,6 +8,9 @@
 // propagation.  One warp owns one word (lane l: vertices 64w+l and 64w+32+l), so the output
 // frontier word (vertices whose label decreased) is written without atomics.  The fixed point
 // (component minimum, reading C13) is the same; tested bit-exact against union-find.
+#include <cub/device/device_scan.cuh>
+#include <vector>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -215,6 +218,188 @@ void launch_pull_cc(const GraphView &g, int32_t *label, uint64_t *out_bits, uint
     if (blocks < 1) blocks = 1;
     note_launch();
     k_pull_cc<<<(int)blocks, CCP_THREADS, 0, s>>>(g, label, out_bits, out_summ, st);
+}
+
+
+// ---- block-major arc copy for the label-blocked pull (CcBlocks) ----------------------------
+// The cbo form above reads, per pass, each row's part into block b from the row-major col_idx:
+// ~8 arcs of a 25-arc row, so most parts straddle two 32-B sectors and a pass moves ~2x its
+// arcs' bytes (ncu at config 3: 2.8 GB per pass, 8.4 GB per pull step for 2.1 GB of col_idx).
+// Here the arcs are copied once per graph into block-major order: block b = for every v the
+// neighbours of v inside [b*S, (b+1)*S), contiguous, with u32 offsets off[b][v] (relative to the
+// block's base).  A pass then streams exactly its block's arcs.
+__global__ void k_ccb_count(const int64_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t n, int nb,
+                            int64_t S, uint32_t *__restrict__ cnt) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += stride) {
+        const int64_t s0 = rp[v], e0 = rp[v + 1];
+        int64_t prev = s0;
+        for (int b = 0; b < nb; b++) {
+            int64_t lo = prev, hi = e0;
+            const int64_t key = (int64_t)(b + 1) * S;   // lower_bound of the next block's first id
+            if (b == nb - 1) {
+                lo = e0;
+            } else {
+                while (lo < hi) {
+                    const int64_t mid = (lo + hi) >> 1;
+                    if ((int64_t)col[mid] < key) lo = mid + 1;
+                    else hi = mid;
+                }
+            }
+            cnt[(size_t)b * (n + 1) + v] = (uint32_t)(lo - prev);
+            prev = lo;
+        }
+    }
+}
+// warp per row: arc i of row v (sorted) goes to block b = col / S at off[b][v] + its rank in the part
+__global__ void k_ccb_fill(const int64_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t n, int nb,
+                           int64_t S, const uint32_t *__restrict__ off, const int64_t *__restrict__ base,
+                           int32_t *__restrict__ out) {
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = gw; v < n; v += nwarps) {
+        const int64_t s0 = rp[v], e0 = rp[v + 1];
+        for (int64_t i = s0 + lane; i < e0; i += 32) {
+            const int32_t c = col[i];
+            const int b = (int)((int64_t)c / S);
+            // rank of arc i inside its part = i - (first arc of the part); parts are in block order
+            int64_t first = s0;
+            for (int bb = 0; bb < b; bb++)
+                first += off[(size_t)bb * (n + 1) + v + 1] - off[(size_t)bb * (n + 1) + v];
+            out[base[b] + off[(size_t)b * (n + 1) + v] + (i - first)] = c;
+        }
+    }
+}
+void launch_ccb_count(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, uint32_t *cnt,
+                      cudaStream_t s) {
+    int64_t blocks = (n + 255) / 256;
+    if (blocks > num_sms() * 16) blocks = num_sms() * 16;
+    note_launch();
+    k_ccb_count<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(rp, col, n, nb, S, cnt);
+}
+void launch_ccb_fill(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, const uint32_t *off,
+                     const int64_t *base, int32_t *out, cudaStream_t s) {
+    int64_t blocks = (n * 32 + 255) / 256;
+    if (blocks > num_sms() * 16) blocks = num_sms() * 16;
+    note_launch();
+    k_ccb_fill<<<(int)(blocks < 1 ? 1 : blocks), 256, 0, s>>>(rp, col, n, nb, S, off, base, out);
+}
+
+// one pass of the blocked pull over the block-major copy (same mapping as k_pull_cc_block)
+__global__ void __launch_bounds__(CCP_THREADS)
+k_pull_ccb(GraphView g, int32_t *__restrict__ label, uint64_t *__restrict__ out_bits, DevStats *st,
+           const uint32_t *__restrict__ off, const int32_t *__restrict__ bcol, int b) {
+    __shared__ unsigned long long s_arcs[CCP_THREADS / 32];
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    unsigned long long arcs = 0;
+    for (int64_t w = g.w1_lo + gw; w < g.w1_hi; w += nwarps) {
+        const int64_t va = w * 64 + lane, vb = va + 32;
+        const bool act_a = va < g.n, act_b = vb < g.n;
+        const int64_t sa = act_a ? __ldg(off + va) : 0, ea = act_a ? __ldg(off + va + 1) : 0;
+        const int64_t sb = act_b ? __ldg(off + vb) : 0, eb = act_b ? __ldg(off + vb + 1) : 0;
+        const int32_t own_a = act_a ? label[va] : 0x7fffffff, own_b = act_b ? label[vb] : 0x7fffffff;
+        int32_t ma = own_a, mb = own_b;
+        arcs += (unsigned long long)((ea - sa) + (eb - sb));
+        for (int64_t ia = sa, ib = sb; ia < ea || ib < eb; ia += 4, ib += 4) {
+            int32_t c[8];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                c[k] = (ia + k < ea) ? __ldg(bcol + ia + k) : -1;
+                c[4 + k] = (ib + k < eb) ? __ldg(bcol + ib + k) : -1;
+            }
+            int32_t l[8];
+#pragma unroll
+            for (int k = 0; k < 8; k++) l[k] = c[k] >= 0 ? label[c[k]] : 0x7fffffff;
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                ma = min(ma, l[k]);
+                mb = min(mb, l[4 + k]);
+            }
+        }
+        const bool ca = ma < own_a, cb = mb < own_b;
+        if (ca) label[va] = ma;
+        if (cb) label[vb] = mb;
+        const uint64_t nbits = (uint64_t)__ballot_sync(0xffffffffu, ca) | ((uint64_t)__ballot_sync(0xffffffffu, cb) << 32);
+        if (lane == 0) {
+            if (b == 0) out_bits[w] = nbits;
+            else if (nbits) out_bits[w] |= nbits;
+        }
+    }
+    arcs = warp_sum(arcs);
+    if (lane == 0) s_arcs[threadIdx.x >> 5] = arcs;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long t = 0;
+        for (int i = 0; i < CCP_THREADS / 32; i++) t += s_arcs[i];
+        if (t) atomicAdd(&st->arcs, t);
+    }
+}
+cudaError_t ccb_build(const int64_t *rp, const int32_t *col, int64_t n, int nb, int64_t S, CcBlocks *out,
+                      cudaStream_t s) {
+    CcBlocks B;
+    B.nb = nb;
+    B.S = S;
+    uint32_t *cnt = nullptr;
+    void *tmp = nullptr;
+    size_t tb = 0;
+    const size_t per = (size_t)(n + 1);
+    cudaError_t e = dev_alloc(&cnt, sizeof(uint32_t) * per * nb, s);
+    if (e == cudaSuccess) e = dev_alloc(&B.off, sizeof(uint32_t) * per * nb, s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(cnt, 0, sizeof(uint32_t) * per * nb, s);
+    if (e == cudaSuccess) {
+        launch_ccb_count(rp, col, n, nb, S, cnt, s);
+        e = cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, B.off, (int64_t)per, s);
+    }
+    if (e == cudaSuccess) e = dev_alloc(&tmp, tb, s);
+    for (int b = 0; b < nb && e == cudaSuccess; b++) {
+        note_launch();
+        e = cub::DeviceScan::ExclusiveSum(tmp, tb, cnt + (size_t)b * per, B.off + (size_t)b * per, (int64_t)per, s);
+    }
+    std::vector<uint32_t> tot(nb, 0);
+    for (int b = 0; b < nb && e == cudaSuccess; b++)
+        e = cudaMemcpyAsync(&tot[b], B.off + (size_t)b * per + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    std::vector<int64_t> base(nb + 1, 0);
+    for (int b = 0; b < nb; b++) base[b + 1] = base[b] + tot[b];
+    B.total = base[nb];
+    if (e == cudaSuccess) e = dev_alloc(&B.base, sizeof(int64_t) * (size_t)(nb + 1), s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(B.base, base.data(), sizeof(int64_t) * (size_t)(nb + 1), cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = dev_alloc(&B.col, sizeof(int32_t) * (size_t)B.total + 64, s);
+    if (e == cudaSuccess) {
+        launch_ccb_fill(rp, col, n, nb, S, B.off, B.base, B.col, s);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (cnt) cudaFreeAsync(cnt, s);
+    if (tmp) cudaFreeAsync(tmp, s);
+    B.h_base = base;
+    if (e != cudaSuccess) {
+        ccb_free(&B);
+        return e;
+    }
+    *out = B;
+    return cudaSuccess;
+}
+void ccb_free(CcBlocks *B) {
+    dev_free(B->off);
+    dev_free(B->base);
+    dev_free(B->col);
+    B->off = nullptr;
+    B->base = nullptr;
+    B->col = nullptr;
+    B->nb = 0;
+}
+
+void launch_pull_ccb(const GraphView &g, int32_t *label, uint64_t *out_bits, DevStats *st, const uint32_t *off,
+                     const int32_t *bcol, int b, cudaStream_t s) {
+    int64_t blocks = ((g.w1_hi - g.w1_lo) * 32 + CCP_THREADS - 1) / CCP_THREADS;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_pull_ccb<<<(int)blocks, CCP_THREADS, 0, s>>>(g, label, out_bits, st, off, bcol, b);
 }
 
 }  // namespace sg
