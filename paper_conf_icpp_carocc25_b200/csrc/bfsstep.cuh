@@ -106,6 +106,42 @@ __device__ __forceinline__ uint32_t bfs_decide(BfsCtrl *c, const DevStats *st, u
     return !go ? SK_STOP : (c->pull ? SK_PULL : (sweep ? SK_SWEEP : (sparse ? SK_SPARSE : SK_PUSH)));
 }
 
+// Decision of a graph-driven SSSP / CC superstep: stop on an empty frontier (or the cap), else
+// the next superstep's direction (CC AUTO: pull when m_f > nnz/4, the host loop's rule); the IF
+// handles of the next input buffer's half get it, only changed handles are set.  One thread.
+__device__ __forceinline__ void val_decide(ValCtrl *c, const DevStats *st, unsigned long long prev_arcs,
+                                           DevStats *zero_prev, int next_in, int first) {
+    const volatile DevStats *vst = st;
+    if (!first) {
+        if (c->pull) c->arcs_pulled += prev_arcs;
+        else c->arcs_pushed += prev_arcs;
+    }
+    const unsigned long long count = vst->count;
+    bool go = count > 0;
+    if (go && c->iters >= (unsigned long long)c->max_iters) {
+        c->overflow = 1;
+        go = false;
+    }
+    bool pull = false;
+    if (go) {
+        pull = c->cc && (c->direction == 2 || (c->direction == 0 && (double)vst->mf * 4.0 > (double)c->nnz));
+        c->pull = pull;
+        if (pull) c->pull_steps++;
+        else c->push_steps++;
+        c->iters++;
+    }
+    uint32_t want = go ? 0x100u : 0u;
+    if (go) want |= 1u << (2 * (pull ? 1 : 0) + next_in);
+    const uint32_t diff = want ^ c->hmask;
+    const unsigned long long *hs[2] = {c->hpush, c->hpull};
+    for (int k = 0; k < 2; k++)
+        for (int b = 0; b < 2; b++)
+            if ((diff >> (2 * k + b)) & 1u) bfs_set_cond(hs[k][b], (want >> (2 * k + b)) & 1u);
+    if (diff & 0x100u) bfs_set_cond(c->hl, go);
+    c->hmask = want;
+    if (zero_prev) *zero_prev = DevStats{};
+}
+
 // Emit a block's slice of the output frontier: `S` = the block's layer-2 words (in shared
 // memory, nS of them, the first = layer-2 word sw0; words at or past w2_hi are not this rank's
 // and are skipped), written as is; their set bits are appended to the word list with one atomic
@@ -181,7 +217,7 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
         }
         if (c && in_st) atomicAdd(&in_st->arcs, c);
         s_last = false;
-        if (o.ctrl || part) {
+        if (o.ctrl || o.vctrl || part) {
             if (part) __threadfence_system();   // this CTA's peer stores before the barrier's epoch
             else __threadfence();
             s_last = atomicAdd(o.done, 1u) == gridDim.x - 1;
@@ -210,6 +246,8 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
             if (o.ctrl) bfs_decide(o.ctrl, o.st, prev_arcs, nullptr, o.half ^ 1, 0);
         } else if (o.ctrl) {
             bfs_decide(o.ctrl, o.st, prev_arcs, o.prev, o.half ^ 1, 0);
+        } else if (o.vctrl) {
+            val_decide(o.vctrl, o.st, prev_arcs, o.prev, o.half ^ 1, 0);
         }
     }
 }

@@ -124,6 +124,16 @@ struct Workspace {
     unsigned int *bfs_done = nullptr;   // CTA completion counter of the BFS output kernels (self-resetting)
     unsigned int *gbar = nullptr;       // grid barrier of the sparse superstep kernel (2 u32)
     unsigned long long hnd[9] = {};     // conditional handles of bfs_graph (loop, push/pull/sweep/sparse x 2)
+    // graph-driven SSSP (index 0) / CC (index 1): one graph per (result buffer, tiers, CC blocks)
+    struct VGraph {
+        cudaGraph_t graph = nullptr;
+        cudaGraphExec_t exec = nullptr;
+        void *result = nullptr;
+        int32_t heavy = 0, small = 0, nb = 0;
+        bool ccb = false;
+        unsigned long long h[5] = {};   // loop, push x2, pull x2
+    } vg[2];
+    ValCtrl *vctrl = nullptr, *h_vctrl = nullptr;
     cudaGraph_t bfs_graph = nullptr;
     cudaGraphExec_t bfs_exec = nullptr;
     uint32_t *bfs_level = nullptr;
@@ -307,6 +317,12 @@ static void free_ws(Workspace *ws) {
         cudaFreeHost(ws->h_bcb);
     }
     if (ws->cap_stream) cudaStreamDestroy(ws->cap_stream);
+    for (auto &v : ws->vg) {
+        if (v.exec) cudaGraphExecDestroy(v.exec);
+        if (v.graph) cudaGraphDestroy(v.graph);
+    }
+    cudaFree(ws->vctrl);
+    cudaFreeHost(ws->h_vctrl);
     cudaFree(ws->ctrl);
     cudaFree(ws->bfs_done);
     cudaFree(ws->gbar);
@@ -1585,6 +1601,159 @@ static void cc_pull_blocked(sg_graph *g, const GraphView &GL, int nb, bool ccb, 
     }
 }
 
+// ---- graph-driven SSSP / CC (no host round trip per superstep) -----------------------------
+// WHILE { half 0 | half 1 }; half h = IF(push_h) [push kernels + k_value_diff] and, for CC,
+// IF(pull_h) [label-blocked pull passes + k_value_diff]; k_value_diff's last CTA decides the next
+// superstep (val_decide).  The value array doubles as the functor state; old = ws->dist_old.
+static int build_val_graph(sg_graph *g, bool cc, uint32_t *val, Tiers t, int nb, bool ccb) {
+    Workspace *ws = g->ws;
+    const GraphView &G = g->v;
+    Workspace::VGraph &V = ws->vg[cc ? 1 : 0];
+    if (V.exec) cudaGraphExecDestroy(V.exec);
+    if (V.graph) cudaGraphDestroy(V.graph);
+    V.exec = nullptr;
+    V.graph = nullptr;
+    if (!ws->cap_stream) CK(cudaStreamCreateWithFlags(&ws->cap_stream, cudaStreamNonBlocking));
+    if (!ws->vctrl) {
+        CK(cudaMalloc(&ws->vctrl, sizeof(ValCtrl)));
+        CK(cudaMallocHost(&ws->h_vctrl, sizeof(ValCtrl)));
+    }
+    if (!ws->dist_old) CK(cudaMalloc(&ws->dist_old, sizeof(uint32_t) * (size_t)(G.n + 4)));
+    cudaStream_t cs = ws->cap_stream;
+    cudaGraph_t root;
+    CK(cudaGraphCreate(&root, 0));
+    V.graph = root;
+    cudaGraphConditionalHandle hl, hpush[2], hpull[2] = {};
+    CK(cudaGraphConditionalHandleCreate(&hl, root, 0, cudaGraphCondAssignDefault));
+    for (int i = 0; i < 2; i++) {
+        CK(cudaGraphConditionalHandleCreate(&hpush[i], root, 0, cudaGraphCondAssignDefault));
+        if (cc) CK(cudaGraphConditionalHandleCreate(&hpull[i], root, 0, cudaGraphCondAssignDefault));
+    }
+    sg_frontier *F[2] = {&ws->fr[0], &ws->fr[1]};
+    std::vector<cudaGraphNode_t> leaves;
+    TRY(capture_begin(cs, root, {}));
+    CK(cudaMemsetAsync(F[0]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
+    CK(cudaMemsetAsync(F[0]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
+    CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), cs));
+    if (cc) {
+        launch_iota_i32(reinterpret_cast<int32_t *>(val), G.n, cs);
+        CK(cudaMemcpyAsync(ws->dist_old, val, sizeof(uint32_t) * (size_t)G.n, cudaMemcpyDeviceToDevice, cs));
+        launch_fill_all(F[0]->bits, F[0]->summ, G.n, G.nw1, G.nw2, cs);   // advance::vertices
+        launch_compact(F[0]->summ, G.nw2, F[0]->offsets, F[0]->st, cs);
+        launch_frontier_stats(G, F[0]->bits, F[0]->st, cs);
+        launch_val_first(ws->vctrl, F[0]->st, cs);
+    } else {
+        CK(cudaMemsetAsync(val, 0xFF, sizeof(uint32_t) * (size_t)G.n, cs));
+        CK(cudaMemsetAsync(ws->dist_old, 0xFF, sizeof(uint32_t) * (size_t)G.n, cs));
+        launch_val_seed(ws->vctrl, val, ws->dist_old, F[0]->bits, F[0]->summ, F[0]->offsets, F[0]->st, cs);
+    }
+    TRY(capture_end(cs, leaves));
+    cudaGraphNode_t wnode;
+    cudaGraph_t body;
+    TRY(add_cond(root, leaves, hl, cudaGraphCondTypeWhile, &wnode, &body));
+    std::vector<cudaGraphNode_t> deps;
+    for (int half = 0; half < 2; half++) {
+        sg_frontier *in = F[half], *out = F[half ^ 1];
+        BfsOut bo{};
+        bo.out_bits = out->bits;
+        bo.out_summ = out->summ;
+        bo.out_offsets = out->offsets;
+        bo.st = out->st;
+        bo.prev = in->st;
+        bo.done = ws->bfs_done;
+        bo.half = half;
+        bo.vctrl = ws->vctrl;
+        cudaGraphNode_t n_push, n_pull = nullptr;
+        cudaGraph_t b_push, b_pull = nullptr;
+        TRY(add_cond(body, deps, hpush[half], cudaGraphCondTypeIf, &n_push, &b_push));
+        if (cc) TRY(add_cond(body, deps, hpull[half], cudaGraphCondTypeIf, &n_pull, &b_pull));
+        PushLaunch L = push_launch(g, in, t, -1);
+        L.batch = t.cf;   // 0: coarsening factor from the device-side count
+        TRY(capture_begin(cs, b_push, {}));
+        if (cc) {
+            launch_push_cc(L, CcArgs{reinterpret_cast<int32_t *>(val), nullptr, nullptr}, cs);
+        } else {
+            SsspArgs sa{val, nullptr, nullptr};
+            sa.diff = 1;
+            launch_push_sssp(L, sa, cs);
+        }
+        launch_value_diff(G, val, ws->dist_old, bo, cc ? 1 : 0, cs);
+        TRY(capture_end(cs, leaves));
+        if (cc) {
+            TRY(capture_begin(cs, b_pull, {}));
+            if (nb > 1) cc_pull_blocked(g, g->vl, nb, ccb, reinterpret_cast<int32_t *>(val), out->bits, in->st, cs);
+            else launch_pull_cc(g->vl, reinterpret_cast<int32_t *>(val), out->bits, out->summ, in->st, cs);
+            launch_value_diff(G, val, ws->dist_old, bo, 1, cs);
+            TRY(capture_end(cs, leaves));
+        }
+        deps = {n_push};
+        if (n_pull) deps.push_back(n_pull);
+    }
+    CK(cudaGraphInstantiate(&V.exec, root, 0));
+    V.result = val;
+    V.heavy = t.heavy;
+    V.small = t.small;
+    V.nb = nb;
+    V.ccb = ccb;
+    V.h[0] = (unsigned long long)hl;
+    for (int i = 0; i < 2; i++) {
+        V.h[1 + i] = (unsigned long long)hpush[i];
+        V.h[3 + i] = cc ? (unsigned long long)hpull[i] : 0ull;
+    }
+    return SG_OK;
+}
+
+static int run_value_graph(sg_graph *g, bool cc, int32_t src, uint32_t *val, const sg_opts &o, int64_t max_iters,
+                           sg_stats *stats) {
+    Workspace *ws = g->ws;
+    cudaStream_t s = stream_of(&o);
+    Tiers t = tiers_from(&o);
+    t.seg = 0;
+    TRY(ensure_heavy(g, t.heavy));
+    bool use_ccb = false;
+    const int nb = cc ? cc_blocks(g, g->vl, o.direction, s, &use_ccb) : 1;
+    Workspace::VGraph &V = ws->vg[cc ? 1 : 0];
+    if (!V.exec || V.result != val || V.heavy != t.heavy || V.small != t.small || V.nb != nb || V.ccb != use_ccb)
+        TRY(build_val_graph(g, cc, val, t, nb, use_ccb));
+    ValCtrl &c = *ws->h_vctrl;
+    memset(&c, 0, sizeof c);
+    c.max_iters = max_iters;
+    c.nnz = g->nnz_global;
+    c.cc = cc ? 1u : 0u;
+    c.direction = (uint32_t)o.direction;
+    c.src = src;
+    c.hl = V.h[0];
+    for (int i = 0; i < 2; i++) {
+        c.hpush[i] = V.h[1 + i];
+        c.hpull[i] = V.h[3 + i];
+    }
+    CK(cudaEventRecord(ws->ev0, s));
+    CK(cudaMemcpyAsync(ws->vctrl, ws->h_vctrl, sizeof(ValCtrl), cudaMemcpyHostToDevice, s));
+    CK(cudaGraphLaunch(V.exec, s));
+    CK(cudaMemcpyAsync(ws->h_vctrl, ws->vctrl, sizeof(ValCtrl), cudaMemcpyDeviceToHost, s));
+    CK(cudaEventRecord(ws->ev1, s));
+    CK(cudaEventSynchronize(ws->ev1));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
+    CK(cudaGetLastError());
+    if (c.overflow) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
+    {   // kernels the graph executed: prologue (SSSP 1, CC 4) + per push step 3, per pull step nb + 1
+        const long long k = (cc ? 4 : 1) + 3 * (long long)c.push_steps + (long long)(nb + 1) * (long long)c.pull_steps;
+        for (long long i = 0; i < k; i++) note_launch();
+    }
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->iterations = (int64_t)c.iters;
+        stats->push_steps = (int64_t)c.push_steps;
+        stats->pull_steps = (int64_t)c.pull_steps;
+        stats->arcs_pushed = (int64_t)c.arcs_pushed;
+        stats->arcs_pulled = (int64_t)c.arcs_pulled;
+        stats->reached = cc ? g->v.n : -1;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
 // ---- SSSP / CC over the 1-D destination partition (xchg.cuh) ------------------
 // Every rank holds the replicated value array (arena vals) and frontier; a superstep = the local
 // advance over the push block (SSSP relax / CC push: atomicMin on owned destinations only) or the
@@ -1705,6 +1874,9 @@ SG_API int run_sssp(const sg_graph *gc, int32_t src, uint32_t *dist, const sg_op
         if (o.sssp_delta > 0) return fail(SG_ERR_UNSUPPORTED, "delta-stepping runs on single-GPU graphs only");
         return run_value_part(g, false, src, dist, o, stats);
     }
+    // default: device-driven loop (CUDA graph); host_loop = 1 keeps the host-driven one below
+    if (!o.host_loop && o.sssp_delta <= 0 && env_or("SG_SSSP_DIFF", 1) != 0)
+        return run_value_graph(g, false, src, dist, o, max_iters, stats);
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;
@@ -1816,6 +1988,8 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     cudaStream_t s = stream_of(&o);
     TRY(ensure_ws(g));
     if (g->ar) return run_value_part(g, true, 0, reinterpret_cast<uint32_t *>(label), o, stats);
+    // default: device-driven loop (CUDA graph); host_loop = 1 keeps the host-driven one below
+    if (!o.host_loop) return run_value_graph(g, true, 0, reinterpret_cast<uint32_t *>(label), o, max_iters, stats);
     const Tiers t = tiers_from(&o);
     TRY(ensure_heavy(g, t.heavy));
     Workspace *ws = g->ws;

@@ -80,6 +80,20 @@ struct DevStats {
 
 constexpr int SG_TRACE_STEPS = 48;
 
+// Device-resident state of a graph-driven SSSP / CC run (vloop: WHILE { half 0 | half 1 }, per
+// half an IF(push) and an IF(pull) node; the output kernel's last CTA decides).
+struct ValCtrl {
+    unsigned long long iters, push_steps, pull_steps, arcs_pushed, arcs_pulled;
+    long long max_iters, nnz;
+    uint32_t overflow;
+    uint32_t cc;             // 1: CC (pull when the frontier's arcs exceed nnz/4 in AUTO), 0: SSSP (push)
+    uint32_t direction;      // SG_DIR_*
+    uint32_t pull;           // direction of the superstep being launched
+    uint32_t hmask;          // current IF handle values (bit 2k+b: kind k (0 push, 1 pull) of buffer b; bit 8 loop)
+    int32_t src;             // SSSP source (the prologue kernel seeds it)
+    unsigned long long hl, hpush[2], hpull[2];
+};
+
 // Device-resident state of a graph-driven BFS (written by k_bfs_decide, read back once per run).
 struct BfsCtrl {
     unsigned long long iters, push_steps, pull_steps, arcs_pushed, arcs_pulled, reached;

@@ -99,6 +99,31 @@ void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *b
     k_bfs_prologue<<<(int)blocks, 256, 0, s>>>(c, n, deg8, bits, summ, offsets, st, visited, vis_old, x);
 }
 
+__global__ void k_val_first(ValCtrl *c, const DevStats *st) { val_decide(c, st, 0ull, nullptr, 0, 1); }
+void launch_val_first(ValCtrl *c, const DevStats *st, cudaStream_t s) {
+    note_launch();
+    k_val_first<<<1, 1, 0, s>>>(c, st);
+}
+// SSSP prologue of the graph-driven loop (dist and dist_old were set to INF): source from the
+// control block, dist[src] = dist_old[src] = 0, input frontier {src} with its word list, decision
+__global__ void k_val_seed(ValCtrl *c, uint32_t *dist, uint32_t *dist_old, uint64_t *bits, uint64_t *summ,
+                           uint32_t *offsets, DevStats *st) {
+    const int32_t src = c->src;
+    dist[src] = 0u;
+    dist_old[src] = 0u;
+    bits[src >> 6] = 1ull << (src & 63);
+    summ[src >> 12] = 1ull << ((src >> 6) & 63);
+    offsets[0] = (uint32_t)(src >> 6);
+    st->count = 1ull;
+    st->nf = 1ull;
+    val_decide(c, st, 0ull, nullptr, 0, 1);
+}
+void launch_val_seed(ValCtrl *c, uint32_t *dist, uint32_t *dist_old, uint64_t *bits, uint64_t *summ,
+                     uint32_t *offsets, DevStats *st, cudaStream_t s) {
+    note_launch();
+    k_val_seed<<<1, 1, 0, s>>>(c, dist, dist_old, bits, summ, offsets, st);
+}
+
 // Barrier across the ranks of a partition (one thread; xchg.cuh)
 __global__ void k_xbarrier(Xchg x) { xbarrier(x, 0ull, 0ull, 0ull, nullptr); }
 void launch_xbarrier(const Xchg &x, cudaStream_t s) {

@@ -104,7 +104,12 @@ struct BfsOut {
     int32_t half = 0;                 // graph mode: index (0/1) of the INPUT frontier buffer
     int32_t sparse = 0;               // 1: the superstep consumed (zeroed) its input (sparse.cu)
     int32_t pull_warp = 0;            // host loop: 1 = the pull runs warp-owned layer-2 words (graph mode: ctrl)
+    ValCtrl *vctrl = nullptr;         // graph-driven SSSP / CC: the last CTA runs val_decide
 };
+// device-driven SSSP / CC: the first decision (after the prologue compacted the input), one thread
+void launch_val_first(ValCtrl *c, const DevStats *st, cudaStream_t s);
+void launch_val_seed(ValCtrl *c, uint32_t *dist, uint32_t *dist_old, uint64_t *bits, uint64_t *summ,
+                     uint32_t *offsets, DevStats *st, cudaStream_t s);
 // pull.cu — bottom-up BFS step (direction-optimising, Beamer): writes its output `o`
 // itself (no k_bfs_diff after it); o.out_bits == NULL: marks visited only (k_bfs_diff after it)
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,

@@ -533,3 +533,28 @@ def test_bfs_fused_sparse_supersteps(sg, monkeypatch, make):
                 assert np.array_equal(sg.as_u32(lv), ref), (s, arcs, d)
             _, st = sg.run_bfs(G, int(s))
             assert (st.iterations, st.push_steps, st.pull_steps) == (st0.iterations, st0.push_steps, st0.pull_steps)
+
+
+@pytest.mark.parametrize("make", [lambda: gen.with_weights(gen.rmat(14, 16, permute=True), seed=2),
+                                  lambda: gen.with_weights(gen.lattice(120, 150, 0.6, seed=5), seed=3),
+                                  lambda: gen.with_weights(gen.gnm(50_000, 30_000, seed=4), seed=4)])
+def test_sssp_cc_graph_driven_equals_host_loop(sg, monkeypatch, make):
+    """The device-driven SSSP / CC loops (CUDA graph, val_decide) give the oracle's values, as the
+    host loop does, for every direction and with label-blocked CC pulls.  (Superstep counts are
+    not compared: with asynchronous relaxation, reading C12, a superstep's frontier depends on
+    the order its atomics land in.)"""
+    g = make()
+    G = load(sg, g)
+    for s in gen.sources(g, 2):
+        d, st = sg.run_sssp(G, int(s))
+        d2, st2 = sg.run_sssp(G, int(s), host_loop=True)
+        ref = oracle.sssp(g, int(s))
+        assert np.array_equal(sg.as_u32(d), ref) and np.array_equal(sg.as_u32(d2), ref)
+    ref = oracle.cc(g)
+    for kb in ("32768", "8"):
+        monkeypatch.setenv("SG_CC_LBLOCK_KB", kb)
+        for dr in (sg.SG_DIR_AUTO, sg.SG_DIR_PUSH, sg.SG_DIR_PULL):
+            lab, st = sg.run_cc(G, direction=dr)
+            lab2, st2 = sg.run_cc(G, direction=dr, host_loop=True)
+            assert np.array_equal(lab.cpu().numpy(), ref) and np.array_equal(lab2.cpu().numpy(), ref)
+            assert st.iterations >= 1 and st.push_steps + st.pull_steps == st.iterations
