@@ -200,6 +200,36 @@ def with_weights(g: CSR, seed: int = 1, wmax: int = 64) -> CSR:
     return g
 
 
+def _mix64(z: np.ndarray) -> np.ndarray:
+    """splitmix64 finaliser, vectorised (uint64, wrapping)."""
+    z = z.astype(np.uint64)
+    with np.errstate(over="ignore"):
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        z = z ^ (z >> np.uint64(31))
+    return z
+
+
+def orient(g: CSR, seed: int = 1, stream: int = 7) -> CSR:
+    """A directed graph from a symmetric one (SURVEY f4 test input): edge {u < v} keeps the arc
+    u -> v iff bit 0 of mix(mix(seed ^ stream << 56) + u*n + v) is set and v -> u iff bit 1 is
+    (so ~1/4 of the edges keep both arcs, ~1/4 neither).  Rows stay sorted; weights follow."""
+    rows = np.repeat(np.arange(g.n, dtype=np.int64), g.degrees())
+    cols = g.col_idx.astype(np.int64)
+    lo, hi = np.minimum(rows, cols), np.maximum(rows, cols)
+    with np.errstate(over="ignore"):
+        base = _mix64(np.array([np.uint64(seed) ^ (np.uint64(stream) << np.uint64(56))], dtype=np.uint64))[0]
+        h = _mix64(base + (lo * g.n + hi).astype(np.uint64))
+    bit = np.where(rows < cols, h & np.uint64(1), (h >> np.uint64(1)) & np.uint64(1)).astype(bool)
+    counts = np.bincount(rows[bit], minlength=g.n)
+    rp = np.zeros(g.n + 1, dtype=np.int64)
+    np.cumsum(counts, out=rp[1:])
+    out = CSR(n=g.n, row_ptr=rp, col_idx=np.ascontiguousarray(g.col_idx[bit]), name=g.name + "-directed")
+    if g.weights is not None:
+        out.weights = np.ascontiguousarray(g.weights[bit])
+    return out
+
+
 def sources(g: CSR, k: int, seed: int = 1, stream: int = 5, eligible: np.ndarray | None = None) -> np.ndarray:
     """First k distinct rnd(seed, stream, i) mod n with degree > 0 (reading C15), restricted to
     eligible[v] != 0 when a mask is given."""

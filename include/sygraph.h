@@ -52,7 +52,12 @@ enum { SG_MEM_HOST = 0, SG_MEM_DEVICE = 1 };          /* where input arrays live
  *   Without SG_F_VALIDATE row order is still checked (O(nnz), every load): a graph whose rows are
  *   not sorted loads, but its hub-segmented push tier, segment-major sweep and label-blocked CC
  *   pull (which binary-search sorted rows) are disabled for it; results stay exact.             */
-enum { SG_F_BORROW = 1, SG_F_VALIDATE = 2 };
+/*   SG_F_DIRECTED  the CSR holds out-arcs of a directed graph (§3.1 "CSR and CSC"; P:299
+ *                  directed datasets): the library builds the transpose (CSC, rows
+ *                  sorted) for pull steps, and a vertex with no in-arc is unreachable.  run_bfs /
+ *                  run_sssp / advance follow arc direction; run_cc / run_bc need a symmetric graph
+ *                  (SG_ERR_UNSUPPORTED); SG_F_VALIDATE skips the symmetry check; single GPU only. */
+enum { SG_F_BORROW = 1, SG_F_VALIDATE = 2, SG_F_DIRECTED = 4 };
 enum { SG_FN_BFS = 0, SG_FN_SSSP = 1, SG_FN_CC = 2, SG_FN_BC_SIGMA = 3 };   /* advance functors */
 enum { SG_DIR_AUTO = 0, SG_DIR_PUSH = 1, SG_DIR_PULL = 2 };                 /* BFS direction */
 

@@ -18,7 +18,7 @@ LIB_PATH = os.environ.get("SYGRAPH_LIB") or os.path.join(_PKG, "lib", "libsygrap
 
 SG_OK, SG_ERR_INVALID, SG_ERR_OOM, SG_ERR_CUDA, SG_ERR_NCCL, SG_ERR_UNSUPPORTED, SG_ERR_STATE = 0, -1, -2, -3, -4, -5, -6
 SG_MEM_HOST, SG_MEM_DEVICE = 0, 1
-SG_F_BORROW, SG_F_VALIDATE = 1, 2
+SG_F_BORROW, SG_F_VALIDATE, SG_F_DIRECTED = 1, 2, 4
 SG_FN_BFS, SG_FN_SSSP, SG_FN_CC, SG_FN_BC_SIGMA = 0, 1, 2, 3
 SG_DIR_AUTO, SG_DIR_PUSH, SG_DIR_PULL = 0, 1, 2
 INF32 = 0xFFFFFFFF
@@ -193,7 +193,8 @@ class Graph:
             pass
 
 
-def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None, borrow=False, comm=None) -> Graph:
+def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None, borrow=False, comm=None,
+                   directed=False) -> Graph:
     """row_ptr int64[n+1], col_idx int32[nnz], weights uint8[nnz] (numpy/host tensors or CUDA tensors).
     borrow (CUDA tensors only): keep the tensors' memory instead of copying (SG_F_BORROW); the
     returned Graph holds references to them.  comm (a Comm): collective partitioned load — this
@@ -207,7 +208,7 @@ def graph_load_csr(row_ptr, col_idx, weights=None, validate=False, stream=None, 
     if len(mems) != 1:
         raise ValueError("row_ptr, col_idx and weights must all be host or all be device arrays")
     h = ctypes.c_void_p()
-    flags = (SG_F_VALIDATE if validate else 0) | (SG_F_BORROW if borrow else 0)
+    flags = (SG_F_VALIDATE if validate else 0) | (SG_F_BORROW if borrow else 0) | (SG_F_DIRECTED if directed else 0)
     _check(load().graph_load_csr(n, nnz, rp, ci if nnz else None, w, m1, flags, _stream_ptr(stream),
                                  comm.handle if comm is not None else None, ctypes.byref(h)))
     G = Graph(h.value, n, nnz, weights is not None)

@@ -179,7 +179,10 @@ struct sg_graph {
     Arena *ar = nullptr;            // exchange arena (partitioned only)
     int nranks = 1, rank = 0;
     sg_comm *comm = nullptr;        // partitioned: graph_free is collective over it
-    int64_t n_iso = 0;              // isolated vertices (deg 0)
+    int64_t n_iso = 0;              // isolated vertices (deg 0; directed: in-degree 0)
+    bool directed = false;          // SG_F_DIRECTED: CSR = out-arcs, rpt / colt = the transpose (pull)
+    int64_t *rpt = nullptr;
+    int32_t *colt = nullptr;
 };
 static std::atomic<int> g_live_graphs{0};
 
@@ -546,7 +549,10 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
     if (nnz < 0 || nnz > (1ll << 40)) return fail(SG_ERR_INVALID, "nnz=%lld outside [0, 2^40]", (long long)nnz);
     if (!row_ptr || (nnz > 0 && !col_idx)) return fail(SG_ERR_INVALID, "row_ptr/col_idx NULL");
     if (mem != SG_MEM_HOST && mem != SG_MEM_DEVICE) return fail(SG_ERR_INVALID, "mem must be SG_MEM_HOST or SG_MEM_DEVICE");
-    if (flags & ~(SG_F_BORROW | SG_F_VALIDATE)) return fail(SG_ERR_INVALID, "unknown flags 0x%x", flags);
+    if (flags & ~(SG_F_BORROW | SG_F_VALIDATE | SG_F_DIRECTED)) return fail(SG_ERR_INVALID, "unknown flags 0x%x", flags);
+    const bool directed = (flags & SG_F_DIRECTED) != 0;
+    if (directed && comm && comm->c.nranks > 1)
+        return fail(SG_ERR_UNSUPPORTED, "a partitioned graph must be symmetric (SG_F_DIRECTED is single-GPU)");
     const bool borrow = (flags & SG_F_BORROW) != 0;
     if (borrow && mem != SG_MEM_DEVICE) return fail(SG_ERR_INVALID, "SG_F_BORROW needs SG_MEM_DEVICE arrays");
     if (mem == SG_MEM_DEVICE) {
@@ -622,15 +628,29 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
         return fail(SG_ERR_INVALID, "CSR validation failed (%llu malformed row_ptr / col_idx entries)", hv[0]);
     }
     launch_row_check(g->v, dscr + 3, s);                           // [3] unsorted pairs, [4] self-loops
-    if (flags & SG_F_VALIDATE) launch_symmetry(g->v, dscr + 5, s); // [5] arcs without reverse
+    if ((flags & SG_F_VALIDATE) && !directed) launch_symmetry(g->v, dscr + 5, s); // [5] arcs without reverse
     CK(dev_alloc(&g->deg8, (size_t)g->v.nw1 * 64, s));
-    launch_deg8(g->rp, n, g->v.nw1 * 64, g->deg8, s);
+    launch_deg8(g->rp, n, g->v.nw1 * 64, g->deg8, s);   // out-degree codes (push cost m_f)
     g->v.deg8 = g->deg8;
+    g->directed = directed;
+    if (directed) {   // pull steps read in-neighbours: the transpose ("CSR and CSC")
+        CK(build_csc(g->rp, g->col, n, nnz, &g->rpt, &g->colt, s));
+    }
+    const int64_t *prp = directed ? g->rpt : g->rp;    // rows a pull step scans
+    const int32_t *pcol = directed ? g->colt : g->col;
     CK(dev_alloc(&g->isolated, sizeof(uint64_t) * (size_t)g->v.nw1, s));
-    launch_isolated(g->deg8, n, g->v.nw1, g->isolated, s);
+    if (directed) {   // unreachable = no in-arc (a directed vertex with out-arcs only is never reached)
+        uint8_t *indeg8 = nullptr;
+        CK(dev_alloc(&indeg8, (size_t)g->v.nw1 * 64, s));
+        launch_deg8(prp, n, g->v.nw1 * 64, indeg8, s);
+        launch_isolated(indeg8, n, g->v.nw1, g->isolated, s);
+        CK(cudaFreeAsync(indeg8, s));
+    } else {
+        launch_isolated(g->deg8, n, g->v.nw1, g->isolated, s);
+    }
     launch_popcount(g->isolated, g->v.nw1, dscr + 6, s);           // [6] isolated vertices
     CK(dev_alloc(&g->fnbr, sizeof(int32_t) * (size_t)(g->v.nw1 ? g->v.nw1 * 64 : 1), s));   // padded: 16-B quad loads
-    launch_first_nbr(g->rp, g->col, g->deg8, n, g->v.nw1 * 64, g->fnbr, s);
+    launch_first_nbr(prp, pcol, g->deg8, n, g->v.nw1 * 64, g->fnbr, s);
     g->v.fnbr = g->fnbr;
     if (g->w) launch_max_weight(g->w, nnz, reinterpret_cast<unsigned int *>(dscr + 1), s);
     // hubs of the destination-segmented BFS tier (deg >= SEG_MIN): index map + vertex list
@@ -672,6 +692,13 @@ SG_API int graph_load_csr(int64_t n, int64_t nnz, const int64_t *row_ptr, const 
         g->v.hub_off = g->hub_off;
     }
     if (!part) g->vl = g->v;
+    if (directed) {   // pull view: the CSC (in-neighbour rows), same frontier layout and degree codes
+        g->vl.rp = g->rpt;
+        g->vl.col = g->colt;
+        g->vl.w = nullptr;
+        g->vl.hub_idx = nullptr;
+        g->vl.hub_off = nullptr;
+    }
     *out = g;
     return SG_OK;
 }
@@ -684,6 +711,8 @@ SG_API int graph_free(sg_graph *g) {
     arena_free(g);
     dev_free(g->rpl);
     dev_free(g->coll);
+    dev_free(g->rpt);
+    dev_free(g->colt);
     if (!g->borrowed) {
         dev_free(g->rp);
         dev_free(g->col);
@@ -1463,7 +1492,7 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         }
         const int pr = prof_begin(ws, pull ? SG_K_PULL : (sweep ? SG_K_SWEEP : SG_K_PUSH), s);
         if (pull) {
-            launch_pull_bfs(G, in->bits, ws->visited, in->st, bo, s);   // writes its output itself
+            launch_pull_bfs(g->vl, in->bits, ws->visited, in->st, bo, s);   // writes its output itself
             pull_steps++;
         } else if (sweep) {
             launch_push_sweep(g->scsr.v, G.rp, in->bits, in->summ, in->offsets, G.nw2, in->st, ws->visited, 0ull, s);
@@ -1987,6 +2016,7 @@ SG_API int run_cc(const sg_graph *gc, int32_t *label, const sg_opts *opts, sg_st
     const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
     cudaStream_t s = stream_of(&o);
     TRY(ensure_ws(g));
+    if (g->directed) return fail(SG_ERR_UNSUPPORTED, "CC by label propagation needs a symmetric graph (reading C8)");
     if (g->ar) return run_value_part(g, true, 0, reinterpret_cast<uint32_t *>(label), o, stats);
     // default: device-driven loop (CUDA graph); host_loop = 1 keeps the host-driven one below
     if (!o.host_loop) return run_value_graph(g, true, 0, reinterpret_cast<uint32_t *>(label), o, max_iters, stats);
@@ -2146,6 +2176,7 @@ SG_API int run_bc(const sg_graph *gc, const int32_t *sources, int32_t k, double 
     t_err.clear();
     if (!gc || !bc || (k > 0 && !sources) || k < 0) return fail(SG_ERR_INVALID, "bad run_bc arguments");
     if (gc->ar) return fail(SG_ERR_UNSUPPORTED, "BC shards sources over full replicas (SURVEY 8(e)), not a partitioned graph");
+    if (gc->directed) return fail(SG_ERR_UNSUPPORTED, "BC (pull-style backward sweep) needs a symmetric graph");
     sg_graph *g = const_cast<sg_graph *>(gc);
     const GraphView &G = g->v;
     for (int32_t i = 0; i < k; i++)

@@ -209,6 +209,9 @@ cudaError_t part_quantiles(const int64_t *rp, int64_t n, int64_t nnz, int P, int
 // push block: the arcs of every row into [lo, hi) (CSR over all n rows; +64 B padding)
 cudaError_t part_push_block(const int64_t *rp, const int32_t *col, const uint8_t *w, int64_t n, int64_t lo, int64_t hi,
                             int64_t **rpp, int32_t **colp, uint8_t **wp, int64_t *nnz, cudaStream_t s);
+// transpose of a directed CSR (in-neighbours, rows sorted), for pull steps
+cudaError_t build_csc(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int64_t **rpt, int32_t **colt,
+                      cudaStream_t s);
 // pull block: rows [lo, hi) (CSR over all n rows, rows outside empty)
 cudaError_t part_pull_block(const int64_t *rp, const int32_t *col, int64_t n, int64_t lo, int64_t hi, int64_t **rpl,
                             int32_t **coll, int64_t *nnz, cudaStream_t s);

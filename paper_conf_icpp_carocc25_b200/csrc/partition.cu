@@ -10,6 +10,7 @@
 //   pull block: the owned rows themselves (symmetric graph: in-neighbours), as a CSR over all n
 //               rows whose rows outside [lo, hi) are empty.
 #include <cub/device/device_scan.cuh>
+#include <cub/device/device_segmented_sort.cuh>
 
 #include "common.cuh"
 #include "kernels.h"
@@ -177,6 +178,78 @@ cudaError_t part_pull_block(const int64_t *rp, const int32_t *col, int64_t n, in
     *rpl_out = rpl;
     *coll_out = coll;
     *nnz_out = m;
+    return cudaSuccess;
+}
+
+
+// ---- transpose (CSC) of a directed CSR for pull steps (§3.1 "CSR and CSC") --
+// in-degree histogram -> exclusive scan -> scatter with per-row cursors -> per-row sort (the pull
+// candidate heuristic scans a row's first arcs; sorted rows keep it deterministic)
+__global__ void k_indeg(const int32_t *__restrict__ col, int64_t nnz, unsigned long long *__restrict__ indeg) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz; e += stride)
+        atomicAdd(indeg + col[e], 1ull);
+}
+__global__ void k_csc_fill(const int64_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t n,
+                           const int64_t *__restrict__ rpt, unsigned long long *__restrict__ cursor,
+                           int32_t *__restrict__ colt) {
+    const int lane = lane_id();
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = gw; u < n; u += nwarps)
+        for (int64_t e = rp[u] + lane; e < rp[u + 1]; e += 32) {
+            const int32_t v = col[e];
+            colt[rpt[v] + (int64_t)atomicAdd(cursor + v, 1ull)] = (int32_t)u;
+        }
+}
+
+cudaError_t build_csc(const int64_t *rp, const int32_t *col, int64_t n, int64_t nnz, int64_t **rpt_out,
+                      int32_t **colt_out, cudaStream_t s) {
+    unsigned long long *cnt = nullptr;
+    int64_t *rpt = nullptr;
+    int32_t *colt = nullptr, *sorted = nullptr;
+    void *tmp = nullptr;
+    size_t tb = 0, tb2 = 0;
+    cudaError_t e = dev_alloc(&cnt, sizeof(unsigned long long) * (size_t)(n + 1), s);
+    if (e == cudaSuccess) e = dev_alloc(&rpt, sizeof(int64_t) * (size_t)(n + 1), s);
+    if (e == cudaSuccess) e = dev_alloc(&colt, sizeof(int32_t) * (size_t)nnz + 64, s);
+    if (e == cudaSuccess) e = dev_alloc(&sorted, sizeof(int32_t) * (size_t)nnz + 64, s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * (size_t)(n + 1), s);
+    if (e == cudaSuccess && nnz) {
+        note_launch();
+        k_indeg<<<grid_of(nnz, 256), 256, 0, s>>>(col, nnz, cnt);
+    }
+    if (e == cudaSuccess)
+        e = cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, reinterpret_cast<unsigned long long *>(rpt), n + 1, s);
+    if (e == cudaSuccess)
+        e = cub::DeviceSegmentedSort::SortKeys(nullptr, tb2, colt, sorted, nnz, n, rpt, rpt + 1, s);
+    if (e == cudaSuccess) e = dev_alloc(&tmp, tb > tb2 ? tb : tb2, s);
+    if (e == cudaSuccess) {
+        note_launch();
+        e = cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, reinterpret_cast<unsigned long long *>(rpt), n + 1, s);
+    }
+    if (e == cudaSuccess) e = cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * (size_t)(n + 1), s);
+    if (e == cudaSuccess && nnz) {
+        note_launch();
+        k_csc_fill<<<grid_of(n * 32, 256), 256, 0, s>>>(rp, col, n, rpt, cnt, colt);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess && nnz) {
+        note_launch();
+        e = cub::DeviceSegmentedSort::SortKeys(tmp, tb2, colt, sorted, nnz, n, rpt, rpt + 1, s);
+    }
+    if (e == cudaSuccess) e = cudaMemsetAsync((char *)sorted + sizeof(int32_t) * (size_t)nnz, 0, 64, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (cnt) cudaFreeAsync(cnt, s);
+    if (tmp) cudaFreeAsync(tmp, s);
+    if (colt) cudaFreeAsync(colt, s);
+    if (e != cudaSuccess) {
+        if (rpt) cudaFreeAsync(rpt, s);
+        if (sorted) cudaFreeAsync(sorted, s);
+        return e;
+    }
+    *rpt_out = rpt;
+    *colt_out = sorted;
     return cudaSuccess;
 }
 

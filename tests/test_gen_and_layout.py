@@ -76,3 +76,23 @@ def test_two_layer_bitmap_fixture():
     assert np.array_equal(w, words)
     assert np.array_equal(oracle.summary_words(w), summ)
     assert np.array_equal(oracle.words_to_mask(w, n), mask)
+
+
+def test_orient_makes_a_directed_subgraph():
+    """gen.orient keeps each arc of a symmetric graph by a hash bit: every kept arc is an arc of
+    the input, rows stay sorted, and both / one / no direction survive about 1/4, 1/2, 1/4."""
+    g = gen.with_weights(gen.rmat(12, 16, permute=True), seed=3)
+    d = gen.orient(g, seed=5)
+    rows = np.repeat(np.arange(g.n), g.degrees())
+    full = set(zip(rows.tolist(), g.col_idx.tolist()))
+    drows = np.repeat(np.arange(d.n), d.degrees())
+    arcs = set(zip(drows.tolist(), d.col_idx.tolist()))
+    assert arcs <= full
+    both = sum(1 for (u, v) in arcs if u < v and (v, u) in arcs)
+    edges = len(full) // 2
+    assert abs(both / edges - 0.25) < 0.03 and abs(len(arcs) / len(full) - 0.5) < 0.03
+    starts = np.zeros(d.nnz + 1, bool)
+    starts[d.row_ptr[:-1]] = True
+    assert ((np.diff(d.col_idx.astype(np.int64)) > 0) | starts[1:-1]).all()
+    w = dict(zip(zip(rows.tolist(), g.col_idx.tolist()), g.weights.tolist()))
+    assert all(w[(u, v)] == x for (u, v), x in zip(zip(drows.tolist(), d.col_idx.tolist()), d.weights.tolist()))

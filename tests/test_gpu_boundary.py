@@ -205,3 +205,28 @@ def test_borrowed_device_csr(sg):
     assert e.value.code == sg.SG_ERR_INVALID
     with pytest.raises(sg.SgError):
         sg.graph_load_csr(g.row_ptr, g.col_idx, borrow=True)   # host arrays cannot be borrowed
+
+
+@pytest.mark.parametrize("make", [lambda: gen.rmat(14, 16, permute=True), lambda: gen.lattice(100, 130, 0.7, seed=2),
+                                  lambda: gen.rmat(12, 4, permute=True)])
+def test_directed_graphs_pull_through_the_transpose(sg, make):
+    """SG_F_DIRECTED ("CSR and CSC", P:299 directed datasets): push follows out-arcs,
+    pull steps scan in-neighbours from the library-built CSC; BFS in every direction / loop mode and
+    SSSP equal the oracle's directed BFS / Dijkstra; CC and BC refuse a directed graph."""
+    g = gen.with_weights(gen.orient(make(), seed=9), seed=4)
+    G = sg.graph_load_csr(g.row_ptr, g.col_idx, g.weights, validate=True, directed=True)
+    with pytest.raises(sg.SgError):          # the same arcs are not a valid symmetric graph
+        sg.graph_load_csr(g.row_ptr, g.col_idx, validate=True)
+    deg = g.degrees()
+    for s in list(gen.sources(g, 3)) + [int(np.argmax(deg))]:
+        ref = oracle.bfs(g, int(s))
+        for d in (sg.SG_DIR_AUTO, sg.SG_DIR_PUSH, sg.SG_DIR_PULL):
+            for hl in (False, True):
+                lv, _ = sg.run_bfs(G, int(s), direction=d, host_loop=hl)
+                assert np.array_equal(sg.as_u32(lv), ref), (s, d, hl)
+        dist, _ = sg.run_sssp(G, int(s))
+        assert np.array_equal(sg.as_u32(dist), oracle.sssp(g, int(s)))
+    for fn in (lambda: sg.run_cc(G), lambda: sg.run_bc(G, [0])):
+        with pytest.raises(sg.SgError) as e:
+            fn()
+        assert e.value.code == sg.SG_ERR_UNSUPPORTED
