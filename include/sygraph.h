@@ -243,6 +243,12 @@ SG_API int64_t sg_launch_count(void);
  * prologue's), globaltimer ns since decision 0, the decision (0 stop, 1 push, 2 pull, 3 sweep,
  * 4 fused sparse superstep) and the frontier it was taken on (words, n_f, m_f).  Returns the
  * number of entries (<= cap); pointers may be NULL. */
+/* Word-width ablation (§4.3 "32-bit integer to match a warp on NVIDIA"): a
+ * self-contained push-only Two-Layer-Bitmap BFS with word_bits = 32 (one bit per lane) or 64 (two
+ * per lane) words in both layers, the paper's warp-per-word / lanes-stride-the-list mapping,
+ * host-driven loop.  Same levels as run_bfs (level: device[n]); device_ms = its time. */
+SG_API int sg_ablation_bfs(const sg_graph *g, int32_t src, uint32_t *level, int32_t word_bits, void *stream,
+                           sg_stats *stats);
 /* Debug accumulators of the last device-driven run_bfs (fused sparse loop phase times, ns). */
 SG_API int sg_ctrl_debug(const sg_graph *g, int64_t out[16]);
 SG_API int sg_bfs_trace(const sg_graph *g, int64_t *t_ns, int32_t *kind, int64_t *count, int64_t *nf, int64_t *mf,

@@ -76,7 +76,7 @@ EXPORTS = ["graph_load_csr", "graph_free", "graph_info", "frontier_init", "front
            "frontier_fill_all", "frontier_clear", "frontier_count", "frontier_view", "frontier_op",
            "frontier_or_into", "advance", "run_bfs", "run_sssp", "run_cc", "run_bc", "sg_opts_default",
            "sg_last_error", "sg_version", "sg_profile", "sg_profile_read", "sg_launch_count", "frontier_filter",
-           "compute_execute", "comm_unique_id", "comm_init", "comm_free", "comm_info", "graph_partition", "sg_bfs_trace", "sg_ctrl_debug"]
+           "compute_execute", "comm_unique_id", "comm_init", "comm_free", "comm_info", "graph_partition", "sg_bfs_trace", "sg_ctrl_debug", "sg_ablation_bfs"]
 SG_PRED_DEGREE_RANGE, SG_PRED_U32_RANGE, SG_PRED_I32_RANGE, SG_PRED_F64_RANGE, SG_PRED_IN_BITMAP = 0, 1, 2, 3, 4
 SG_OP_SET_U32, SG_OP_SET_I32, SG_OP_SET_F64, SG_OP_ADD_U32, SG_OP_ADD_F64 = 0, 1, 2, 3, 4
 
@@ -98,6 +98,7 @@ def load():
         "graph_partition": (c_int, [vp, ctypes.POINTER(i64), ctypes.POINTER(i64)]),
         "sg_bfs_trace": (c_int, [vp, vp, vp, vp, vp, vp, i32]),
         "sg_ctrl_debug": (c_int, [vp, vp]),
+        "sg_ablation_bfs": (c_int, [vp, i32, vp, i32, vp, ctypes.POINTER(SgStats)]),
         "comm_unique_id": (c_int, [ctypes.c_char_p]),
         "comm_init": (c_int, [ctypes.c_char_p, c_int, c_int, c_int, pp]),
         "comm_free": (c_int, [vp]),
@@ -471,6 +472,16 @@ def bfs_trace(g: Graph) -> list:
         out.append({"step": i, "kind": TRACE_KINDS.get(k[i], k[i]), "words": c[i], "nf": nf[i], "mf": mf[i],
                     "us": (t[i + 1] - t[i]) / 1e3})
     return out
+
+
+def ablation_bfs(g: Graph, src: int, word_bits: int, level=None, stream=None):
+    """Word-width ablation BFS (sg_ablation_bfs): push-only 2LB with 32- or 64-bit words."""
+    import torch
+    level = _out_tensor(g.n, torch.int32, level)
+    st = SgStats()
+    _check(load().sg_ablation_bfs(g.handle, int(src), level.data_ptr(), int(word_bits), _stream_ptr(stream),
+                                  ctypes.byref(st)))
+    return level, st
 
 
 def ctrl_debug(g: Graph) -> list:

@@ -148,15 +148,16 @@ __device__ __forceinline__ void val_decide(ValCtrl *c, const DevStats *st, unsig
 // per block (ascending within the block).  Partitioned: the same layer-2 words and list entries
 // go to every peer's replica (one remote atomic per block and peer).  Call with the whole block;
 // ends with __syncthreads.
+template <bool P = true>
 __device__ __forceinline__ void bfs_emit_words(const BfsOut &o, int64_t w2_hi, int64_t sw0, const uint64_t *S, int nS,
                                                uint32_t *s_base) {
     const Xchg &x = o.x;
-    if ((int)threadIdx.x < nS && sw0 + threadIdx.x < w2_hi) xstore(x, o.out_summ + sw0 + threadIdx.x, S[threadIdx.x]);
+    if ((int)threadIdx.x < nS && sw0 + threadIdx.x < w2_hi) xstore<P>(x, o.out_summ + sw0 + threadIdx.x, S[threadIdx.x]);
     if (threadIdx.x == 0) {
         uint32_t tot = 0;
         for (int i = 0; i < nS; i++) tot += (uint32_t)__popcll(S[i]);
         s_base[0] = tot ? (uint32_t)atomicAdd(&o.st->count, (unsigned long long)tot) : 0u;
-        if (x.nranks > 1 && tot) {
+        if (P && x.nranks > 1 && tot) {
             unsigned long long b[SG_MAX_RANKS];
 #pragma unroll
             for (int j = 0; j < SG_MAX_RANKS; j++)   // all remote atomics in flight together
@@ -175,7 +176,7 @@ __device__ __forceinline__ void bfs_emit_words(const BfsOut &o, int64_t w2_hi, i
             for (int j = 0; j < i; j++) pos += (uint32_t)__popcll(S[j]);
             const uint32_t val = (uint32_t)((sw0 + i) * 64 + b);
             o.out_offsets[s_base[0] + pos] = val;
-            if (x.nranks > 1) {
+            if (P && x.nranks > 1) {
                 for (int j = 0; j < x.nranks; j++)
                     if (j != x.rank) xpeer(x, o.out_offsets, j)[s_base[1 + j] + pos] = val;
             }
@@ -189,28 +190,33 @@ __device__ __forceinline__ void bfs_emit_words(const BfsOut &o, int64_t w2_hi, i
 // CTA first runs the superstep barrier (xchg.cuh) and replaces st's n_f / m_f by the global sums;
 // it zeroes the input's control block BEFORE publishing (peers add their word-list counts into it
 // as soon as they pass this barrier: it is the next superstep's output).  Whole block.
+template <bool P = true>
 __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long nf, unsigned long long mf,
-                                           unsigned long long arcs, DevStats *in_st) {
-    __shared__ unsigned long long s_r[3][32];
+                                           unsigned long long arcs, DevStats *in_st, unsigned long long scans = 0) {
+    __shared__ unsigned long long s_r[4][32];
     __shared__ bool s_last;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const bool part = o.x.nranks > 1;
+    const bool part = P && o.x.nranks > 1;
     nf = warp_sum(nf);
     mf = warp_sum(mf);
     arcs = warp_sum(arcs);
+    scans = warp_sum(scans);
     if (lane == 0) {
         s_r[0][wid] = nf;
         s_r[1][wid] = mf;
         s_r[2][wid] = arcs;
+        s_r[3][wid] = scans;
     }
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned long long a = 0, b = 0, c = 0;
+        unsigned long long a = 0, b = 0, c = 0, d = 0;
         for (int i = 0; i < (int)(blockDim.x >> 5); i++) {
             a += s_r[0][i];
             b += s_r[1][i];
             c += s_r[2][i];
+            d += s_r[3][i];
         }
+        if (d && in_st) atomicAdd(&in_st->scans, d);
         if (a) {
             atomicAdd(&o.st->nf, a);
             atomicAdd(&o.st->mf, b);
@@ -225,7 +231,8 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
     }
     __syncthreads();
     if (s_last && threadIdx.x == 0) {
-        __threadfence_system();
+        if (part) __threadfence_system();
+        else __threadfence();
         *o.done = 0u;
         DevStats *prev = o.prev ? o.prev : in_st;
         unsigned long long prev_arcs = prev ? reinterpret_cast<const volatile DevStats *>(prev)->arcs : 0ull;

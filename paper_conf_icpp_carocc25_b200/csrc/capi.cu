@@ -5,6 +5,7 @@
 // is empty.  Per superstep the host reads back one 128-byte control block (frontier sizes for
 // empty() and the direction policy); everything else stays on the device stream.
 #include <atomic>
+#include <cstddef>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -137,7 +138,7 @@ struct Workspace {
     cudaGraph_t bfs_graph = nullptr;
     cudaGraphExec_t bfs_exec = nullptr;
     uint32_t *bfs_level = nullptr;
-    int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1, bfs_cf = -1, bfs_scsr = -1;
+    int32_t bfs_heavy = 0, bfs_small = 0, bfs_seg = -1, bfs_cf = -1, bfs_scsr = -1, bfs_shape = -1;
     SegItem *seg = nullptr;        // destination-segmented hub queue (BFS)
     uint32_t seg_cap = 0;
     // source-batched BC (bcb.cu)
@@ -1246,14 +1247,17 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     cudaGraph_t root;
     CK(cudaGraphCreate(&root, 0));
     ws->bfs_graph = root;
-    cudaGraphConditionalHandle h_loop, h_push[2], h_pull[2], h_sweep[2], h_sparse[2];
+    cudaGraphConditionalHandle h_loop, h_push[2], h_pull[2], h_sweep[2], h_sparse[2] = {};
+    // the fused small-frontier loop's IF nodes exist only when it is enabled (SG_SPARSE=1): an
+    // untaken IF still costs ~0.4 us per superstep
+    const bool sp = env_or("SG_SPARSE", 0) != 0;
     const bool sc = t.scsr != 0 && g->scsr_state == 1;
     CK(cudaGraphConditionalHandleCreate(&h_loop, root, 0, cudaGraphCondAssignDefault));
     for (int i = 0; i < 2; i++) {
         CK(cudaGraphConditionalHandleCreate(&h_push[i], root, 0, cudaGraphCondAssignDefault));
         CK(cudaGraphConditionalHandleCreate(&h_pull[i], root, 0, cudaGraphCondAssignDefault));
         if (sc) CK(cudaGraphConditionalHandleCreate(&h_sweep[i], root, 0, cudaGraphCondAssignDefault));
-        CK(cudaGraphConditionalHandleCreate(&h_sparse[i], root, 0, cudaGraphCondAssignDefault));
+        if (sp) CK(cudaGraphConditionalHandleCreate(&h_sparse[i], root, 0, cudaGraphCondAssignDefault));
     }
     sg_frontier *F[2] = {&ws->fr[0], &ws->fr[1]};
     std::vector<cudaGraphNode_t> leaves;
@@ -1273,7 +1277,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         ws->hnd[1 + i] = (unsigned long long)h_push[i];
         ws->hnd[3 + i] = (unsigned long long)h_pull[i];
         ws->hnd[5 + i] = sc ? (unsigned long long)h_sweep[i] : 0ull;
-        ws->hnd[7 + i] = (unsigned long long)h_sparse[i];
+        ws->hnd[7 + i] = sp ? (unsigned long long)h_sparse[i] : 0ull;
     }
     TRY(capture_end(cs, leaves));
     cudaGraphNode_t wnode;
@@ -1290,7 +1294,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         cudaGraphNode_t n_sweep = nullptr, n_sparse = nullptr;
         cudaGraph_t b_sweep = nullptr, b_sparse = nullptr;
         if (sc) TRY(add_cond(body, deps, h_sweep[half], cudaGraphCondTypeIf, &n_sweep, &b_sweep));
-        TRY(add_cond(body, deps, h_sparse[half], cudaGraphCondTypeIf, &n_sparse, &b_sparse));
+        if (sp) TRY(add_cond(body, deps, h_sparse[half], cudaGraphCondTypeIf, &n_sparse, &b_sparse));
         PushLaunch L = push_launch(g, in, t, -1);
         L.batch = t.cf;   // 0: coarsening factor computed on the device from the count
         L.sparse_ok = 1;  // n_f of every BFS frontier is exact (prologue statistics / output kernels)
@@ -1314,7 +1318,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         TRY(capture_begin(cs, b_pull, {}));
         launch_pull_bfs(g->vl, in->bits, ws->visited, in->st, bo, cs);   // writes its output itself
         TRY(capture_end(cs, leaves));
-        {   // small frontiers: the whole superstep in one kernel (sparse.cu)
+        if (sp) {   // small frontiers: the whole superstep in one kernel (sparse.cu)
             BfsOut bs = bo;
             bs.sparse = 1;
             PushLaunch Ls = push_launch(g, in, t, -1);
@@ -1322,7 +1326,8 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
             launch_bfs_sparse(Ls, a, bs, in->bits, in->summ, ws->gbar, cs);
             TRY(capture_end(cs, leaves));
         }
-        deps = {n_push, n_pull, n_sparse};
+        deps = {n_push, n_pull};
+        if (n_sparse) deps.push_back(n_sparse);
         if (n_sweep) deps.push_back(n_sweep);
     }
     CK(cudaGraphInstantiate(&ws->bfs_exec, root, 0));
@@ -1348,9 +1353,12 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     Workspace *ws = g->ws;
     cudaStream_t s = stream_of(&o);
     const int32_t sc_mode = t.scsr != 0 && g->scsr_state == 1 ? t.scsr : 0;
+    const int shape = (env_or("SG_SPARSE", 0) != 0 ? 1 : 0) | (env_or("SG_PULL_WARP_FRAC", 8) != 0 ? 2 : 0);
     if (!ws->bfs_exec || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small || ws->bfs_seg != t.seg ||
-        ws->bfs_cf != t.cf || ws->bfs_scsr != sc_mode)
+        ws->bfs_cf != t.cf || ws->bfs_scsr != sc_mode || ws->bfs_shape != shape) {
         TRY(build_bfs_graph(g, t));
+        ws->bfs_shape = shape;
+    }
     BfsCtrl &c = *ws->h_ctrl;
     memset(&c, 0, sizeof c);
     c.level = level;
@@ -1382,7 +1390,9 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         c.hsparse[i] = ws->hnd[7 + i];
     }
     CK(cudaEventRecord(ws->ev0, s));
-    CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, sizeof(BfsCtrl), cudaMemcpyHostToDevice, s));
+    // the control block up to the trace arrays (those are read on demand by sg_bfs_trace)
+    const size_t hot = offsetof(BfsCtrl, t_ns);
+    CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, hot, cudaMemcpyHostToDevice, s));
     CK(cudaGraphLaunch(ws->bfs_exec, s));
     if (g->ar && !o.owned_only) {   // result gather: owned level slices into every rank's replica
         const Arena *A = g->ar;
@@ -1390,7 +1400,7 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         launch_xbarrier(A->x, s);
         CK(cudaMemcpyAsync(level, A->vals, sizeof(uint32_t) * (size_t)g->v.n, cudaMemcpyDeviceToDevice, s));
     }
-    CK(cudaMemcpyAsync(ws->h_ctrl, ws->ctrl, sizeof(BfsCtrl), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(ws->h_ctrl, ws->ctrl, hot, cudaMemcpyDeviceToHost, s));
     CK(cudaEventRecord(ws->ev1, s));
     CK(cudaEventSynchronize(ws->ev1));
     float ms = 0.f;
@@ -1404,7 +1414,8 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         // count + sweep + output, pull = 1)
         const long long per_push = 3 + (t.seg && ws->seg && g->v.hub_idx ? 1 : 0);
         const long long k = 1 + per_push * (long long)(c.push_steps - c.sweep_steps - c.sparse_steps) +
-                            3 * (long long)c.sweep_steps + (long long)c.sparse_steps + 2 * (long long)c.pull_steps;
+                            3 * (long long)c.sweep_steps + (long long)c.sparse_steps +
+                            (ws->bfs_shape & 2 ? 2 : 1) * (long long)c.pull_steps;
         for (long long i = 0; i < k; i++) note_launch();
     }
     if (stats) {
@@ -1526,13 +1537,13 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
             // per output word, layer 2 8 B per word.  pull (with its output): visited 8 B per
             // word read, fnbr / col_idx 4 B per candidate / arc tested, output word 8 B per word,
             // level + degree code 5 B per new vertex, visited + vis_old 16 B + list entry 4 B
-            // per output word, layer 2 8 B per word
+            // per output word, layer 2 8 B per word, row_ptr 16 B per list-scanned vertex
             const DevStats &ho = ws->h_st[in_idx ^ 1];
             const double n_new = (double)ho.nf, c_out = (double)ho.count;
             double bytes;
-            if (pull)
-                bytes = 16.0 * (double)G.nw1 + 4.0 * (double)ws->h_st[in_idx].arcs + 5.0 * n_new + 20.0 * c_out +
-                        8.0 * (double)G.nw2;
+            if (pull)   // + 16 B of row_ptr per list-scanned vertex (candidate missed)
+                bytes = 16.0 * (double)G.nw1 + 4.0 * (double)ws->h_st[in_idx].arcs +
+                        16.0 * (double)ws->h_st[in_idx].scans + 5.0 * n_new + 20.0 * c_out + 8.0 * (double)G.nw2;
             else
                 bytes = 4.0 * (double)ws->h_st[in_idx].arcs + 16.0 * (double)nf + 8.0 * (double)count + 8.0 * c_out;
             prof_bytes(ws, pr, bytes);
@@ -2301,8 +2312,28 @@ SG_API int sg_profile_read(const sg_graph *g, sg_kprof *out) {
 
 SG_API int64_t sg_launch_count(void) { return (int64_t)g_launches.load(); }
 
+SG_API int sg_ablation_bfs(const sg_graph *g, int32_t src, uint32_t *level, int32_t word_bits, void *stream,
+                           sg_stats *stats) {
+    t_err.clear();
+    if (!g || !level || (word_bits != 32 && word_bits != 64)) return fail(SG_ERR_INVALID, "bad sg_ablation_bfs arguments");
+    if (src < 0 || src >= g->v.n) return fail(SG_ERR_INVALID, "src outside [0, n)");
+    if (g->ar) return fail(SG_ERR_UNSUPPORTED, "ablation paths are single-GPU");
+    int64_t it = 0;
+    float ms = 0.f;
+    if (ablation_bfs_words(g->v, src, level, word_bits, (cudaStream_t)stream, &it, &ms) != 0)
+        return fail(SG_ERR_CUDA, "ablation BFS failed: %s", cudaGetErrorString(cudaGetLastError()));
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->iterations = it;
+        stats->push_steps = it;
+        stats->device_ms = ms;
+    }
+    return SG_OK;
+}
+
 SG_API int sg_ctrl_debug(const sg_graph *g, int64_t out[16]) {
     if (!g || !g->ws || !g->ws->h_ctrl || !out) return fail(SG_ERR_STATE, "no device-driven BFS has run on this graph");
+    CK(cudaMemcpy(g->ws->h_ctrl, g->ws->ctrl, sizeof(BfsCtrl), cudaMemcpyDeviceToHost));
     for (int i = 0; i < 16; i++) out[i] = (int64_t)g->ws->h_ctrl->dbg[i];
     return SG_OK;
 }
@@ -2310,6 +2341,7 @@ SG_API int sg_ctrl_debug(const sg_graph *g, int64_t out[16]) {
 SG_API int sg_bfs_trace(const sg_graph *g, int64_t *t_ns, int32_t *kind, int64_t *count, int64_t *nf, int64_t *mf,
                         int32_t cap) {
     if (!g || !g->ws || !g->ws->h_ctrl) return fail(SG_ERR_STATE, "no device-driven BFS has run on this graph");
+    CK(cudaMemcpy(g->ws->h_ctrl, g->ws->ctrl, sizeof(BfsCtrl), cudaMemcpyDeviceToHost));
     const BfsCtrl &c = *g->ws->h_ctrl;
     const int n = (int)(c.tr_n < (unsigned long long)SG_TRACE_STEPS ? c.tr_n : SG_TRACE_STEPS);
     for (int i = 0; i < n && i < cap; i++) {

@@ -4,6 +4,7 @@
 //   layer 2  uint64 summ[nw2], nw2 = ceil(nw1/64): bit (w & 63) of word (w >> 6) <=> bits[w] != 0
 #pragma once
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 namespace sg {
@@ -75,7 +76,9 @@ struct DevStats {
     unsigned long long batch;        // push: next word batch (dynamic CTA scheduling)
     unsigned long long heavy_count;  // push: CTA/grid-tier chunks queued
     unsigned long long seg_count;    // push: destination-segmented hub chunks queued (BFS)
-    unsigned long long pad;
+    unsigned long long pad;          // partitioned host loops: the superstep's global arcs
+    unsigned long long scans;        // pull: vertices whose candidate missed (a row_ptr pair + list scan)
+    unsigned long long pad2;
 };
 
 constexpr int SG_TRACE_STEPS = 48;
@@ -292,6 +295,8 @@ inline cudaMemPool_t graph_pool() {
     return pools[dev];
 }
 inline cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s) {
+    static const bool dflt = getenv("SG_DEFAULT_POOL") != nullptr;   // A/B knob: the device's default pool
+    if (dflt) return cudaMallocAsync(p, bytes, s);
     cudaMemPool_t pool = graph_pool();
     if (!pool) return cudaMallocAsync(p, bytes, s);
     return cudaMallocFromPoolAsync(p, bytes, pool, s);

@@ -416,6 +416,7 @@ void launch_seed(uint64_t *bits, uint64_t *summ, uint64_t *visited, int32_t src,
 #endif
 constexpr int DIFF_WORDS_PER_ROUND = SG_DIFF_WPR;
 constexpr int DIFF_THREADS = 256;
+template <bool P>
 __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const uint64_t *__restrict__ visited, BfsOut o) {
     __shared__ uint64_t s_S[DIFF_THREADS / 64];
     __shared__ uint32_t s_ch[DIFF_THREADS / 32];
@@ -441,13 +442,13 @@ __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const ui
         const uint64_t da = na & ~oa;
         uint32_t ch = __ballot_sync(0xffffffffu, da != 0);
         if (lane == 0) s_ch[wid] = ch;
-        if (wa < g.w1_hi) xstore(o.x, o.out_bits + wa, da);
+        if (wa < g.w1_hi) xstore<P>(o.x, o.out_bits + wa, da);
         if (da) o.vis_old[wa] = na;
         __syncthreads();
         if (threadIdx.x < DIFF_THREADS / 64)
             s_S[threadIdx.x] = (uint64_t)s_ch[2 * threadIdx.x] | ((uint64_t)s_ch[2 * threadIdx.x + 1] << 32);
         __syncthreads();
-        bfs_emit_words(o, g.w2_hi, base >> 6, s_S, DIFF_THREADS / 64, s_base);
+        bfs_emit_words<P>(o, g.w2_hi, base >> 6, s_S, DIFF_THREADS / 64, s_base);
         if (ch && !lvl) {
             lvl = o.level_pp ? *o.level_pp : o.level;
             nx = o.next_ptr ? *o.next_ptr : o.next;
@@ -491,14 +492,15 @@ __global__ void __launch_bounds__(DIFF_THREADS) k_bfs_diff(GraphView g, const ui
             }
         }
     }
-    bfs_finish(o, nf, mf, 0ull, nullptr);
+    bfs_finish<P>(o, nf, mf, 0ull, nullptr);
 }
 void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &o, cudaStream_t s) {
     int64_t blocks = (g.w1_hi - g.w1_lo + DIFF_THREADS - 1) / DIFF_THREADS;   // 256 layer-1 words per CTA
     if (blocks > SG_DIFF_BLOCKS) blocks = SG_DIFF_BLOCKS;
     if (blocks < 1) blocks = 1;
     note_launch();
-    k_bfs_diff<<<(int)blocks, DIFF_THREADS, 0, s>>>(g, visited, o);
+    if (o.x.nranks > 1) k_bfs_diff<true><<<(int)blocks, DIFF_THREADS, 0, s>>>(g, visited, o);
+    else k_bfs_diff<false><<<(int)blocks, DIFF_THREADS, 0, s>>>(g, visited, o);
 }
 // Output of a diff-mode SSSP / CC superstep (FnSssp::diff; CC pulls and pushes in place): the
 // vertices whose value decreased (value < old, unsigned; CC labels are >= 0).  A CTA of 256
@@ -509,6 +511,7 @@ void launch_bfs_diff(const GraphView &g, const uint64_t *visited, const BfsOut &
 // only; the changed quads' new values and the output words are stored into every peer's replica
 // (a value that did not change needs no exchange: peers already hold it), and the last CTA runs
 // the superstep barrier.
+template <bool P>
 __global__ void __launch_bounds__(256) k_value_diff(GraphView g, uint32_t *__restrict__ dist,
                                                     uint32_t *__restrict__ dist_old, BfsOut o, int want_mf) {
     __shared__ uint64_t s_S[1];
@@ -535,7 +538,7 @@ __global__ void __launch_bounds__(256) k_value_diff(GraphView g, uint32_t *__res
                     m = (a.x < b.x ? 1u : 0u) | (a.y < b.y ? 2u : 0u) | (a.z < b.z ? 4u : 0u) | (a.w < b.w ? 8u : 0u);
                     if (m) {
                         *reinterpret_cast<uint4 *>(dist_old + v0) = a;
-                        if (o.x.nranks > 1)
+                        if (P && o.x.nranks > 1)
                             for (int j = 0; j < o.x.nranks; j++)
                                 if (j != o.x.rank) *reinterpret_cast<uint4 *>(xpeer(o.x, dist + v0, j)) = a;
                     }
@@ -546,7 +549,7 @@ __global__ void __launch_bounds__(256) k_value_diff(GraphView g, uint32_t *__res
                         if (a < dist_old[v0 + k]) {
                             m |= 1u << k;
                             dist_old[v0 + k] = a;
-                            if (o.x.nranks > 1)
+                            if (P && o.x.nranks > 1)
                                 for (int j = 0; j < o.x.nranks; j++)
                                     if (j != o.x.rank) *xpeer(o.x, dist + v0 + k, j) = a;
                         }
@@ -561,14 +564,14 @@ __global__ void __launch_bounds__(256) k_value_diff(GraphView g, uint32_t *__res
             const uint64_t nb = (uint64_t)__reduce_or_sync(half, (uint32_t)mine) |
                                 ((uint64_t)__reduce_or_sync(half, (uint32_t)(mine >> 32)) << 32);
             if ((lane & 15) == 0 && w < g.w1_hi) {
-                xstore(o.x, o.out_bits + w, nb);
+                xstore<P>(o.x, o.out_bits + w, nb);
                 if (nb) atomicOr(reinterpret_cast<unsigned long long *>(s_S), 1ull << (w & 63));
             }
         }
         __syncthreads();
-        bfs_emit_words(o, g.w2_hi, sw, s_S, 1, s_base);
+        bfs_emit_words<P>(o, g.w2_hi, sw, s_S, 1, s_base);
     }
-    bfs_finish(o, nf, mf, 0ull, nullptr);
+    bfs_finish<P>(o, nf, mf, 0ull, nullptr);
 }
 void launch_value_diff(const GraphView &g, uint32_t *value, uint32_t *old, const BfsOut &o, int want_mf,
                        cudaStream_t s) {
@@ -576,7 +579,8 @@ void launch_value_diff(const GraphView &g, uint32_t *value, uint32_t *old, const
     if (blocks > num_sms() * 16) blocks = num_sms() * 16;
     if (blocks < 1) blocks = 1;
     note_launch();
-    k_value_diff<<<(int)blocks, 256, 0, s>>>(g, value, old, o, want_mf);
+    if (o.x.nranks > 1) k_value_diff<true><<<(int)blocks, 256, 0, s>>>(g, value, old, o, want_mf);
+    else k_value_diff<false><<<(int)blocks, 256, 0, s>>>(g, value, old, o, want_mf);
 }
 void launch_sssp_diff(const GraphView &g, const uint32_t *dist, uint32_t *dist_old, uint64_t *out_bits,
                       uint64_t *out_summ, uint32_t *out_offsets, DevStats *st, cudaStream_t s) {

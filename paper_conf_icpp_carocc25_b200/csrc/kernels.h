@@ -190,6 +190,10 @@ void launch_push_sweep(const ScsrView &v, const int64_t *rp, const uint64_t *in_
                        const uint32_t *offsets, int64_t nw2, DevStats *st, uint64_t *visited,
                        unsigned long long min_mf, cudaStream_t s);
 
+// ablate.cu — word-width ablation (f3): push-only 2LB BFS with 32- or 64-bit words, host loop;
+// returns 0 on success, the supersteps and the device time
+int ablation_bfs_words(const GraphView &g, int32_t src, uint32_t *level, int word_bits, cudaStream_t s, int64_t *iters,
+                       float *ms);
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 // level init + seed + the seed frontier's word list / statistics + first decision, one kernel
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,

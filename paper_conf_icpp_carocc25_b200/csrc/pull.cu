@@ -64,6 +64,9 @@ constexpr int PULL_ARCS = SG_PULL_ARCS;
 #if SG_PULL_PF && SG_PULL_WSKIP
 #error "SG_PULL_PF assumes every round loads its visited word: build it with SG_PULL_WSKIP=0"
 #endif
+#ifndef SG_PULL_COUNT_SCANS
+#define SG_PULL_COUNT_SCANS 1   // count list-scanned vertices (16 B of row_ptr each in the roofline bytes)
+#endif
 #ifndef SG_PULL_MINB
 #define SG_PULL_MINB 8
 #endif
@@ -93,6 +96,7 @@ __device__ __forceinline__ bool pull_scan(const GraphView &g, const uint32_t *__
     return hit;
 }
 
+template <bool P>
 __global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
            BfsOut o) {
@@ -108,6 +112,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
     uint32_t *const lvl = o.level_pp ? *o.level_pp : o.level;
     const uint32_t nx = o.next_ptr ? *o.next_ptr : o.next;
     unsigned long long nf = 0, mf = 0, arcs = 0;
+    uint32_t scans = 0;
     const int lane = lane_id(), wid = threadIdx.x >> 5;
     const uint32_t *in32 = reinterpret_cast<const uint32_t *>(in_bits);
     const int64_t nq = g.nw1 * 16;
@@ -146,8 +151,8 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
         const uint32_t mxw = max(s_mx[par][0], s_mx[par][1]);
         par ^= 1;
         if (full == ~0ull) {
-            if (threadIdx.x < 64 && sw * 64 + threadIdx.x < g.nw1) xstore(o.x, o.out_bits + sw * 64 + threadIdx.x, 0ull);
-            if (threadIdx.x == 0) xstore(o.x, o.out_summ + sw, 0ull);
+            if (threadIdx.x < 64 && sw * 64 + threadIdx.x < g.nw1) xstore<P>(o.x, o.out_bits + sw * 64 + threadIdx.x, 0ull);
+            if (threadIdx.x == 0) xstore<P>(o.x, o.out_summ + sw, 0ull);
             continue;
         }
 #if SG_PULL_WORD_MAX > 0
@@ -181,12 +186,15 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                             arcs++;
                             hit = (x[k] >> (c[k] & 31)) & 1u;
                         }
-                        if (!hit) hit = pull_scan(g, in32, w * 64 + b[k], arcs);
+                        if (!hit) {
+                            if (SG_PULL_COUNT_SCANS) scans++;
+                            hit = pull_scan(g, in32, w * 64 + b[k], arcs);
+                        }
                         if (hit) nbw |= 1ull << b[k];
                     }
                 }
                 if (w < g.nw1) {
-                    xstore(o.x, o.out_bits + w, nbw);
+                    xstore<P>(o.x, o.out_bits + w, nbw);
                     if (nbw) {
                         visited[w] = my_vis | nbw;
                         o.vis_old[w] = my_vis | nbw;
@@ -204,7 +212,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             __syncthreads();
             if (threadIdx.x == 0) s_S[0] = s_wm[0] | (s_wm[1] << 32);
             __syncthreads();
-            bfs_emit_words(o, g.w2_hi, sw, s_S, 1, s_base);
+            bfs_emit_words<P>(o, g.w2_hi, sw, s_S, 1, s_base);
             continue;
         }
 #endif
@@ -216,7 +224,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             const int64_t w = qd >> 4;
 #if SG_PULL_WSKIP
             if (((full >> (r * (PULL_THREADS / 16) + wid * 2)) & 3ull) == 3ull) {
-                if ((lane & 15) == 0 && ok) xstore(o.x, o.out_bits + w, 0ull);
+                if ((lane & 15) == 0 && ok) xstore<P>(o.x, o.out_bits + w, 0ull);
                 continue;
             }
 #endif
@@ -232,7 +240,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             const uint32_t valid = !ok ? 0u : rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
             const uint32_t unv = (uint32_t)(~vis >> sh) & valid;
             if (__all_sync(0xffffffffu, unv == 0u)) {   // the warp's two words are fully visited:
-                if ((lane & 15) == 0 && ok) xstore(o.x, o.out_bits + w, 0ull);   // no new vertices, no work
+                if ((lane & 15) == 0 && ok) xstore<P>(o.x, o.out_bits + w, 0ull);   // no new vertices, no work
                 continue;
             }
             uint32_t found = 0, codes = 0;
@@ -253,6 +261,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                 // 2. list scans of the vertices whose candidate missed
                 for (uint32_t miss = unv & ~found; miss; miss &= miss - 1) {
                     const int k = __ffs(miss) - 1;
+                    if (SG_PULL_COUNT_SCANS) scans++;
                     const bool hit = pull_scan(g, in32, v0 + k, arcs);
                     if (hit) found |= 1u << k;
                 }
@@ -274,7 +283,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
                     if ((t >> (16 * i)) & 1u) lw[16 * i] = nx;
             }
             if ((lane & 15) == 0 && ok) {
-                xstore(o.x, o.out_bits + w, nb);   // every output word is written
+                xstore<P>(o.x, o.out_bits + w, nb);   // every output word is written
                 if (nb) {
                     visited[w] = vis | nb;
                     o.vis_old[w] = vis | nb;
@@ -291,14 +300,15 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             s_S[0] = S;
         }
         __syncthreads();
-        bfs_emit_words(o, g.w2_hi, sw, s_S, 1, s_base);
+        bfs_emit_words<P>(o, g.w2_hi, sw, s_S, 1, s_base);
     }
-    bfs_finish(o, nf, mf, arcs, st);
+    bfs_finish<P>(o, nf, mf, arcs, st, scans);
 }
 
 // Late pull steps (few unvisited vertices left): one warp per layer-2 word (pullw.cuh), no CTA
 // barrier, misses drained cooperatively.  Runs iff ctrl->pull_warp (graph mode; both kernels are
 // in the pull node and the other one returns at once) or o.pull_warp (host loop).
+template <bool P>
 __global__ void __launch_bounds__(256, 4)
 k_pull_bfs_w(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
              BfsOut o) {
@@ -311,31 +321,35 @@ k_pull_bfs_w(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__rest
     const uint32_t nx = o.next_ptr ? *o.next_ptr : o.next;
     const int wid = threadIdx.x >> 5;
     const uint32_t *in32 = reinterpret_cast<const uint32_t *>(in_bits);
-    unsigned long long nf = 0, mf = 0, arcs = 0;
+    unsigned long long nf = 0, mf = 0, arcs = 0, scans = 0;
     const int64_t gwarp = (int64_t)blockIdx.x * 8 + wid, nwarps = (int64_t)gridDim.x * 8;
     for (int64_t sw = g.w2_lo + gwarp; sw < g.w2_hi; sw += nwarps)
-        pull_l2_warp(g, sw, in32, visited, o, s_w[wid], s_lut, lvl, nx, nf, mf, arcs);
-    bfs_finish(o, nf, mf, arcs, st);
+        pull_l2_warp<P>(g, sw, in32, visited, o, s_w[wid], s_lut, lvl, nx, nf, mf, arcs, scans);
+    bfs_finish<P>(o, nf, mf, arcs, st, scans);
 }
 
 void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,
                      cudaStream_t s) {
-    // graph mode launches both kernels (the device-side decision picks one); the host loop one
-    const bool both = o.ctrl != nullptr;
+    // graph mode launches both kernels (the device-side decision picks one; with the late-pull rule
+    // off, SG_PULL_WARP_FRAC=0, only the CTA kernel); the host loop launches one
+    const char *fr = getenv("SG_PULL_WARP_FRAC");
+    const bool both = o.ctrl != nullptr && !(fr && atoi(fr) == 0);
     if (both || !o.pull_warp) {
         // one CTA per layer-2 word in a grid-stride loop over SG_PULL_WAVES CTAs per SM
         int64_t blocks = g.w2_hi - g.w2_lo;
         if (blocks > num_sms() * SG_PULL_WAVES) blocks = num_sms() * SG_PULL_WAVES;
         if (blocks < 1) blocks = 1;
         note_launch();
-        k_pull_bfs<<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);
+        if (o.x.nranks > 1) k_pull_bfs<true><<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);
+        else k_pull_bfs<false><<<(int)blocks, PULL_THREADS, 0, s>>>(g, in_bits, visited, st, o);
     }
-    if (both || o.pull_warp) {
+    if (both || (o.ctrl == nullptr && o.pull_warp)) {
         int64_t blocks = (g.w2_hi - g.w2_lo + 7) / 8;   // one warp per layer-2 word
         if (blocks > num_sms() * 4) blocks = num_sms() * 4;
         if (blocks < 1) blocks = 1;
         note_launch();
-        k_pull_bfs_w<<<(int)blocks, 256, 0, s>>>(g, in_bits, visited, st, o);
+        if (o.x.nranks > 1) k_pull_bfs_w<true><<<(int)blocks, 256, 0, s>>>(g, in_bits, visited, st, o);
+        else k_pull_bfs_w<false><<<(int)blocks, 256, 0, s>>>(g, in_bits, visited, st, o);
     }
 }
 

@@ -111,10 +111,12 @@ __device__ __forceinline__ void p2_drain(const GraphView &g, const uint32_t *__r
 
 // One layer-2 word `sw` on one warp (visited words, candidates, queue drain, output words, layer-2
 // word, list append).  Warp-synchronous; no CTA barrier.
+template <bool P>
 __device__ __forceinline__ void pull_l2_warp(const GraphView &g, int64_t sw, const uint32_t *__restrict__ in32,
                                              uint64_t *__restrict__ visited, const BfsOut &o, P2Warp &W,
                                              const uint32_t *s_lut, uint32_t *lvl, uint32_t nx, unsigned long long &nf,
-                                             unsigned long long &mf, unsigned long long &arcs) {
+                                             unsigned long long &mf, unsigned long long &arcs,
+                                             unsigned long long &scans) {
     const int lane = lane_id();
     // ---- the layer-2 word's 64 visited words: lane owns wa = 64 sw + lane and wb = wa + 32 ----
     const int64_t wa = sw * 64 + lane, wb = wa + 32;
@@ -127,9 +129,9 @@ __device__ __forceinline__ void pull_l2_warp(const GraphView &g, int64_t sw, con
     const uint64_t ua = ~va & valid(wa), ub = ~vb & valid(wb);
     const uint32_t fa = __ballot_sync(0xffffffffu, ua == 0ull), fb = __ballot_sync(0xffffffffu, ub == 0ull);
     if ((fa & fb) == 0xffffffffu) {   // no unvisited vertex: 64 zero output words
-        if (wa < g.nw1) xstore(o.x, o.out_bits + wa, 0ull);
-        if (wb < g.nw1) xstore(o.x, o.out_bits + wb, 0ull);
-        if (lane == 0) xstore(o.x, o.out_summ + sw, 0ull);
+        if (wa < g.nw1) xstore<P>(o.x, o.out_bits + wa, 0ull);
+        if (wb < g.nw1) xstore<P>(o.x, o.out_bits + wb, 0ull);
+        if (lane == 0) xstore<P>(o.x, o.out_summ + sw, 0ull);
         return;
     }
     W.found[lane] = 0ull;
@@ -180,6 +182,7 @@ __device__ __forceinline__ void pull_l2_warp(const GraphView &g, int64_t sw, con
 #pragma unroll
                 for (int k = 0; k < 4; k++)
                     if ((miss >> k) & 1u) W.q[pos++] = (int32_t)(w * 64 + b[k]);
+                scans += (unsigned)cnt;
                 nq += tot;
                 __syncwarp();
             }
@@ -261,6 +264,7 @@ __device__ __forceinline__ void pull_l2_warp(const GraphView &g, int64_t sw, con
 #pragma unroll
                 for (int k = 0; k < 4; k++)
                     if ((miss >> k) & 1u) W.q[pos++] = (int32_t)(v0 + k);
+                scans += (unsigned)cnt;
                 nq += tot;
             }
             __syncwarp();
@@ -271,14 +275,14 @@ __device__ __forceinline__ void pull_l2_warp(const GraphView &g, int64_t sw, con
     // ---- output: 64 words, visited / vis_old, layer-2 word, list entries ----
     const uint64_t na = W.found[lane], nbw = W.found[lane + 32];
     if (wa < g.nw1) {
-        xstore(o.x, o.out_bits + wa, na);
+        xstore<P>(o.x, o.out_bits + wa, na);
         if (na) {
             visited[wa] = va | na;
             o.vis_old[wa] = va | na;
         }
     }
     if (wb < g.nw1) {
-        xstore(o.x, o.out_bits + wb, nbw);
+        xstore<P>(o.x, o.out_bits + wb, nbw);
         if (nbw) {
             visited[wb] = vb | nbw;
             o.vis_old[wb] = vb | nbw;
@@ -289,11 +293,12 @@ __device__ __forceinline__ void pull_l2_warp(const GraphView &g, int64_t sw, con
     const int tot = __popcll(S);
     unsigned long long base[SG_MAX_RANKS + 1] = {};
     if (lane == 0) {
-        xstore(o.x, o.out_summ + sw, S);
+        xstore<P>(o.x, o.out_summ + sw, S);
         if (tot) {
             base[0] = atomicAdd(&o.st->count, (unsigned long long)tot);
-            for (int j = 0; j < o.x.nranks; j++)
-                if (j != o.x.rank) base[1 + j] = atomicAdd(&xpeer(o.x, o.st, j)->count, (unsigned long long)tot);
+            if (P)
+                for (int j = 0; j < o.x.nranks; j++)
+                    if (j != o.x.rank) base[1 + j] = atomicAdd(&xpeer(o.x, o.st, j)->count, (unsigned long long)tot);
         }
     }
     if (tot) {
@@ -302,7 +307,7 @@ __device__ __forceinline__ void pull_l2_warp(const GraphView &g, int64_t sw, con
         const unsigned long long b0 = __shfl_sync(0xffffffffu, base[0], 0);
         if (na) o.out_offsets[b0 + pa] = (uint32_t)wa;
         if (nbw) o.out_offsets[b0 + pb] = (uint32_t)wb;
-        for (int j = 0; j < o.x.nranks; j++) {
+        for (int j = 0; P && j < o.x.nranks; j++) {
             if (j == o.x.rank) continue;
             const unsigned long long bj = __shfl_sync(0xffffffffu, base[1 + j], 0);
             if (na) xpeer(o.x, o.out_offsets, j)[bj + pa] = (uint32_t)wa;

@@ -22,12 +22,12 @@ __device__ __forceinline__ T *xpeer(const Xchg &x, T *p, int j) {
     return reinterpret_cast<T *>(reinterpret_cast<char *>(p) + x.delta[j]);
 }
 
-// store v at p locally and in every peer replica
-template <class T, class V>
+// store v at p locally and in every peer replica (P = false: single-GPU instantiation, local only)
+template <bool P = true, class T, class V>
 __device__ __forceinline__ void xstore(const Xchg &x, T *p, V vv) {
     const T v = (T)vv;
     *p = v;
-    if (x.nranks > 1) {
+    if (P && x.nranks > 1) {
 #pragma unroll
         for (int j = 0; j < SG_MAX_RANKS; j++)
             if (j < x.nranks && j != x.rank) *xpeer(x, p, j) = v;

@@ -83,6 +83,25 @@ def main():
             base = base or ms
             print(json.dumps({"graph": gname, "n": g.n, "nnz": g.nnz, "variant": name, "ms_per_bfs": ms,
                               "gteps": statistics.median(teps), "speedup_vs_plain": base / ms}), flush=True)
+        # word width (§4.3: 32-bit words "to match a warp on NVIDIA"): the self-contained
+        # push-only 2LB BFS of ablate.cu with 32- and 64-bit words, otherwise identical
+        for wb in (32, 64):
+            times, teps = [], []
+            for s in roots:
+                sg.ablation_bfs(G, int(s), wb, level)
+                t = []
+                for _ in range(args.reps):
+                    _, st = sg.ablation_bfs(G, int(s), wb, level)
+                    t.append(st.device_ms)
+                lv = sg.as_u32(level)
+                assert np.array_equal(lv, ref[int(s)]), ("word", wb, s)
+                ms = statistics.median(t)
+                times.append(ms)
+                teps.append(int(deg[lv != 0xFFFFFFFF].sum()) // 2 / (ms / 1e3) / 1e9)
+            print(json.dumps({"graph": gname, "n": g.n, "nnz": g.nnz,
+                              "variant": f"word-width ablation: {wb}-bit words, paper mapping (warp per word, "
+                                         f"lanes stride the list), 2LB, push-only, host loop",
+                              "ms_per_bfs": statistics.median(times), "gteps": statistics.median(teps)}), flush=True)
         del G
 
 

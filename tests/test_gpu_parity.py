@@ -558,3 +558,15 @@ def test_sssp_cc_graph_driven_equals_host_loop(sg, monkeypatch, make):
             lab2, st2 = sg.run_cc(G, direction=dr, host_loop=True)
             assert np.array_equal(lab.cpu().numpy(), ref) and np.array_equal(lab2.cpu().numpy(), ref)
             assert st.iterations >= 1 and st.push_steps + st.pull_steps == st.iterations
+
+
+@pytest.mark.parametrize("bits", [32, 64])
+@pytest.mark.parametrize("make", [lambda: gen.rmat(13, 16, permute=True), lambda: gen.path(200),
+                                  lambda: gen.lattice(70, 90, 0.6, seed=2), lambda: gen.empty_graph(100)])
+def test_word_width_ablation_bfs(sg, make, bits):
+    """sg_ablation_bfs (f3): the 32- and 64-bit-word push-only 2LB BFS reach the oracle's levels."""
+    g = make()
+    G = load(sg, g)
+    for s in list(gen.sources(g, 2)) + [0, g.n - 1]:
+        lv, st = sg.ablation_bfs(G, int(s), bits)
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (bits, s)
