@@ -27,7 +27,10 @@ constexpr size_t SEG_SMEM = (size_t)SEG_WORDS * sizeof(uint64_t);
 #define SG_SEG_OWNER 1   // 1: a CTA owns one segment (one slice load / flush); 0: every CTA walks all
 #endif
 #ifndef SG_SEG_UNROLL
-#define SG_SEG_UNROLL 4
+#define SG_SEG_UNROLL 8
+#endif
+#ifndef SG_SEG_LQ
+#define SG_SEG_LQ 4   // long parts: int4 loads per lane in flight per iteration (2 / 4 / 8 measured: 4)
 #endif
 #ifndef SG_SEG_LONG
 #define SG_SEG_LONG 192
@@ -109,18 +112,25 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
                         if (!(s_vis32[vv >> 5] & m)) atomicOr(s_vis32 + (vv >> 5), m);
                     }
                 }
-                for (int64_t i = a + 4 * lane; i < bb; i += 256) {
-                    const bool two = i + 128 < bb;
-                    const int4 q0 = __ldg(reinterpret_cast<const int4 *>(p.g.col + i));
-                    int4 q1 = make_int4(vbase, vbase, vbase, vbase);
-                    if (two) q1 = __ldg(reinterpret_cast<const int4 *>(p.g.col + i + 128));
-                    const int32_t vv[8] = {q0.x - vbase, q0.y - vbase, q0.z - vbase, q0.w - vbase,
-                                           q1.x - vbase, q1.y - vbase, q1.z - vbase, q1.w - vbase};
+                // SG_SEG_LQ int4 loads per lane per iteration (4 * SG_SEG_LQ arcs), all issued
+                // before any shared-memory update: 128 * SG_SEG_LQ arcs of the part in flight per warp
+                for (int64_t i = a + 4 * lane; i < bb; i += 128 * SG_SEG_LQ) {
+                    int4 q[SG_SEG_LQ];
 #pragma unroll
-                    for (int k = 0; k < 8; k++) {
-                        if (k >= 4 && !two) break;
-                        const uint32_t m = 1u << (vv[k] & 31);
-                        if (!(s_vis32[vv[k] >> 5] & m)) atomicOr(s_vis32 + (vv[k] >> 5), m);
+                    for (int u = 0; u < SG_SEG_LQ; u++) {
+                        const int64_t iu = i + 128 * u;
+                        q[u] = iu < bb ? __ldg(reinterpret_cast<const int4 *>(p.g.col + iu))
+                                       : make_int4(-1 + vbase, -1 + vbase, -1 + vbase, -1 + vbase);
+                    }
+#pragma unroll
+                    for (int u = 0; u < SG_SEG_LQ; u++) {
+                        const int32_t vv[4] = {q[u].x - vbase, q[u].y - vbase, q[u].z - vbase, q[u].w - vbase};
+#pragma unroll
+                        for (int k = 0; k < 4; k++) {
+                            if (vv[k] < 0) continue;
+                            const uint32_t m = 1u << (vv[k] & 31);
+                            if (!(s_vis32[vv[k] >> 5] & m)) atomicOr(s_vis32 + (vv[k] >> 5), m);
+                        }
                     }
                 }
             }

@@ -22,7 +22,8 @@ roots = gen.config_sources(cfg, g)
 G = sg.graph_load_csr(g.row_ptr, g.col_idx)
 d = {"push": sg.SG_DIR_PUSH, "pull": sg.SG_DIR_PULL, "auto": sg.SG_DIR_AUTO}[mode]
 seg = int(os.environ.get("SG_SEGMENTED", "0"))
+alpha = float(os.environ.get("SG_ALPHA", "14"))
 # host-driven loop: ncu cannot profile kernels inside graphs with conditional nodes
-lv, st = sg.run_bfs(G, int(roots[ri]), direction=d, host_loop=True, segmented=seg)
+lv, st = sg.run_bfs(G, int(roots[ri]), direction=d, host_loop=True, segmented=seg, alpha=alpha)
 torch.cuda.synchronize()
 print(st.as_dict())
