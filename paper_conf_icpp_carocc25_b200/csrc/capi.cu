@@ -1353,7 +1353,8 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     Workspace *ws = g->ws;
     cudaStream_t s = stream_of(&o);
     const int32_t sc_mode = t.scsr != 0 && g->scsr_state == 1 ? t.scsr : 0;
-    const int shape = (env_or("SG_SPARSE", 0) != 0 ? 1 : 0) | (env_or("SG_PULL_WARP_FRAC", 8) != 0 ? 2 : 0);
+    const int shape = (env_or("SG_SPARSE", 0) != 0 ? 1 : 0) | (env_or("SG_PULL_WARP_FRAC", 8) != 0 ? 2 : 0) |
+                      ((int)env_or("SG_PULL_WORD_MAX", 16) << 2);   // knobs baked into the captured graph
     if (!ws->bfs_exec || ws->bfs_heavy != t.heavy || ws->bfs_small != t.small || ws->bfs_seg != t.seg ||
         ws->bfs_cf != t.cf || ws->bfs_scsr != sc_mode || ws->bfs_shape != shape) {
         TRY(build_bfs_graph(g, t));

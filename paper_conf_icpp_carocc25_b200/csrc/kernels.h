@@ -104,6 +104,8 @@ struct BfsOut {
     int32_t half = 0;                 // graph mode: index (0/1) of the INPUT frontier buffer
     int32_t sparse = 0;               // 1: the superstep consumed (zeroed) its input (sparse.cu)
     int32_t pull_warp = 0;            // host loop: 1 = the pull runs warp-owned layer-2 words (graph mode: ctrl)
+    int32_t word_max = 16;            // CTA pull: word mode when no layer-1 word has more unvisited vertices
+                                      // (SG_PULL_WORD_MAX at launch / capture; 0 = off)
     ValCtrl *vctrl = nullptr;         // graph-driven SSSP / CC: the last CTA runs val_decide
 };
 // device-driven SSSP / CC: the first decision (after the prologue compacted the input), one thread

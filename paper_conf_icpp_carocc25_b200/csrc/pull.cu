@@ -156,7 +156,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             continue;
         }
 #if SG_PULL_WORD_MAX > 0
-        if (mxw <= SG_PULL_WORD_MAX) {
+        if (mxw <= (uint32_t)o.word_max) {
             // word mode (late pull steps: a few unvisited vertices per word): thread t < 64 owns
             // layer-1 word sw*64+t and walks its unvisited vertices one by one (candidate test,
             // then the list scan), so the CTA spends 2 warps instead of 32 quad rounds on it.
@@ -328,8 +328,13 @@ k_pull_bfs_w(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__rest
     bfs_finish<P>(o, nf, mf, arcs, st, scans);
 }
 
-void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o,
+void launch_pull_bfs(const GraphView &g, const uint64_t *in_bits, uint64_t *visited, DevStats *st, const BfsOut &o_in,
                      cudaStream_t s) {
+    BfsOut o = o_in;
+    {   // word-mode threshold of the CTA kernel: a runtime parameter (tests force 0 / 64)
+        const char *wm = getenv("SG_PULL_WORD_MAX");
+        o.word_max = wm ? atoi(wm) : SG_PULL_WORD_MAX;
+    }
     // graph mode launches both kernels (the device-side decision picks one; with the late-pull rule
     // off, SG_PULL_WARP_FRAC=0, only the CTA kernel); the host loop launches one
     const char *fr = getenv("SG_PULL_WARP_FRAC");

@@ -570,3 +570,43 @@ def test_word_width_ablation_bfs(sg, make, bits):
     for s in list(gen.sources(g, 2)) + [0, g.n - 1]:
         lv, st = sg.ablation_bfs(G, int(s), bits)
         assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s))), (bits, s)
+
+
+@pytest.mark.parametrize("word_max", ["0", "4", "64"])
+@pytest.mark.parametrize("host_loop", [False, True])
+def test_bfs_pull_word_mode_threshold(sg, monkeypatch, word_max, host_loop):
+    """The CTA pull's word mode (a thread per layer-1 word, pull.cu) is a runtime threshold:
+    off (0), narrow (4) and forced on dense words (64) all give the oracle's levels, with and
+    without the late warp-owned pulls (SG_PULL_WARP_FRAC=0 keeps every pull on the CTA kernel)."""
+    g = gen.rmat(15, 16, permute=True)
+    G = load(sg, g)
+    monkeypatch.setenv("SG_PULL_WORD_MAX", word_max)
+    for frac in ("0", "8"):
+        monkeypatch.setenv("SG_PULL_WARP_FRAC", frac)
+        for s in gen.sources(g, 3):
+            ref = oracle.bfs(g, int(s))
+            for d in (sg.SG_DIR_PULL, sg.SG_DIR_AUTO):
+                lv, _ = sg.run_bfs(G, int(s), direction=d, host_loop=host_loop)
+                assert np.array_equal(sg.as_u32(lv), ref), (word_max, frac, d)
+
+
+def test_bfs_pull_128_thread_variant(sg):
+    """The SG_PULL_THREADS=128 layout (a measured round-1 variant) built as its own library and
+    run in a subprocess: pull-only and auto BFS equal the oracle."""
+    import os
+    import subprocess
+    import sys
+    from paper_conf_icpp_carocc25_b200 import _build
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    lib = _build.build(defines=("SG_PULL_THREADS=128",), lib=os.path.join(root, "build", "variants", "pull128",
+                                                                          "libsygraph.so"))
+    code = ("import numpy as np, gen, oracle, paper_conf_icpp_carocc25_b200 as sg\n"
+            "g = gen.rmat(14, 16, permute=True); G = sg.graph_load_csr(g.row_ptr, g.col_idx)\n"
+            "for s in gen.sources(g, 3):\n"
+            "    for d in (sg.SG_DIR_PULL, sg.SG_DIR_AUTO):\n"
+            "        lv, _ = sg.run_bfs(G, int(s), direction=d)\n"
+            "        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s)))\n"
+            "print('ok')\n")
+    env = dict(os.environ, SYGRAPH_LIB=lib, PYTHONPATH=root)
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, cwd=root)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
