@@ -346,7 +346,9 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
-        os.environ.setdefault("OMP_NUM_THREADS", str(max(1, (os.cpu_count() or 8) // world)))
+        # torchrun sets OMP_NUM_THREADS=1; rank 0 alone runs the (OpenMP) generator for all ranks
+        # (shared_graph), so give it the host's cores
+        os.environ["OMP_NUM_THREADS"] = str(os.cpu_count() or 8)
     if args.impl == "reference":
         return run_reference(args, rank)
 

@@ -248,7 +248,7 @@ static int ensure_ws(sg_graph *g) {
     CK(cudaMemset(ws->bfs_done, 0, sizeof(unsigned int)));
     CK(cudaMalloc(&ws->gbar, 4 * sizeof(unsigned int)));
     CK(cudaMemset(ws->gbar, 0, 4 * sizeof(unsigned int)));
-    CK(cudaMalloc(&ws->visited, sizeof(uint64_t) * (size_t)g->v.nw1));
+    CK(cudaMalloc(&ws->visited, sizeof(uint64_t) * (size_t)(g->v.nw1 + 8)));   // +8: 16-B bulk copies of a tail
     CK(cudaMalloc(&ws->vis_old, sizeof(uint64_t) * (size_t)g->v.nw1));
     CK(cudaMalloc(&ws->scratch, 8 * sizeof(unsigned long long)));
     CK(cudaMallocHost(&ws->h_scratch, 8 * sizeof(unsigned long long)));

@@ -40,6 +40,8 @@ constexpr uint32_t SEG_LONG = SG_SEG_LONG;   // parts at least this long are str
 
 __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs f) {
     extern __shared__ __align__(16) uint64_t s_vis[];
+    __shared__ __align__(8) uint64_t s_bar;   // slice load: cp.async.bulk completion
+    __shared__ uint32_t s_next;                 // next item batch (dynamic deal to warps)
     const unsigned long long cnt = p.st->seg_count;
     const uint32_t nitems = (uint32_t)(cnt < p.seg_cap ? cnt : p.seg_cap);
     if (nitems == 0) return;
@@ -62,6 +64,8 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
 #endif
     const int warp = threadIdx.x >> 5, lane = lane_id();
     constexpr int NW = SEG_THREADS / 32;
+    uint32_t bar_phase = 0u;
+    bool bar_ready = false;
     uint32_t *level = f.level_pp ? *f.level_pp : f.level;
     const uint32_t next = f.next_ptr ? *f.next_ptr : f.next;
 #if SG_SEG_OWNER
@@ -71,15 +75,45 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
 #endif
         const int64_t w0 = (int64_t)b * SEG_WORDS;
         const int nw = (int)min((int64_t)SEG_WORDS, p.g.nw1 - w0);
-        for (int i = threadIdx.x; i < nw; i += SEG_THREADS) s_vis[i] = f.visited[w0 + i];
+        // the slice (up to 192 KB) arrives by TMA bulk copies (one mbarrier, copies of <= 48 KB):
+        // a thread-per-word copy loop was latency-bound (24 dependent load/store rounds per thread,
+        // 28 % of the kernel's stall samples in ncu); visited carries 8 words of tail padding
+        if (threadIdx.x == 0) {
+            s_next = 0u;
+            if (bar_phase == 0u && !bar_ready) {
+                mbar_init(&s_bar, 1);
+                asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+            }
+            // the previous segment's shared-memory atomics (generic proxy) before the async copy
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            const uint32_t bytes = (uint32_t)((((int64_t)nw * 8) + 15) & ~15ll);
+            mbar_expect_tx(&s_bar, bytes);
+            constexpr uint32_t PIECE = 48 * 1024;
+            for (uint32_t o = 0; o < bytes; o += PIECE)
+                bulk_g2s(reinterpret_cast<char *>(s_vis) + o, reinterpret_cast<const char *>(f.visited + w0) + o,
+                         min(PIECE, bytes - o), &s_bar);
+        }
+        bar_ready = true;
         __syncthreads();
+        mbar_wait(&s_bar, bar_phase);
+        bar_phase ^= 1u;
         const int32_t vbase = (int32_t)(w0 * 64);
         uint32_t *s_vis32 = reinterpret_cast<uint32_t *>(s_vis);   // 32-bit ATOMS.OR is native (64-bit is a CAS loop)
         // items are dealt to warps with stride NW: consecutive chunks of one hub (which fall into
         // the same segment) spread over all warps instead of piling onto one
-        for (uint32_t r = 0; i0 + r * 32 * NW + warp < i1; r++) {
-            // lane k: the part of item i0 + (r*32 + k)*NW + warp inside segment b
-            const uint32_t item = i0 + (r * 32 + lane) * NW + warp;
+        // batches (r, slot) = the items i0 + (r*32 + k)*NW + slot, k = lane (consecutive chunks of
+        // one hub spread over batches), taken dynamically by the warps: part lengths vary 0..4096,
+        // a static deal left warps idle at the flush barrier (ncu: barrier stalls 5.1)
+        const uint32_t nbatch = ((i1 - i0 + 32 * NW - 1) / (32 * NW)) * NW;
+        for (;;) {
+            uint32_t q = 0;
+            if (lane == 0) q = atomicAdd(&s_next, 1u);
+            q = __shfl_sync(0xffffffffu, q, 0);
+            if (q >= nbatch) break;
+            const uint32_t r = q / NW, slot = q % NW;
+            if (i0 + r * 32 * NW + slot >= i1) continue;
+            // lane k: the part of item i0 + (r*32 + k)*NW + slot inside segment b
+            const uint32_t item = i0 + (r * 32 + lane) * NW + slot;
             int64_t lo = 0;
             uint32_t len = 0;
             if (item < i1) {
@@ -93,38 +127,59 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
                     len = (uint32_t)(e - a);
                 }
             }
-            // long parts: the whole warp streams each with 16-B loads (no per-arc owner search)
-            uint32_t longm = __ballot_sync(0xffffffffu, len >= SEG_LONG);
-            while (longm) {
-                const int src = __ffs(longm) - 1;
-                longm &= longm - 1;
-                const int64_t s = __shfl_sync(0xffffffffu, lo, src);
-                const int64_t e = s + __shfl_sync(0xffffffffu, len, src);
-                int64_t a = (s + 3) & ~3ll;
-                const int64_t bb = a + ((e - a) & ~3ll);
-                {   // ragged head [s, a) on lanes 0..2, tail [bb, e) on lanes 4..6
-                    int64_t i = -1;
-                    if (lane < a - s) i = s + lane;
-                    else if (lane >= 4 && lane - 4 < e - bb) i = bb + (lane - 4);
-                    if (i >= 0) {
-                        const int32_t vv = __ldg(p.g.col + i) - vbase;
-                        const uint32_t m = 1u << (vv & 31);
-                        if (!(s_vis32[vv >> 5] & m)) atomicOr(s_vis32 + (vv >> 5), m);
-                    }
+            // long parts: the whole warp streams each with 16-B loads (no per-arc owner search).
+            // Each lane first handles the ragged head / tail (< 4 arcs each) of its own part; the
+            // aligned bodies are then walked as one sequence of 128*LQ-arc windows over the
+            // warp's long parts, the next window's loads issued before the current one's
+            // shared-memory updates (software pipelining across windows and parts).
+            const bool is_long = len >= SEG_LONG;
+            const uint32_t longm = __ballot_sync(0xffffffffu, is_long);
+            int64_t la = 0, lb = 0;
+            if (is_long) {
+                const int64_t e = lo + len;
+                la = (lo + 3) & ~3ll;
+                lb = la + ((e - la) & ~3ll);
+                for (int64_t i = lo; i < la; i++) {
+                    const int32_t vv = __ldg(p.g.col + i) - vbase;
+                    const uint32_t m = 1u << (vv & 31);
+                    if (!(s_vis32[vv >> 5] & m)) atomicOr(s_vis32 + (vv >> 5), m);
                 }
-                // SG_SEG_LQ int4 loads per lane per iteration (4 * SG_SEG_LQ arcs), all issued
-                // before any shared-memory update: 128 * SG_SEG_LQ arcs of the part in flight per warp
-                for (int64_t i = a + 4 * lane; i < bb; i += 128 * SG_SEG_LQ) {
-                    int4 q[SG_SEG_LQ];
+                for (int64_t i = lb; i < e; i++) {
+                    const int32_t vv = __ldg(p.g.col + i) - vbase;
+                    const uint32_t m = 1u << (vv & 31);
+                    if (!(s_vis32[vv >> 5] & m)) atomicOr(s_vis32 + (vv >> 5), m);
+                }
+            }
+            if (longm) {
+                constexpr int64_t WIN = 128 * SG_SEG_LQ;
+                auto load_win = [&](int4 (&q)[SG_SEG_LQ], int64_t i, int64_t pb) {
 #pragma unroll
                     for (int u = 0; u < SG_SEG_LQ; u++) {
-                        const int64_t iu = i + 128 * u;
-                        q[u] = iu < bb ? __ldg(reinterpret_cast<const int4 *>(p.g.col + iu))
-                                       : make_int4(-1 + vbase, -1 + vbase, -1 + vbase, -1 + vbase);
+                        const int64_t iu = i + 4 * lane + 128 * u;
+                        q[u] = iu < pb ? __ldg(reinterpret_cast<const int4 *>(p.g.col + iu))
+                                       : make_int4(vbase - 1, vbase - 1, vbase - 1, vbase - 1);
                     }
+                };
+                int src = __ffs(longm) - 1;
+                int64_t i = __shfl_sync(0xffffffffu, la, src), pb = __shfl_sync(0xffffffffu, lb, src);
+                int4 cur[SG_SEG_LQ];
+                load_win(cur, i, pb);
+                while (src >= 0) {
+                    int nsrc = src;
+                    int64_t ni = i + WIN, npb = pb;
+                    if (ni >= pb) {   // next part in the mask
+                        const uint32_t rest = longm & ~((2u << src) - 1u);
+                        nsrc = rest ? __ffs(rest) - 1 : -1;
+                        if (nsrc >= 0) {
+                            ni = __shfl_sync(0xffffffffu, la, nsrc);
+                            npb = __shfl_sync(0xffffffffu, lb, nsrc);
+                        }
+                    }
+                    int4 nxt[SG_SEG_LQ];
+                    if (nsrc >= 0) load_win(nxt, ni, npb);
 #pragma unroll
                     for (int u = 0; u < SG_SEG_LQ; u++) {
-                        const int32_t vv[4] = {q[u].x - vbase, q[u].y - vbase, q[u].z - vbase, q[u].w - vbase};
+                        const int32_t vv[4] = {cur[u].x - vbase, cur[u].y - vbase, cur[u].z - vbase, cur[u].w - vbase};
 #pragma unroll
                         for (int k = 0; k < 4; k++) {
                             if (vv[k] < 0) continue;
@@ -132,6 +187,12 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
                             if (!(s_vis32[vv[k] >> 5] & m)) atomicOr(s_vis32 + (vv[k] >> 5), m);
                         }
                     }
+                    if (nsrc < 0) break;
+#pragma unroll
+                    for (int u = 0; u < SG_SEG_LQ; u++) cur[u] = nxt[u];
+                    src = nsrc;
+                    i = ni;
+                    pb = npb;
                 }
             }
             if (len >= SEG_LONG) len = 0;
