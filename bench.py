@@ -49,8 +49,8 @@ def parse():
     p.add_argument("--config", type=int, default=4)
     p.add_argument("--seed", type=int, default=1)
     p.add_argument("--direction", default="auto", choices=["auto", "push", "pull"])
-    p.add_argument("--alpha", type=float, default=14.0)
-    p.add_argument("--beta", type=float, default=24.0)
+    p.add_argument("--alpha", type=float, default=5.0)
+    p.add_argument("--beta", type=float, default=48.0)
     p.add_argument("--heavy-degree", type=int, default=0, help="CTA/grid-tier degree threshold (0: library default)")
     p.add_argument("--scsr", type=int, default=0, help="segmented push advance: 0 auto, 1 off, 2 always")
     p.add_argument("--e2e-steps", type=int, default=3)

@@ -92,7 +92,7 @@ typedef struct {              /* BC forward sigma (P:161 Brandes): dst not in `v
 typedef struct {
     void *stream;             /* cudaStream_t; NULL = legacy default stream */
     int direction;            /* SG_DIR_* for run_bfs (default AUTO = Beamer direction optimising) */
-    double alpha, beta;       /* Beamer thresholds (defaults 14, 24): push->pull when m_f > m_u/alpha,
+    double alpha, beta;       /* Beamer thresholds (defaults 5, 48: tuned on B200, DESIGN R2): push->pull when m_f > m_u/alpha,
                                  pull->push when n_f < n/beta */
     int64_t max_iters;        /* superstep cap (0 = n + 1); exceeding it returns SG_ERR_STATE */
     int32_t heavy_degree;     /* push tiers: degree > heavy_degree goes to the CTA/grid tier (0 = default) */
@@ -254,7 +254,7 @@ SG_API int sg_ctrl_debug(const sg_graph *g, int64_t out[16]);
 SG_API int sg_bfs_trace(const sg_graph *g, int64_t *t_ns, int32_t *kind, int64_t *count, int64_t *nf, int64_t *mf,
                         int32_t cap);
 
-/* Defaults for sg_opts (stream NULL, AUTO direction, alpha 14, beta 24). */
+/* Defaults for sg_opts (stream NULL, AUTO direction, alpha 5, beta 48). */
 SG_API void sg_opts_default(sg_opts *o);
 /* Thread-local message of the last error on this thread ("" if none). */
 SG_API const char *sg_last_error(void);

@@ -162,7 +162,7 @@ def _ptr_mem(a):
     return a.data_ptr(), (SG_MEM_DEVICE if a.is_cuda else SG_MEM_HOST)
 
 
-def opts(stream=None, direction=SG_DIR_AUTO, alpha=14.0, beta=24.0, max_iters=0, heavy_degree=0, small_degree=0,
+def opts(stream=None, direction=SG_DIR_AUTO, alpha=5.0, beta=48.0, max_iters=0, heavy_degree=0, small_degree=0,
          host_loop=False, segmented=0, one_layer=False, coarsening=0, sssp_delta=0, scsr=0, owned_only=False):
     """segmented: BFS hub tier with the visited slice in shared memory (0 auto, 1 off, 2 always);
     one_layer: ablation without the summary layer; coarsening: words per warp grab (0 auto);

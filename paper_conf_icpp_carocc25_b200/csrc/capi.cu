@@ -359,8 +359,8 @@ SG_API void sg_opts_default(sg_opts *o) {
     if (!o) return;
     memset(o, 0, sizeof *o);
     o->direction = SG_DIR_AUTO;
-    o->alpha = 14.0;
-    o->beta = 24.0;
+    o->alpha = 5.0;   // Beamer alpha / beta tuned on B200 (DESIGN R2; profiles/r02_alpha_beta.txt)
+    o->beta = 48.0;
 }
 
 // ---- 1-D destination partition: bounds, blocks, exchange arena -------------------------------
@@ -1442,8 +1442,8 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     if (src < 0 || src >= G.n) return fail(SG_ERR_INVALID, "src %d outside [0,%lld)", src, (long long)G.n);
     sg_opts o;
     if (opts) o = *opts; else sg_opts_default(&o);
-    if (o.alpha <= 0) o.alpha = 14.0;
-    if (o.beta <= 0) o.beta = 24.0;
+    if (o.alpha <= 0) o.alpha = 5.0;
+    if (o.beta <= 0) o.beta = 48.0;
     const int64_t max_iters = o.max_iters > 0 ? o.max_iters : G.n + 1;
     cudaStream_t s = stream_of(&o);
     TRY(ensure_ws(g));

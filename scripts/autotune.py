@@ -22,9 +22,9 @@ import gen  # noqa: E402
 import paper_conf_icpp_carocc25_b200 as sg  # noqa: E402
 
 OPT_KNOBS = {"heavy_degree": [1024, 2048, 4096], "small_degree": [16, 32, 64], "coarsening": [0, 2, 4],
-             "alpha": [10.0, 14.0, 20.0], "beta": [16.0, 24.0, 48.0]}
+             "alpha": [3.0, 5.0, 8.0, 14.0], "beta": [24.0, 48.0, 96.0]}
 ENV_KNOBS = {"SG_PULL_WARP_FRAC": ["0", "8", "16"], "SG_SPARSE": ["0", "1"]}
-DEFAULTS = {"heavy_degree": 2048, "small_degree": 32, "coarsening": 0, "alpha": 14.0, "beta": 24.0,
+DEFAULTS = {"heavy_degree": 2048, "small_degree": 32, "coarsening": 0, "alpha": 5.0, "beta": 48.0,
             "SG_PULL_WARP_FRAC": "8", "SG_SPARSE": "0"}
 
 

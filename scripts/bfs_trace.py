@@ -26,8 +26,8 @@ def main():
     ap.add_argument("--env", nargs="*", default=[""])
     ap.add_argument("--json", default=None)
     ap.add_argument("--quiet", action="store_true")
-    ap.add_argument("--alpha", type=float, default=14.0)
-    ap.add_argument("--beta", type=float, default=24.0)
+    ap.add_argument("--alpha", type=float, default=5.0)
+    ap.add_argument("--beta", type=float, default=48.0)
     ap.add_argument("--segmented", type=int, default=0)
     a = ap.parse_args()
     torch.cuda.set_device(0)
