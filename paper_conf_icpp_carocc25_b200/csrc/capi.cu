@@ -998,7 +998,7 @@ static unsigned long long sweep_threshold(int64_t nnz) {
 }
 // auto mode: the segmented tier pays for its per-segment slice loads only on heavy supersteps
 #ifndef SG_SEG_THRESHOLD_M
-#define SG_SEG_THRESHOLD_M 32
+#define SG_SEG_THRESHOLD_M 8   // (32 in r01; 8: an 18 M-arc level-2 hub push 133 -> 121 us)
 #endif
 static const unsigned long long kSegThreshold = (unsigned long long)SG_SEG_THRESHOLD_M << 20;   // est. frontier arcs
 

@@ -67,8 +67,35 @@ constexpr int PULL_ARCS = SG_PULL_ARCS;
 #ifndef SG_PULL_COUNT_SCANS
 #define SG_PULL_COUNT_SCANS 1   // count list-scanned vertices (16 B of row_ptr each in the roofline bytes)
 #endif
-#ifndef SG_PULL_MINB
-#define SG_PULL_MINB 8
+// Miss queue of the quad rounds (SG_PULL_QUEUE=1): a vertex whose candidate missed is not scanned
+// by its own thread (a quad's up to 4 misses, 2 arcs per dependent round trip each, serialised on
+// one thread: long-scoreboard 13 on the hub-heavy level-2 pulls, profiles/r02h_ncu_full.txt) but
+// appended to a CTA queue in shared memory; after the 4 rounds the CTA drains it: stage A gives
+// each queued vertex a thread for its first SG_PULLQ_SHORT arcs, all loaded and probed together
+// (row bounds -> arcs -> probes: 3 round trips); rows still open go to stage B, a warp per row,
+// 64 arcs per round.  Found bits gather in the layer-2 word's 64 output words in shared memory,
+// written once at the end.  Same set of new vertices as the per-thread scan (any frontier
+// neighbour); only the number of arcs inspected differs (stage A probes a batch past the hit).
+#ifndef SG_PULL_QUEUE
+#define SG_PULL_QUEUE 1
+#endif
+#ifndef SG_PULLQ_SHORT
+#define SG_PULLQ_SHORT 8
+#endif
+constexpr int PQ_CAP = 4096;    // a layer-2 word has 4,096 vertices: the queue never overflows
+#ifndef SG_PULLQ_RB
+#define SG_PULLQ_RB 1   // quad rounds whose loads are issued together (1, 2 or 4 with 256 threads)
+#endif
+constexpr int PQ_RB = SG_PULLQ_RB;
+#ifndef SG_PULLQ2_CAP
+#define SG_PULLQ2_CAP 1024
+#endif
+constexpr int PQ2_CAP = SG_PULLQ2_CAP;   // open rows after stage A (overflow: the thread scans the rest)
+#ifndef SG_PULL_MINB   // resident CTAs per SM the registers are sized for (queue: 40 registers, 6 CTAs
+#define SG_PULL_MINB (SG_PULL_QUEUE ? 6 : 8)   // measured best: 3.37 vs 3.77 ms pull class at 8)
+#endif
+#if SG_PULL_QUEUE && !SG_PULL_WSKIP
+#error "SG_PULL_QUEUE needs SG_PULL_WSKIP (the prologue's visited words)"
 #endif
 // list scan of v: true iff some u in N(v) is in the input frontier (stops at the first hit);
 // PULL_ARCS arcs in flight per step, `arcs` counts the arcs tested
@@ -96,6 +123,79 @@ __device__ __forceinline__ bool pull_scan(const GraphView &g, const uint32_t *__
     return hit;
 }
 
+#if SG_PULL_QUEUE
+// Drain the CTA's miss queue (whole CTA; starts and ends with a barrier).  Found vertices: bit in
+// s_found32 (64 output words as 128 u32 halves), level, n_f / m_f.
+__device__ __forceinline__ void pullq_drain(const GraphView &g, const uint32_t *__restrict__ in32, const int32_t *s_q,
+                                            uint32_t qn, int32_t *s_q2, uint32_t *s_q2n, uint32_t *s_found32,
+                                            uint32_t *lvl, uint32_t nx, const uint32_t *s_lut, unsigned long long &nf,
+                                            unsigned long long &mf, unsigned long long &arcs) {
+    constexpr int S = SG_PULLQ_SHORT;
+    auto mark = [&](int32_t v) {
+        atomicOr(s_found32 + (((v >> 6) & 63) * 2 + ((v >> 5) & 1)), 1u << (v & 31));
+        lvl[v] = nx;
+        nf++;
+        mf += s_lut[__ldg(g.deg8 + v)];
+    };
+    // stage A: a thread per queued vertex, its first S arcs in flight together
+    for (uint32_t i = threadIdx.x; i < qn; i += blockDim.x) {
+        const int32_t v = s_q[i];
+        const int64_t r = __ldg(g.rp + v), e = __ldg(g.rp + v + 1);
+        int32_t u[S];
+        uint32_t y[S];
+#pragma unroll
+        for (int j = 0; j < S; j++) u[j] = r + j < e ? __ldg(g.col + r + j) : -1;
+#pragma unroll
+        for (int j = 0; j < S; j++) y[j] = u[j] >= 0 ? __ldg(in32 + (u[j] >> 5)) : 0u;
+        int hit = -1;
+#pragma unroll
+        for (int j = S - 1; j >= 0; j--)
+            if (u[j] >= 0 && ((y[j] >> (u[j] & 31)) & 1u)) hit = j;
+        if (hit >= 0) {
+            arcs += (unsigned long long)(hit + 1);
+            mark(v);
+        } else {
+            arcs += (unsigned long long)min((int64_t)S, e - r);
+            if (r + S < e) {
+                const uint32_t p = atomicAdd(s_q2n, 1u);
+                if (p < (uint32_t)PQ2_CAP) {
+                    s_q2[p] = v;
+                } else {   // stage-B queue full: scan the rest here
+                    bool h = false;
+                    for (int64_t k = r + S; k < e && !h; k++) {
+                        const int32_t uu = __ldg(g.col + k);
+                        arcs++;
+                        h = (__ldg(in32 + (uu >> 5)) >> (uu & 31)) & 1u;
+                    }
+                    if (h) mark(v);
+                }
+            }
+        }
+    }
+    __syncthreads();
+    // stage B: a warp per open row, 64 arcs per round (2 per lane in flight)
+    const uint32_t q2n = min(*s_q2n, (uint32_t)PQ2_CAP);
+    const int lane = lane_id(), wid = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+    for (uint32_t j = wid; j < q2n; j += nwarp) {
+        const int32_t v = s_q2[j];
+        const int64_t s = __ldg(g.rp + v) + S, e = __ldg(g.rp + v + 1);
+        bool hit = false;
+        for (int64_t r = s; r < e && !hit; r += 64) {
+            const int64_t k0 = r + lane, k1 = r + 32 + lane;
+            const int32_t u0 = k0 < e ? __ldg(g.col + k0) : -1, u1 = k1 < e ? __ldg(g.col + k1) : -1;
+            const uint32_t y0 = u0 >= 0 ? __ldg(in32 + (u0 >> 5)) : 0u, y1 = u1 >= 0 ? __ldg(in32 + (u1 >> 5)) : 0u;
+            const uint32_t b0 = __ballot_sync(0xffffffffu, u0 >= 0 && ((y0 >> (u0 & 31)) & 1u));
+            const uint32_t b1 = __ballot_sync(0xffffffffu, u1 >= 0 && ((y1 >> (u1 & 31)) & 1u));
+            if (lane == 0)
+                arcs += (unsigned long long)(b0 ? __ffs(b0) : b1 ? 32 + __ffs(b1) : (int)min((int64_t)64, e - r));
+            hit = (b0 | b1) != 0u;
+        }
+        if (hit && lane == 0) mark(v);
+    }
+    __syncthreads();
+}
+#endif
+
 template <bool P>
 __global__ void __launch_bounds__(PULL_THREADS, SG_PULL_MINB)
 k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restrict__ visited, DevStats *st,
@@ -105,6 +205,11 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
 #if SG_PULL_WSKIP
     __shared__ uint32_t s_full[2][2], s_mx[2][2];   // double-buffered by iteration parity (no barrier at reuse)
     int par = 0;
+#endif
+#if SG_PULL_QUEUE
+    __shared__ uint32_t s_found32[128];   // the layer-2 word's 64 output words (u32 halves)
+    __shared__ int32_t s_q[PQ_CAP], s_q2[PQ2_CAP];
+    __shared__ uint32_t s_qn, s_q2n;
 #endif
     if (o.ctrl ? o.ctrl->pull_warp[o.half] : o.pull_warp) return;   // late pull: k_pull_bfs_w takes it
     deg8_lut_init(s_lut);
@@ -131,6 +236,14 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
         // A layer-2 word with no unvisited vertex writes its 64 zero output words and is done;
         // otherwise a warp whose two words are full skips its round without loading them.
         uint64_t my_vis = ~0ull, my_unv = 0ull;   // threads < 64: layer-1 word sw*64+threadIdx.x
+#if SG_PULL_QUEUE
+        // (the previous layer-2 word's last reads of these ended at bfs_emit_words' barrier)
+        if (threadIdx.x < 128) s_found32[threadIdx.x] = 0u;
+        if (threadIdx.x == 0) {
+            s_qn = 0u;
+            s_q2n = 0u;
+        }
+#endif
         if (threadIdx.x < 64) {
             const int64_t w = sw * 64 + threadIdx.x;
             if (w < g.nw1) {
@@ -217,6 +330,116 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
         }
 #endif
 #endif
+#if SG_PULL_QUEUE
+        // quad rounds, SG_PULLQ_RB of them at once (all their candidate loads and probes in
+        // flight together: the rounds are independent now that misses are queued); misses
+        // queued with one shared atomic per warp and batch
+#pragma unroll 1
+        for (int rb = 0; rb < PULL_ROUNDS; rb += PQ_RB) {
+            uint32_t unv[PQ_RB], codes[PQ_RB], x[PQ_RB][4];
+            int4 c4[PQ_RB];
+            int64_t w[PQ_RB];
+            bool act[PQ_RB];
+#pragma unroll
+            for (int j = 0; j < PQ_RB; j++) {
+                const int r = rb + j;
+                const int64_t qd = sw * 1024 + r * PULL_THREADS + threadIdx.x;
+                w[j] = qd >> 4;
+                const int64_t v0 = w[j] * 64 + (qd & 15) * 4;
+                const int64_t rem = g.n - v0;
+                const uint32_t valid = qd >= nq ? 0u : rem >= 4 ? 0xfu : (rem > 0 ? (1u << rem) - 1u : 0u);
+                const bool skip = ((full >> (r * (PULL_THREADS / 16) + wid * 2)) & 3ull) == 3ull;
+                unv[j] = skip ? 0u : (uint32_t)(~vis_at(qd) >> ((qd & 15) * 4)) & valid;
+                act[j] = __any_sync(0xffffffffu, unv[j] != 0u);
+                c4[j] = make_int4(-1, -1, -1, -1);
+                codes[j] = 0u;
+                if (unv[j]) {
+                    c4[j] = __ldg(reinterpret_cast<const int4 *>(g.fnbr + v0));
+                    codes[j] = __ldg(reinterpret_cast<const uint32_t *>(g.deg8 + v0));
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < PQ_RB; j++) {
+                const int32_t c[4] = {c4[j].x, c4[j].y, c4[j].z, c4[j].w};
+#pragma unroll
+                for (int k = 0; k < 4; k++) x[j][k] = ((unv[j] >> k) & 1u) && c[k] >= 0 ? __ldg(in32 + (c[k] >> 5)) : 0u;
+            }
+            uint32_t found[PQ_RB], miss[PQ_RB];
+            int cnt = 0;
+#pragma unroll
+            for (int j = 0; j < PQ_RB; j++) {
+                const int32_t c[4] = {c4[j].x, c4[j].y, c4[j].z, c4[j].w};
+                found[j] = miss[j] = 0u;
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    if (!((unv[j] >> k) & 1u)) continue;
+                    if (c[k] >= 0) {
+                        arcs++;
+                        if ((x[j][k] >> (c[k] & 31)) & 1u) {
+                            found[j] |= 1u << k;
+                            continue;
+                        }
+                    }
+                    miss[j] |= 1u << k;
+                }
+                cnt += __popc(miss[j]);
+            }
+            const int incl = warp_inclusive_scan(cnt);
+            const int tot = __shfl_sync(0xffffffffu, incl, 31);
+            if (tot) {
+                uint32_t qb = 0;
+                if (lane == 31) qb = atomicAdd(&s_qn, (uint32_t)tot);
+                qb = __shfl_sync(0xffffffffu, qb, 31);
+                int pos = (int)qb + incl - cnt;
+#pragma unroll
+                for (int j = 0; j < PQ_RB; j++) {
+                    const int32_t v0 = (int32_t)(w[j] * 64 + (lane & 15) * 4);
+#pragma unroll
+                    for (int k = 0; k < 4; k++)
+                        if ((miss[j] >> k) & 1u) s_q[pos++] = v0 + k;
+                }
+                if (SG_PULL_COUNT_SCANS) scans += (uint32_t)cnt;
+            }
+#pragma unroll
+            for (int j = 0; j < PQ_RB; j++) {
+                if (!act[j]) continue;
+                const int sh = (lane & 15) * 4;
+                const uint64_t mine = (uint64_t)found[j] << sh;
+                const uint32_t nlo = __reduce_or_sync(half, (uint32_t)mine), nhi = __reduce_or_sync(half, (uint32_t)(mine >> 32));
+                if (found[j]) {
+                    nf += __popc(found[j]);
+                    mf += quad_mf(s_lut, codes[j], found[j]);
+                }
+                if (nlo | nhi) {   // candidate hits: level stores strided over the half-warp (64-B runs)
+                    const uint64_t t = ((uint64_t)nhi << 32 | nlo) >> (lane & 15);
+                    uint32_t *lw = lvl + w[j] * 64 + (lane & 15);
+#pragma unroll
+                    for (int i = 0; i < 4; i++)
+                        if ((t >> (16 * i)) & 1u) lw[16 * i] = nx;
+                    if ((lane & 15) == 0) {
+                        const int wi = (int)(w[j] & 63);
+                        s_found32[2 * wi] = nlo;
+                        s_found32[2 * wi + 1] = nhi;
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        if (s_qn) pullq_drain(g, in32, s_q, s_qn, s_q2, &s_q2n, s_found32, lvl, nx, s_lut, nf, mf, arcs);
+        // output: the 64 words, visited / vis_old, the warp masks of changed words
+        if (threadIdx.x < 64) {
+            const int64_t w = sw * 64 + threadIdx.x;
+            const uint64_t nb = (uint64_t)s_found32[2 * threadIdx.x] | ((uint64_t)s_found32[2 * threadIdx.x + 1] << 32);
+            if (w < g.nw1) {
+                xstore<P>(o.x, o.out_bits + w, nb);
+                if (nb) {
+                    visited[w] = my_vis | nb;
+                    o.vis_old[w] = my_vis | nb;
+                }
+            }
+            wm = (uint64_t)__ballot_sync(0xffffffffu, nb != 0ull) << (32 * wid);
+        }
+#else
 #pragma unroll 1
         for (int r = 0; r < PULL_ROUNDS; r++) {
             const int64_t qd = sw * 1024 + r * PULL_THREADS + threadIdx.x;
@@ -292,6 +515,7 @@ k_pull_bfs(GraphView g, const uint64_t *__restrict__ in_bits, uint64_t *__restri
             const uint32_t act = __ballot_sync(0xffffffffu, nb != 0ull && (lane & 15) == 0);
             wm |= (uint64_t)((act & 1u) | ((act >> 15) & 2u)) << (r * (PULL_THREADS / 16) + wid * 2);
         }
+#endif
         if (lane == 0) s_wm[wid] = wm;
         __syncthreads();
         if (threadIdx.x == 0) {

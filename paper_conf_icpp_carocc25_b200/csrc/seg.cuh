@@ -35,7 +35,16 @@ constexpr size_t SEG_SMEM = (size_t)SEG_WORDS * sizeof(uint64_t);
 #ifndef SG_SEG_LONG
 #define SG_SEG_LONG 192
 #endif
+#ifndef SG_SEG_CHECK
+#define SG_SEG_CHECK 0   // 1: test the slice bit before the shared-memory atomic (0: atomic on every arc;
+                         // measured faster: the level-2 hub pushes mark mostly fresh bits, so the test
+                         // was an extra LDS per arc - 283 -> 264 us on a 133 M-arc level)
+#endif
 constexpr int SEG_UNROLL = SG_SEG_UNROLL;
+// mark a destination in the shared-memory slice (32-bit ATOMS.OR is native; 64-bit is a CAS loop)
+__device__ __forceinline__ void seg_mark(uint32_t *s_vis32, int i, uint32_t m) {
+    if (!SG_SEG_CHECK || !(s_vis32[i] & m)) atomicOr(s_vis32 + i, m);
+}
 constexpr uint32_t SEG_LONG = SG_SEG_LONG;   // parts at least this long are streamed with int4 loads
 
 __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs f) {
@@ -142,12 +151,12 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
                 for (int64_t i = lo; i < la; i++) {
                     const int32_t vv = __ldg(p.g.col + i) - vbase;
                     const uint32_t m = 1u << (vv & 31);
-                    if (!(s_vis32[vv >> 5] & m)) atomicOr(s_vis32 + (vv >> 5), m);
+                    seg_mark(s_vis32, vv >> 5, m);
                 }
                 for (int64_t i = lb; i < e; i++) {
                     const int32_t vv = __ldg(p.g.col + i) - vbase;
                     const uint32_t m = 1u << (vv & 31);
-                    if (!(s_vis32[vv >> 5] & m)) atomicOr(s_vis32 + (vv >> 5), m);
+                    seg_mark(s_vis32, vv >> 5, m);
                 }
             }
             if (longm) {
@@ -184,7 +193,7 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
                         for (int k = 0; k < 4; k++) {
                             if (vv[k] < 0) continue;
                             const uint32_t m = 1u << (vv[k] & 31);
-                            if (!(s_vis32[vv[k] >> 5] & m)) atomicOr(s_vis32 + (vv[k] >> 5), m);
+                            seg_mark(s_vis32, vv[k] >> 5, m);
                         }
                     }
                     if (nsrc < 0) break;
@@ -222,7 +231,7 @@ __global__ void __launch_bounds__(SEG_THREADS, 1) k_push_seg(PushParams p, FnBfs
                 for (int j = 0; j < SEG_UNROLL; j++) {
                     if (v[j] < 0) continue;
                     const uint32_t m = 1u << (v[j] & 31);
-                    if (!(s_vis32[v[j] >> 5] & m)) atomicOr(s_vis32 + (v[j] >> 5), m);
+                    seg_mark(s_vis32, v[j] >> 5, m);
                 }
             }
         }

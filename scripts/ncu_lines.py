@@ -5,7 +5,8 @@ import csv
 import subprocess
 import sys
 
-out = subprocess.run(["ncu", "-i", sys.argv[1], "--page", "source", "--csv", "--print-source", "cuda,sass"],
+EXTRA = ["--launch-skip", sys.argv[3], "--launch-count", "1"] if len(sys.argv) > 3 else []
+out = subprocess.run(["ncu", "-i", sys.argv[1], "--page", "source", "--csv", "--print-source", "cuda,sass", *EXTRA],
                      capture_output=True, text=True).stdout
 top = int(sys.argv[2]) if len(sys.argv) > 2 else 30
 rows = list(csv.reader(out.splitlines()))

@@ -590,22 +590,30 @@ def test_bfs_pull_word_mode_threshold(sg, monkeypatch, word_max, host_loop):
                 assert np.array_equal(sg.as_u32(lv), ref), (word_max, frac, d)
 
 
-def test_bfs_pull_128_thread_variant(sg):
-    """The SG_PULL_THREADS=128 layout (a measured round-1 variant) built as its own library and
-    run in a subprocess: pull-only and auto BFS equal the oracle."""
+@pytest.mark.parametrize("name,defines", [
+    ("pull128", ("SG_PULL_THREADS=128",)),
+    ("pullnoq", ("SG_PULL_QUEUE=0",)),
+    ("pullq2", ("SG_PULLQ_SHORT=2", "SG_PULLQ2_CAP=4")),
+])
+def test_bfs_pull_build_variants(sg, name, defines):
+    """Compile-time layouts of the CTA pull, each built as its own library and run in a
+    subprocess: 128-thread CTAs (a measured round-1 variant), the per-thread list scan without
+    the miss queue, and the queue with a 2-arc stage A and a 4-row stage-B queue (so stage B and
+    its overflow path, the thread scanning the rest itself, both run).  Pull-only and auto BFS
+    equal the oracle."""
     import os
     import subprocess
     import sys
     from paper_conf_icpp_carocc25_b200 import _build
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    lib = _build.build(defines=("SG_PULL_THREADS=128",), lib=os.path.join(root, "build", "variants", "pull128",
-                                                                          "libsygraph.so"))
+    lib = _build.build(defines=defines, lib=os.path.join(root, "build", "variants", name, "libsygraph.so"))
     code = ("import numpy as np, gen, oracle, paper_conf_icpp_carocc25_b200 as sg\n"
-            "g = gen.rmat(14, 16, permute=True); G = sg.graph_load_csr(g.row_ptr, g.col_idx)\n"
-            "for s in gen.sources(g, 3):\n"
-            "    for d in (sg.SG_DIR_PULL, sg.SG_DIR_AUTO):\n"
-            "        lv, _ = sg.run_bfs(G, int(s), direction=d)\n"
-            "        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s)))\n"
+            "for g in (gen.rmat(14, 16, permute=True), gen.rmat(16, 4, permute=True)):\n"
+            "    G = sg.graph_load_csr(g.row_ptr, g.col_idx)\n"
+            "    for s in gen.sources(g, 3):\n"
+            "        for d in (sg.SG_DIR_PULL, sg.SG_DIR_AUTO):\n"
+            "            lv, _ = sg.run_bfs(G, int(s), direction=d)\n"
+            "            assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, int(s)))\n"
             "print('ok')\n")
     env = dict(os.environ, SYGRAPH_LIB=lib, PYTHONPATH=root)
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, cwd=root)
