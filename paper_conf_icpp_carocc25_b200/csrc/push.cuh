@@ -21,6 +21,7 @@
 //     flight before any decision, then the functor's act (atomics on 64-bit words, summary
 //     bit only on the word's 0 -> non-zero transition).
 #pragma once
+#include <type_traits>
 #include "common.cuh"
 #include "functors.cuh"
 
@@ -56,8 +57,18 @@ struct PushParams {
     int32_t chunk = HEAVY_CHUNK;   // arcs per queued CTA/grid-tier item (the sparse kernel: a warp round)
 };
 
+constexpr int HUBQ = 64;   // hubs a warp buffers before queueing their segment-tier chunks
+// segmented hub tier (BFS): hubs found by a warp, queued in bulk (one seg_count atomic per flush
+// instead of one per hub: 13-18 K hubs on one counter serialised a level-2 k_push_words at 36 us,
+// profiles/r02i)
+struct PushHubQ {
+    int64_t hq_s[HUBQ], hq_e[HUBQ];
+    int32_t hq_u[HUBQ];
+    int32_t nhq;
+};
+struct PushNoHubQ {};
 template <class F>
-struct PushWarpSmem {
+struct PushWarpSmem : std::conditional_t<F::kSeg, PushHubQ, PushNoHubQ> {
     int64_t start[64];
     uint32_t pre[64];
     typename F::Ctx ctx[64];
@@ -147,6 +158,49 @@ __device__ __forceinline__ void enqueue_seg(const PushParams &p, int32_t h, int6
     }
 }
 
+// queue the warp's buffered hubs as segment-tier chunks: one atomic for all of them, each
+// lane writes the chunks of its entries (whole warp; sm.nhq warp-uniform)
+template <class F>
+__device__ __forceinline__ void flush_hubs(const PushParams &p, PushWarpSmem<F> &sm) {
+    const int lane = lane_id();
+    const int n = sm.nhq;
+    if (n == 0) return;
+    int64_t s[2] = {0, 0}, e[2] = {0, 0};
+    int32_t h[2] = {0, 0};
+    uint32_t nch[2] = {0u, 0u};
+#pragma unroll
+    for (int k = 0; k < 2; k++) {
+        const int i = lane + 32 * k;
+        if (i < n) {
+            s[k] = sm.hq_s[i];
+            e[k] = sm.hq_e[i];
+            h[k] = __ldg(p.g.hub_idx + sm.hq_u[i]);
+            nch[k] = (uint32_t)((e[k] - s[k] + HEAVY_CHUNK - 1) / HEAVY_CHUNK);
+        }
+    }
+    const uint32_t mine = nch[0] + nch[1];
+    const uint32_t incl = warp_inclusive_scan(mine);
+    const uint32_t tot = __shfl_sync(0xffffffffu, incl, 31);
+    unsigned long long base = 0;
+    if (lane == 31) base = atomicAdd(&p.st->seg_count, (unsigned long long)tot);
+    base = __shfl_sync(0xffffffffu, base, 31) + (incl - mine);
+#pragma unroll
+    for (int k = 0; k < 2; k++) {
+        for (uint32_t j = 0; j < nch[k]; j++, base++) {
+            if (base >= p.seg_cap) break;   // cannot happen: capacity bound in DESIGN.md
+            SegItem it;
+            it.begin = s[k] + (int64_t)j * HEAVY_CHUNK;
+            it.row = s[k];
+            it.len = (int32_t)min((int64_t)HEAVY_CHUNK, e[k] - it.begin);
+            it.h = h[k];
+            p.seg[base] = it;
+        }
+    }
+    __syncwarp();
+    if (lane == 0) sm.nhq = 0;
+    __syncwarp();
+}
+
 // ---- one word on one warp ----------------------------------------------------------------
 template <class F>
 __device__ __forceinline__ unsigned long long push_word(const PushParams &p, const F &f, int64_t w,
@@ -158,14 +212,32 @@ __device__ __forceinline__ unsigned long long push_word(const PushParams &p, con
     const int32_t ua = (int32_t)(w * 64 + lane), ub = ua + 32;
     const int64_t d_total = (ea - sa) + (eb - sb);
     if constexpr (F::kSeg) {
-        if (seg_on) {   // hubs go to the destination-segmented tier (visited slice in shared memory)
-            if (ea - sa >= SEG_MIN) {
-                enqueue_seg(p, __ldg(p.g.hub_idx + ua), sa, ea);
-                sa = ea;
-            }
-            if (eb - sb >= SEG_MIN) {
-                enqueue_seg(p, __ldg(p.g.hub_idx + ub), sb, eb);
-                sb = eb;
+        if (seg_on) {   // hubs go to the destination-segmented tier (visited slice in shared memory),
+                        // buffered per warp and queued in bulk (flush_hubs)
+            const bool qa = ea - sa >= SEG_MIN, qb = eb - sb >= SEG_MIN;
+            const uint32_t ba = __ballot_sync(0xffffffffu, qa), bb = __ballot_sync(0xffffffffu, qb);
+            const int nq = __popc(ba) + __popc(bb);
+            if (nq) {
+                if (sm.nhq + nq > HUBQ) flush_hubs(p, sm);
+                const uint32_t lt = (1u << lane) - 1u;
+                const int n0 = sm.nhq;
+                if (qa) {
+                    const int i = n0 + __popc(ba & lt);
+                    sm.hq_s[i] = sa;
+                    sm.hq_e[i] = ea;
+                    sm.hq_u[i] = ua;
+                    sa = ea;
+                }
+                if (qb) {
+                    const int i = n0 + __popc(ba) + __popc(bb & lt);
+                    sm.hq_s[i] = sb;
+                    sm.hq_e[i] = eb;
+                    sm.hq_u[i] = ub;
+                    sb = eb;
+                }
+                __syncwarp();
+                if (lane == 0) sm.nhq = n0 + nq;
+                __syncwarp();
             }
         }
     }
@@ -349,6 +421,10 @@ __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) 
     const bool sparse = SG_SPARSE_WORDS && p.sparse_ok && p.st->nf <= 2ull * count && p.st->mf <= 16ull * p.st->nf;
     // a warp's first grab is static (warp id x grab), later ones dynamic (after all static
     // grabs): a small frontier costs no atomic storm of idle warps on one counter
+    if constexpr (F::kSeg) {
+        if (lane_id() == 0) s_warp[wid].nhq = 0;
+        __syncwarp();
+    }
     const uint32_t gwarp = (blockIdx.x * PUSH_THREADS + threadIdx.x) >> 5;
     const uint32_t nwarps = gridDim.x * PUSH_WARPS;
     const uint32_t grab = sparse ? 32u : batch;
@@ -367,6 +443,7 @@ __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) 
         if (lane_id() == 0) nb = statics + atomicAdd(&p.st->batch, (unsigned long long)grab);
         b0l = __shfl_sync(0xffffffffu, nb, 0);
     }
+    if constexpr (F::kSeg) flush_hubs(p, s_warp[wid]);
     arcs = warp_sum(arcs);
     if (lane_id() == 0) s_arcs[wid] = arcs;
     __syncthreads();
