@@ -1264,13 +1264,18 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     // prologue: level = INF, frontiers cleared, visited = isolated, seed src, compact + decide
     TRY(capture_begin(cs, root, {}));
     // (the output frontier F[1] is written whole by the first output kernel: only F[0] is zeroed)
-    CK(cudaMemsetAsync(F[0]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
-    CK(cudaMemsetAsync(F[0]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
-    CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), cs));
-    CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
-    CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
-    launch_bfs_prologue(ws->ctrl, G.n, G.deg8, F[0]->bits, F[0]->summ, F[0]->offsets, F[0]->st, ws->visited,
-                        ws->vis_old, g->ar ? g->ar->x : Xchg{}, cs);
+    if (!g->ar) {   // single GPU: one kernel (memsets / copies folded in)
+        launch_bfs_prologue1(ws->ctrl, G.n, G.nw1, G.nw2, G.deg8, g->isolated, F[0]->bits, F[0]->summ,
+                             F[0]->offsets, F[0]->st, F[1]->st, ws->visited, ws->vis_old, cs);
+    } else {
+        CK(cudaMemsetAsync(F[0]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
+        CK(cudaMemsetAsync(F[0]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
+        CK(cudaMemsetAsync(ws->st, 0, 2 * sizeof(DevStats), cs));
+        CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
+        CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
+        launch_bfs_prologue(ws->ctrl, G.n, G.deg8, F[0]->bits, F[0]->summ, F[0]->offsets, F[0]->st, ws->visited,
+                            ws->vis_old, g->ar->x, cs);
+    }
     // the handles go to the device with every run's control block (run_bfs_graph)
     ws->hnd[0] = (unsigned long long)h_loop;
     for (int i = 0; i < 2; i++) {

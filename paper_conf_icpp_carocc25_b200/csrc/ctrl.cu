@@ -89,6 +89,64 @@ __global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint6
         bfs_decide(c, st, 0ull, nullptr, 0, 1);
     }
 }
+// Single-GPU graph prologue with the frontier / bitmap initialisation folded in (one kernel
+// instead of 5 memset / copy nodes + the prologue, ~1 us each in the graph): per layer-1 word w,
+// visited[w] = vis_old[w] = isolated[w] (| src's bit), the input frontier's word = src's bit or 0;
+// layer 2 likewise; both control blocks written whole by thread 0; then the level pass and the
+// first decision as k_bfs_prologue.  Every store lands in a distinct word, so no ordering is needed
+// inside the kernel (the supersteps read them after the kernel boundary).
+__global__ void k_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2, const uint8_t *deg8,
+                                const uint64_t *__restrict__ isolated, uint64_t *bits, uint64_t *summ,
+                                uint32_t *offsets, DevStats *st, DevStats *st_out, uint64_t *visited,
+                                uint64_t *vis_old) {
+    uint32_t *level = c->level;
+    const int32_t src = c->src;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t ws = src >> 6;
+    const uint64_t sb = 1ull << (src & 63);
+    for (int64_t w = t; w < nw1; w += stride) {
+        const uint64_t v = isolated[w] | (w == ws ? sb : 0ull);
+        visited[w] = v;
+        vis_old[w] = v;
+        bits[w] = w == ws ? sb : 0ull;
+    }
+    for (int64_t w = t; w < nw2; w += stride) summ[w] = w == (src >> 12) ? 1ull << ((src >> 6) & 63) : 0ull;
+    if (((uintptr_t)level & 15) == 0) {
+        uint4 *l4 = reinterpret_cast<uint4 *>(level);
+        for (int64_t i = t; i < n / 4; i += stride) {
+            uint4 q = make_uint4(INF32, INF32, INF32, INF32);
+            if (i == (src >> 2)) (&q.x)[src & 3] = 0u;
+            l4[i] = q;
+        }
+        for (int64_t i = (n / 4) * 4 + t; i < n; i += stride) level[i] = i == src ? 0u : INF32;
+    } else {
+        for (int64_t i = t; i < n; i += stride) level[i] = i == src ? 0u : INF32;
+    }
+    if (t == 0) {
+        offsets[0] = (uint32_t)ws;
+        DevStats d{};
+        d.count = 1ull;
+        d.nf = 1ull;
+        d.mf = deg8_decode(deg8[src]);
+        *st = d;
+        *st_out = DevStats{};
+        c->dirty[0] = 0u;
+        c->dirty[1] = 1u;
+        c->saved_count[1] = ~0ull;
+        bfs_decide(c, st, 0ull, nullptr, 0, 1);
+    }
+}
+void launch_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2, const uint8_t *deg8,
+                          const uint64_t *isolated, uint64_t *bits, uint64_t *summ, uint32_t *offsets, DevStats *st,
+                          DevStats *st_out, uint64_t *visited, uint64_t *vis_old, cudaStream_t s) {
+    int64_t blocks = (n / 4 + 255) / 256;
+    if (blocks > num_sms() * 8) blocks = num_sms() * 8;
+    if (blocks < 1) blocks = 1;
+    note_launch();
+    k_bfs_prologue1<<<(int)blocks, 256, 0, s>>>(c, n, nw1, nw2, deg8, isolated, bits, summ, offsets, st, st_out,
+                                                visited, vis_old);
+}
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                          uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old, const Xchg &x,
                          cudaStream_t s) {

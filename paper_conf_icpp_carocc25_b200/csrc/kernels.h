@@ -198,6 +198,10 @@ int ablation_bfs_words(const GraphView &g, int32_t src, uint32_t *level, int wor
                        float *ms);
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 // level init + seed + the seed frontier's word list / statistics + first decision, one kernel
+// single-GPU: the same with the frontier, visited / vis_old and control-block initialisation folded in
+void launch_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2, const uint8_t *deg8,
+                          const uint64_t *isolated, uint64_t *bits, uint64_t *summ, uint32_t *offsets, DevStats *st,
+                          DevStats *st_out, uint64_t *visited, uint64_t *vis_old, cudaStream_t s);
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                          uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old, const Xchg &x,
                          cudaStream_t s);
