@@ -38,7 +38,8 @@ enum : uint32_t { SK_STOP = 0, SK_PUSH = 1, SK_PULL = 2, SK_SWEEP = 3, SK_SPARSE
 // switched off (the fused sparse loop may end on either parity; its half is then skipped and the
 // WHILE loop comes back to the right one).  Returns the decision (SK_*).  One thread.
 __device__ __forceinline__ uint32_t bfs_decide(BfsCtrl *c, const DevStats *st, unsigned long long prev_arcs,
-                                               DevStats *zero_prev, int next_in, int first, bool defer_sparse = false) {
+                                               DevStats *zero_prev, int next_in, int first, bool defer_sparse = false,
+                                               bool dead_end = false) {
     // control blocks were filled by atomics of other CTAs / kernels: volatile (L2) reads
     const volatile DevStats *vst = st;
     if (!first) {
@@ -47,13 +48,19 @@ __device__ __forceinline__ uint32_t bfs_decide(BfsCtrl *c, const DevStats *st, u
     }
     const unsigned long long count = vst->count;
     bool go = count > 0;
+    if (go) {
+        if (!first) c->reached += vst->nf;
+        // every vertex is visited (the reached ones + the never-reachable ones): expanding this
+        // frontier cannot find a new vertex, so the BFS ends here instead of one empty superstep later
+        if ((long long)c->reached + c->n_iso - c->src_iso >= c->n) go = false;
+        if (dead_end) go = false;   // lookahead: no arc of this frontier leads to an unvisited vertex
+    }
     if (go && c->iters >= (unsigned long long)c->max_iters) {
         c->overflow = 1;
         go = false;
     }
     if (go) {
         const long long nf = (long long)vst->nf, mf = (long long)vst->mf;
-        if (!first) c->reached += (unsigned long long)nf;
         c->mu -= mf;
         if (c->auto_dir) {
             if (!c->pull && nf > c->nf_prev && (double)mf > (double)c->mu / c->alpha) c->pull = 1;
@@ -185,6 +192,61 @@ __device__ __forceinline__ void bfs_emit_words(const BfsOut &o, int64_t w2_hi, i
     __syncthreads();
 }
 
+// Dead-end lookahead (single GPU, the last CTA of a BFS output kernel, whole CTA): when the
+// output frontier is tiny (<= 64 listed words, m_f <= 64) test its arcs against the final visited
+// bitmap; if none leads to an unvisited vertex, the next superstep would produce an empty frontier,
+// so the BFS ends now (st->pad2 = 1; bfs_decide) instead of one ~20 us superstep later - the last
+// superstep of every config-4 BFS (2-22 leaves whose neighbours are all visited).  Five dependent
+// loads (list, word, row bounds, arcs, visited) in one CTA.  Returns the verdict (CTA-uniform).
+__device__ __forceinline__ bool bfs_lookahead(const BfsOut &o) {
+    constexpr int LV = 64, LA = 256;
+    __shared__ int64_t s_start[LV];
+    __shared__ uint32_t s_pre[LV + 1];
+    __shared__ int32_t s_v[LV];
+    __shared__ uint32_t s_nv;
+    __shared__ int s_dead;
+    const volatile DevStats *vst = o.st;
+    const unsigned long long count = vst->count, mf = vst->mf;
+    if (!o.rp || count == 0 || count > (unsigned long long)LV || mf > (unsigned long long)LV) return false;
+    if (threadIdx.x == 0) {
+        s_nv = 0u;
+        s_dead = 1;
+    }
+    __syncthreads();
+    if (threadIdx.x < count) {
+        const uint32_t w = o.out_offsets[threadIdx.x];
+        for (uint64_t b = o.out_bits[w]; b; b &= b - 1) {
+            const uint32_t i = atomicAdd(&s_nv, 1u);
+            if (i < (uint32_t)LV) s_v[i] = (int32_t)(w * 64u + (uint32_t)(__ffsll((long long)b) - 1));
+        }
+    }
+    __syncthreads();
+    const uint32_t nv = s_nv;
+    if (nv > (uint32_t)LV) return false;   // (uniform) cannot happen: every frontier vertex has an arc
+    if (threadIdx.x < nv) {
+        const int32_t v = s_v[threadIdx.x];
+        const int64_t a = o.rp[v];
+        s_start[threadIdx.x] = a;
+        s_pre[threadIdx.x + 1] = (uint32_t)min(o.rp[v + 1] - a, (int64_t)LA + 1);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        s_pre[0] = 0u;
+        for (uint32_t i = 0; i < nv; i++) s_pre[i + 1] += s_pre[i];
+    }
+    __syncthreads();
+    const uint32_t total = s_pre[nv];
+    if (total > (uint32_t)LA) return false;   // (uniform) degree codes under-estimated a row
+    for (uint32_t t = threadIdx.x; t < total; t += blockDim.x) {
+        uint32_t k = 0;
+        while (s_pre[k + 1] <= t) k++;
+        const int32_t u = o.col[s_start[k] + (t - s_pre[k])];
+        if (!((o.visited[u >> 6] >> (u & 63)) & 1ull)) s_dead = 0;
+    }
+    __syncthreads();
+    return s_dead != 0;
+}
+
 // End of the output kernel: block sums of n_f / m_f (and `arcs` into the input's control block),
 // then the last CTA to finish takes the direction decision (graph mode).  Partitioned: the last
 // CTA first runs the superstep barrier (xchg.cuh) and replaces st's n_f / m_f by the global sums;
@@ -223,13 +285,19 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
         }
         if (c && in_st) atomicAdd(&in_st->arcs, c);
         s_last = false;
-        if (o.ctrl || o.vctrl || part) {
+        if (o.ctrl || o.vctrl || part || o.rp) {
             if (part) __threadfence_system();   // this CTA's peer stores before the barrier's epoch
             else __threadfence();
             s_last = atomicAdd(o.done, 1u) == gridDim.x - 1;
         }
     }
     __syncthreads();
+    bool dead = false;
+    if (s_last && !part && o.rp) {   // (uniform across the last CTA)
+        __threadfence();
+        dead = bfs_lookahead(o);
+        if (dead && threadIdx.x == 0) o.st->pad2 = 1ull;   // the host loop reads the verdict here
+    }
     if (s_last && threadIdx.x == 0) {
         if (part) __threadfence_system();
         else __threadfence();
@@ -252,7 +320,7 @@ __device__ __forceinline__ void bfs_finish(const BfsOut &o, unsigned long long n
             vst->pad = tot.arcs;   // host loops read the superstep's global arcs here
             if (o.ctrl) bfs_decide(o.ctrl, o.st, prev_arcs, nullptr, o.half ^ 1, 0);
         } else if (o.ctrl) {
-            bfs_decide(o.ctrl, o.st, prev_arcs, o.prev, o.half ^ 1, 0);
+            bfs_decide(o.ctrl, o.st, prev_arcs, o.prev, o.half ^ 1, 0, false, dead);
         } else if (o.vctrl) {
             val_decide(o.vctrl, o.st, prev_arcs, o.prev, o.half ^ 1, 0);
         }

@@ -1309,6 +1309,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, nullptr, 0u, &ws->ctrl->next,
                   &ws->ctrl->level, out->st, ws->ctrl, in->st, ws->bfs_done};
         if (g->ar) bo.x = g->ar->x;   // partitioned: owned slice replicated to the peers + barrier
+        else bo.rp = G.rp, bo.col = G.col, bo.visited = ws->visited;   // dead-end lookahead
         bo.half = half;
         TRY(capture_begin(cs, b_push, {}));
         launch_push_bfs(L, a, cs);
@@ -1485,13 +1486,21 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
     int64_t reached = 1;
     uint32_t d = 0;
     int in_idx = 0;
+    int64_t src_iso = 0;   // the source is one of the never-reachable vertices (bfs_decide's rule)
+    {
+        uint64_t w = 0;
+        CK(cudaMemcpy(&w, g->isolated + (src >> 6), sizeof w, cudaMemcpyDeviceToHost));
+        src_iso = (int64_t)((w >> (src & 63)) & 1ull);
+    }
     for (;;) {
         const DevStats &hs = ws->h_st[in_idx];
         const int64_t count = (int64_t)hs.count;
         if (count == 0) break;
-        if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
         const int64_t nf = (int64_t)hs.nf, mf = (int64_t)hs.mf;
         if (iters > 0) reached += nf;
+        if (reached + g->n_iso - src_iso >= G.n) break;   // every vertex visited (bfs_decide)
+        if (iters > 0 && hs.pad2) break;                   // dead-end lookahead of the output kernel
+        if (iters >= max_iters) return fail(SG_ERR_STATE, "iteration cap %lld reached", (long long)max_iters);
         mu -= mf;
         if (auto_dir) {   // Beamer: push -> pull on a growing frontier with m_f > m_u / alpha,
                           // pull -> push on a shrinking frontier with n_f < n / beta
@@ -1503,6 +1512,12 @@ SG_API int run_bfs(const sg_graph *gc, int32_t src, uint32_t *level, const sg_op
         const bool sweep = !pull && scsr_on && (t.scsr == 2 || (unsigned long long)mf >= sweep_threshold(G.nnz));
         CK(cudaMemsetAsync(out->st, 0, sizeof(DevStats), s));
         BfsOut bo{ws->vis_old, out->bits, out->summ, out->offsets, level, d + 1, nullptr, nullptr, out->st};
+        if (!o.one_layer) {   // dead-end lookahead (bfsstep.cuh): needs the output kernel's done counter
+            bo.rp = G.rp;
+            bo.col = G.col;
+            bo.visited = ws->visited;
+            bo.done = ws->bfs_done;
+        }
         {   // late pulls: warp-owned layer-2 words (same rule as bfs_decide)
             const long long frac = (long long)env_or("SG_PULL_WARP_FRAC", 8), live = G.n - g->n_iso;
             bo.pull_warp = frac > 0 && (live - reached) * frac < live ? 1 : 0;

@@ -131,6 +131,7 @@ struct BfsCtrl {
                              // both pull kernels of the current superstep read the current one
     uint32_t pull_warp_frac; // ... when unvisited non-isolated vertices < (n - n_iso) / pull_warp_frac
     long long n_iso;         // isolated vertices (visited from the start, never reached)
+    long long src_iso;       // 1 iff the source itself is one of them (counted in reached too)
     uint32_t sp_kind;        // the fused sparse loop's last decision (read by all its CTAs)
     uint32_t sp_epoch;       // bumped by CTA 0 once sp_kind is written (the loop's broadcast)
     uint32_t hmask;          // current values of the IF handles (bit 2k+b: kind k of buffer b; bit 8: loop);

@@ -74,6 +74,7 @@ __global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint6
         for (int64_t i = t; i < n; i += stride) level[i] = i == src ? 0u : INF32;
     }
     if (t == 0) {
+        c->src_iso = (long long)((visited[src >> 6] >> (src & 63)) & 1ull);   // visited = isolated (copied before)
         bits[src >> 6] = 1ull << (src & 63);
         summ[src >> 12] = 1ull << ((src >> 6) & 63);
         visited[src >> 6] |= 1ull << (src & 63);
@@ -125,6 +126,7 @@ __global__ void k_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2,
     }
     if (t == 0) {
         offsets[0] = (uint32_t)ws;
+        c->src_iso = (long long)((isolated[ws] >> (src & 63)) & 1ull);
         DevStats d{};
         d.count = 1ull;
         d.nf = 1ull;

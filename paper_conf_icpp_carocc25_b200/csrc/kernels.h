@@ -107,6 +107,10 @@ struct BfsOut {
     int32_t word_max = 16;            // CTA pull: word mode when no layer-1 word has more unvisited vertices
                                       // (SG_PULL_WORD_MAX at launch / capture; 0 = off)
     ValCtrl *vctrl = nullptr;         // graph-driven SSSP / CC: the last CTA runs val_decide
+    // single-GPU BFS: the graph for the dead-end lookahead of a tiny output frontier (bfsstep.cuh)
+    const int64_t *rp = nullptr;
+    const int32_t *col = nullptr;
+    const uint64_t *visited = nullptr;
 };
 // device-driven SSSP / CC: the first decision (after the prologue compacted the input), one thread
 void launch_val_first(ValCtrl *c, const DevStats *st, cudaStream_t s);

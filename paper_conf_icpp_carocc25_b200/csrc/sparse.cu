@@ -268,6 +268,21 @@ __global__ void __launch_bounds__(SP_THREADS) k_bfs_sparse_loop(SpLoop L) {
             __threadfence();
         }
         mark(5);
+        // dead-end lookahead of the output frontier (bfsstep.cuh; single GPU), whole CTA 0
+        bool dead = false;
+        if (blockIdx.x == 0) {
+            __syncthreads();   // (the lead has seen every CTA arrive)
+            if (x.nranks <= 1) {
+                BfsOut lo{};
+                lo.out_bits = Fo.bits;
+                lo.out_offsets = Fo.offsets;
+                lo.st = Fo.st;
+                lo.rp = L.p.g.rp;
+                lo.col = L.p.g.col;
+                lo.visited = L.f.visited;
+                dead = bfs_lookahead(lo);
+            }
+        }
         // 4. decision (CTA 0): the input is retired as all-zero (cleared word by word above)
         if (lead) {
             DevStats *prev = Fi.st;
@@ -287,7 +302,7 @@ __global__ void __launch_bounds__(SP_THREADS) k_bfs_sparse_loop(SpLoop L) {
                 vo->pad = tot.arcs;
                 kind = bfs_decide(c, Fo.st, tot.arcs, nullptr, out, 0, true);
             } else {
-                kind = bfs_decide(c, Fo.st, prev_arcs, prev, out, 0, true);
+                kind = bfs_decide(c, Fo.st, prev_arcs, prev, out, 0, true, dead);
             }
             c->sp_kind = kind;
             __threadfence();

@@ -95,8 +95,31 @@ def test_bfs_config1(sg, direction, host_loop):
     g = gen.rmat(10, 16)
     G = load(sg, g)
     lv, st = sg.run_bfs(G, 0, direction=_dir(sg, direction), host_loop=host_loop)
-    assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, 0))
-    assert st.iterations == int(oracle.bfs(g, 0)[oracle.bfs(g, 0) != INF].max()) + 1
+    ref = oracle.bfs(g, 0)
+    assert np.array_equal(sg.as_u32(lv), ref)
+    # one superstep per level; the last level is expanded (finding nothing) unless the device
+    # proves it a dead end first (every vertex visited, or a tiny last frontier whose arcs all
+    # lead to visited vertices: bfs_decide / bfs_lookahead)
+    L = int(ref[ref != INF].max())
+    assert st.iterations in (L, L + 1)
+
+
+@pytest.mark.parametrize("host_loop", [False, True])
+def test_bfs_stops_when_everything_is_visited(sg, host_loop):
+    """The BFS runs one superstep per level and skips the empty one after the last level when it
+    can prove the last frontier a dead end: every vertex visited (path, grid, a 5,000-leaf star),
+    or a tiny last frontier (<= 64 words and arcs) whose arcs all lead to visited vertices (a
+    path with a second component).  A wide last level next to an unreached component (the star
+    plus one extra edge) is expanded.  Levels equal the oracle in every case."""
+    leaves = list(range(1, 5001))
+    cases = [(gen.path(300), 299), (gen.grid(20, 30), 48), (gen.from_edges(10, [0, 1, 5], [1, 2, 6]), 2),
+             (gen.from_edges(5001, [0] * 5000, leaves), 1),
+             (gen.from_edges(5003, [0] * 5000 + [5001], leaves + [5002]), 2)]
+    for g, want in cases:
+        G = load(sg, g)
+        lv, st = sg.run_bfs(G, 0, host_loop=host_loop)
+        assert np.array_equal(sg.as_u32(lv), oracle.bfs(g, 0))
+        assert st.iterations == want, (g.n, st.iterations, want)
 
 
 def test_bfs_graph_and_host_loop_agree_on_stats(sg):

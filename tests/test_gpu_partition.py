@@ -50,9 +50,13 @@ def _worker(rank, world, q_id, q_out, case):
                     lv, st = sg.run_bfs(G, int(s), direction=d)
                     _check(f"bfs root {s} dir {d}", np.array_equal(sg.as_u32(lv), ref), errs)
                     _, st1 = sg.run_bfs(Gs, int(s), direction=d)
+                    # same supersteps as the single-GPU run, except that the single-GPU run may
+                    # skip the empty last one (dead-end lookahead, single GPU only)
+                    extra = st.iterations - st1.iterations
                     _check(f"bfs stats root {s} dir {d}",
-                           (st.iterations, st.push_steps, st.pull_steps, st.reached) ==
-                           (st1.iterations, st1.push_steps, st1.pull_steps, st1.reached), errs)
+                           st.reached == st1.reached and extra in (0, 1) and
+                           st.push_steps >= st1.push_steps and st.pull_steps >= st1.pull_steps and
+                           st.push_steps + st.pull_steps == st.iterations, errs)
                 lv, _ = sg.run_bfs(G, int(s), owned_only=True)
                 _check(f"bfs owned_only root {s}", np.array_equal(sg.as_u32(lv)[lo:hi], ref[lo:hi]), errs)
             os.environ["SG_SPARSE"] = "1"        # fused small supersteps (peer inserts + clear barrier)
