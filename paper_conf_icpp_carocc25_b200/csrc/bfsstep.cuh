@@ -110,6 +110,20 @@ __device__ __forceinline__ uint32_t bfs_decide(BfsCtrl *c, const DevStats *st, u
         c->hmask = want;
     }
     if (zero_prev) *zero_prev = DevStats{};
+    if (!go && c->res) {   // the run's counters to the host (mapped memory; read after the graph)
+        volatile BfsResult *r = c->res;
+        r->iters = c->iters;
+        r->push_steps = c->push_steps;
+        r->pull_steps = c->pull_steps;
+        r->arcs_pushed = c->arcs_pushed;
+        r->arcs_pulled = c->arcs_pulled;
+        r->reached = c->reached;
+        r->sweep_steps = c->sweep_steps;
+        r->sparse_steps = c->sparse_steps;
+        r->overflow = c->overflow;
+        __threadfence_system();
+        r->done = 1u;
+    }
     return !go ? SK_STOP : (c->pull ? SK_PULL : (sweep ? SK_SWEEP : (sparse ? SK_SPARSE : SK_PUSH)));
 }
 

@@ -122,6 +122,10 @@ struct Workspace {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     // CUDA-graph driven BFS (ctrl.cu): instantiated once per (level buffer, tiers)
     BfsCtrl *ctrl = nullptr, *h_ctrl = nullptr;
+    BfsResult *h_res = nullptr, *d_res = nullptr;   // mapped pinned: the graph-driven BFS's counters
+    BfsProArgs pro_args{};                           // single GPU: the prologue node's argument block
+    void *pro_slot[1] = {};
+    cudaGraphNode_t pro_node = nullptr;
     unsigned int *bfs_done = nullptr;   // CTA completion counter of the BFS output kernels (self-resetting)
     unsigned int *gbar = nullptr;       // grid barrier of the sparse superstep kernel (2 u32)
     unsigned long long hnd[9] = {};     // conditional handles of bfs_graph (loop, push/pull/sweep/sparse x 2)
@@ -331,6 +335,7 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->bfs_done);
     cudaFree(ws->gbar);
     cudaFreeHost(ws->h_ctrl);
+    if (ws->h_res) cudaFreeHost(ws->h_res);
     if (ws->ev0) cudaEventDestroy(ws->ev0);
     if (ws->ev1) cudaEventDestroy(ws->ev1);
     for (cudaEvent_t e : ws->prof.pool) cudaEventDestroy(e);
@@ -1242,6 +1247,8 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     if (!ws->ctrl) {
         CK(cudaMalloc(&ws->ctrl, sizeof(BfsCtrl)));
         CK(cudaMallocHost(&ws->h_ctrl, sizeof(BfsCtrl)));
+        CK(cudaHostAlloc(&ws->h_res, sizeof(BfsResult), cudaHostAllocMapped));
+        CK(cudaHostGetDevicePointer(&ws->d_res, ws->h_res, 0));
     }
     cudaStream_t cs = ws->cap_stream;
     cudaGraph_t root;
@@ -1264,9 +1271,26 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     // prologue: level = INF, frontiers cleared, visited = isolated, seed src, compact + decide
     TRY(capture_begin(cs, root, {}));
     // (the output frontier F[1] is written whole by the first output kernel: only F[0] is zeroed)
-    if (!g->ar) {   // single GPU: one kernel (memsets / copies folded in)
-        launch_bfs_prologue1(ws->ctrl, G.n, G.nw1, G.nw2, G.deg8, g->isolated, F[0]->bits, F[0]->summ,
-                             F[0]->offsets, F[0]->st, F[1]->st, ws->visited, ws->vis_old, cs);
+    if (!g->ar) {   // single GPU: one kernel node (memsets / copies folded in; init as its parameter)
+        BfsProArgs &pa = ws->pro_args;
+        pa.c = ws->ctrl;
+        pa.n = G.n;
+        pa.nw1 = G.nw1;
+        pa.nw2 = G.nw2;
+        pa.deg8 = G.deg8;
+        pa.isolated = g->isolated;
+        pa.bits = F[0]->bits;
+        pa.summ = F[0]->summ;
+        pa.offsets = F[0]->offsets;
+        pa.st = F[0]->st;
+        pa.st_out = F[1]->st;
+        pa.visited = ws->visited;
+        pa.vis_old = ws->vis_old;
+        cudaKernelNodeParams kp;
+        bfs_prologue1_node(&pa, ws->pro_slot, &kp);
+        TRY(capture_end(cs, leaves));   // (nothing captured)
+        CK(cudaGraphAddKernelNode(&ws->pro_node, root, nullptr, 0, &kp));
+        leaves = {ws->pro_node};
     } else {
         CK(cudaMemsetAsync(F[0]->bits, 0, sizeof(uint64_t) * (size_t)G.nw1, cs));
         CK(cudaMemsetAsync(F[0]->summ, 0, sizeof(uint64_t) * (size_t)G.nw2, cs));
@@ -1284,7 +1308,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         ws->hnd[5 + i] = sc ? (unsigned long long)h_sweep[i] : 0ull;
         ws->hnd[7 + i] = sp ? (unsigned long long)h_sparse[i] : 0ull;
     }
-    TRY(capture_end(cs, leaves));
+    if (g->ar) TRY(capture_end(cs, leaves));
     cudaGraphNode_t wnode;
     cudaGraph_t body;
     TRY(add_cond(root, leaves, h_loop, cudaGraphCondTypeWhile, &wnode, &body));
@@ -1389,6 +1413,8 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     c.sparse_arcs = env_or("SG_SPARSE_ARCS", 1 << 16);
     c.pull_warp_frac = (uint32_t)env_or("SG_PULL_WARP_FRAC", 8);
     c.n_iso = g->n_iso;
+    c.res = ws->d_res;
+    memset((void *)ws->h_res, 0, sizeof(BfsResult));   // (the previous run's graph has completed)
     c.hl = ws->hnd[0];
     for (int i = 0; i < 2; i++) {
         c.hpush[i] = ws->hnd[1 + i];
@@ -1399,7 +1425,14 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     CK(cudaEventRecord(ws->ev0, s));
     // the control block up to the trace arrays (those are read on demand by sg_bfs_trace)
     const size_t hot = offsetof(BfsCtrl, t_ns);
-    CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, hot, cudaMemcpyHostToDevice, s));
+    if (!g->ar) {   // single GPU: the control block's init rides on the prologue node's parameters
+        memcpy(ws->pro_args.hot, ws->h_ctrl, hot);
+        cudaKernelNodeParams kp;
+        bfs_prologue1_node(&ws->pro_args, ws->pro_slot, &kp);
+        CK(cudaGraphExecKernelNodeSetParams(ws->bfs_exec, ws->pro_node, &kp));
+    } else {
+        CK(cudaMemcpyAsync(ws->ctrl, ws->h_ctrl, hot, cudaMemcpyHostToDevice, s));
+    }
     CK(cudaGraphLaunch(ws->bfs_exec, s));
     if (g->ar && !o.owned_only) {   // result gather: owned level slices into every rank's replica
         const Arena *A = g->ar;
@@ -1407,9 +1440,21 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         launch_xbarrier(A->x, s);
         CK(cudaMemcpyAsync(level, A->vals, sizeof(uint32_t) * (size_t)g->v.n, cudaMemcpyDeviceToDevice, s));
     }
-    CK(cudaMemcpyAsync(ws->h_ctrl, ws->ctrl, hot, cudaMemcpyDeviceToHost, s));
     CK(cudaEventRecord(ws->ev1, s));
     CK(cudaEventSynchronize(ws->ev1));
+    {   // the counters the stopping decision wrote into mapped host memory
+        const volatile BfsResult *r = ws->h_res;
+        if (!r->done) return fail(SG_ERR_STATE, "the BFS graph ended without a stopping decision");
+        c.iters = r->iters;
+        c.push_steps = r->push_steps;
+        c.pull_steps = r->pull_steps;
+        c.arcs_pushed = r->arcs_pushed;
+        c.arcs_pulled = r->arcs_pulled;
+        c.reached = r->reached;
+        c.sweep_steps = r->sweep_steps;
+        c.sparse_steps = r->sparse_steps;
+        c.overflow = r->overflow;
+    }
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, ws->ev0, ws->ev1));
     CK(cudaGetLastError());

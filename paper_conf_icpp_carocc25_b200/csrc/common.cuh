@@ -97,6 +97,14 @@ struct ValCtrl {
     unsigned long long hl, hpush[2], hpull[2];
 };
 
+// A graph-driven BFS's final counters, written by the stopping decision straight into mapped
+// pinned host memory (no device->host copy after the graph: ~7 us per BFS, scripts/micro/bfs_fixed_cost.py)
+struct BfsResult {
+    unsigned long long iters, push_steps, pull_steps, arcs_pushed, arcs_pulled, reached, sweep_steps, sparse_steps,
+        hub_steps;
+    uint32_t overflow, done;
+};
+
 // Device-resident state of a graph-driven BFS (written by k_bfs_decide, read back once per run).
 struct BfsCtrl {
     unsigned long long iters, push_steps, pull_steps, arcs_pushed, arcs_pulled, reached;
@@ -132,6 +140,7 @@ struct BfsCtrl {
     uint32_t pull_warp_frac; // ... when unvisited non-isolated vertices < (n - n_iso) / pull_warp_frac
     long long n_iso;         // isolated vertices (visited from the start, never reached)
     long long src_iso;       // 1 iff the source itself is one of them (counted in reached too)
+    BfsResult *res;          // mapped host memory: the stopping decision writes the run's counters there
     uint32_t sp_kind;        // the fused sparse loop's last decision (read by all its CTAs)
     uint32_t sp_epoch;       // bumped by CTA 0 once sp_kind is written (the loop's broadcast)
     uint32_t hmask;          // current values of the IF handles (bit 2k+b: kind k of buffer b; bit 8: loop);

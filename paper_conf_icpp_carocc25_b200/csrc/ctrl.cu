@@ -95,24 +95,25 @@ __global__ void k_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint6
 // visited[w] = vis_old[w] = isolated[w] (| src's bit), the input frontier's word = src's bit or 0;
 // layer 2 likewise; both control blocks written whole by thread 0; then the level pass and the
 // first decision as k_bfs_prologue.  Every store lands in a distinct word, so no ordering is needed
-// inside the kernel (the supersteps read them after the kernel boundary).
-__global__ void k_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2, const uint8_t *deg8,
-                                const uint64_t *__restrict__ isolated, uint64_t *bits, uint64_t *summ,
-                                uint32_t *offsets, DevStats *st, DevStats *st_out, uint64_t *visited,
-                                uint64_t *vis_old) {
-    uint32_t *level = c->level;
-    const int32_t src = c->src;
+// inside the kernel (the supersteps read them after the kernel boundary).  The run's control-block
+// initialisation arrives as a kernel parameter (set on the graph node before each launch): no
+// host->device copy before the graph.
+__global__ void k_bfs_prologue1(const BfsProArgs a) {
+    const BfsCtrl *h = reinterpret_cast<const BfsCtrl *>(a.hot);   // the control block's leading part
+    uint32_t *level = h->level;
+    const int32_t src = h->src;
+    const int64_t n = a.n;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t ws = src >> 6;
     const uint64_t sb = 1ull << (src & 63);
-    for (int64_t w = t; w < nw1; w += stride) {
-        const uint64_t v = isolated[w] | (w == ws ? sb : 0ull);
-        visited[w] = v;
-        vis_old[w] = v;
-        bits[w] = w == ws ? sb : 0ull;
+    for (int64_t w = t; w < a.nw1; w += stride) {
+        const uint64_t v = a.isolated[w] | (w == ws ? sb : 0ull);
+        a.visited[w] = v;
+        a.vis_old[w] = v;
+        a.bits[w] = w == ws ? sb : 0ull;
     }
-    for (int64_t w = t; w < nw2; w += stride) summ[w] = w == (src >> 12) ? 1ull << ((src >> 6) & 63) : 0ull;
+    for (int64_t w = t; w < a.nw2; w += stride) a.summ[w] = w == (src >> 12) ? 1ull << ((src >> 6) & 63) : 0ull;
     if (((uintptr_t)level & 15) == 0) {
         uint4 *l4 = reinterpret_cast<uint4 *>(level);
         for (int64_t i = t; i < n / 4; i += stride) {
@@ -125,29 +126,37 @@ __global__ void k_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2,
         for (int64_t i = t; i < n; i += stride) level[i] = i == src ? 0u : INF32;
     }
     if (t == 0) {
-        offsets[0] = (uint32_t)ws;
-        c->src_iso = (long long)((isolated[ws] >> (src & 63)) & 1ull);
+        BfsCtrl *c = a.c;
+        unsigned long long *cw = reinterpret_cast<unsigned long long *>(c);
+        for (int i = 0; i < BFS_CTRL_HOT_WORDS; i++) cw[i] = a.hot[i];
+        a.offsets[0] = (uint32_t)ws;
+        c->src_iso = (long long)((a.isolated[ws] >> (src & 63)) & 1ull);
         DevStats d{};
         d.count = 1ull;
         d.nf = 1ull;
-        d.mf = deg8_decode(deg8[src]);
-        *st = d;
-        *st_out = DevStats{};
+        d.mf = deg8_decode(a.deg8[src]);
+        *a.st = d;
+        *a.st_out = DevStats{};
         c->dirty[0] = 0u;
         c->dirty[1] = 1u;
         c->saved_count[1] = ~0ull;
-        bfs_decide(c, st, 0ull, nullptr, 0, 1);
+        bfs_decide(c, a.st, 0ull, nullptr, 0, 1);
     }
 }
-void launch_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2, const uint8_t *deg8,
-                          const uint64_t *isolated, uint64_t *bits, uint64_t *summ, uint32_t *offsets, DevStats *st,
-                          DevStats *st_out, uint64_t *visited, uint64_t *vis_old, cudaStream_t s) {
-    int64_t blocks = (n / 4 + 255) / 256;
+// kernel-node parameters of k_bfs_prologue1 for `a` (its address must stay valid while the node
+// parameters are set: kernelParams points at it)
+void bfs_prologue1_node(BfsProArgs *a, void **arg_slot, cudaKernelNodeParams *kp) {
+    int64_t blocks = (a->n / 4 + 255) / 256;
     if (blocks > num_sms() * 8) blocks = num_sms() * 8;
     if (blocks < 1) blocks = 1;
-    note_launch();
-    k_bfs_prologue1<<<(int)blocks, 256, 0, s>>>(c, n, nw1, nw2, deg8, isolated, bits, summ, offsets, st, st_out,
-                                                visited, vis_old);
+    arg_slot[0] = a;
+    *kp = cudaKernelNodeParams{};
+    kp->func = (void *)k_bfs_prologue1;
+    kp->gridDim = dim3((unsigned)blocks);
+    kp->blockDim = dim3(256);
+    kp->sharedMemBytes = 0;
+    kp->kernelParams = arg_slot;
+    kp->extra = nullptr;
 }
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                          uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old, const Xchg &x,

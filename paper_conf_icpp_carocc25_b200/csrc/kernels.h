@@ -1,5 +1,6 @@
 // kernels.h — host-side launchers of the sm_100a kernels (internal to libsygraph).
 #pragma once
+#include <cstddef>
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <vector>
@@ -202,10 +203,22 @@ int ablation_bfs_words(const GraphView &g, int32_t src, uint32_t *level, int wor
                        float *ms);
 // ctrl.cu — device-side superstep control (CUDA-graph driven loops)
 // level init + seed + the seed frontier's word list / statistics + first decision, one kernel
-// single-GPU: the same with the frontier, visited / vis_old and control-block initialisation folded in
-void launch_bfs_prologue1(BfsCtrl *c, int64_t n, int64_t nw1, int64_t nw2, const uint8_t *deg8,
-                          const uint64_t *isolated, uint64_t *bits, uint64_t *summ, uint32_t *offsets, DevStats *st,
-                          DevStats *st_out, uint64_t *visited, uint64_t *vis_old, cudaStream_t s);
+// single-GPU: the same with the frontier, visited / vis_old and control-block initialisation folded
+// in, added to the graph as a kernel node whose argument block carries the run's control-block
+// initialisation (`hot`: the leading BFS_CTRL_HOT_WORDS words of BfsCtrl)
+constexpr int BFS_CTRL_HOT_WORDS = (int)((offsetof(BfsCtrl, t_ns) + 7) / 8);
+struct BfsProArgs {
+    BfsCtrl *c;
+    int64_t n, nw1, nw2;
+    const uint8_t *deg8;
+    const uint64_t *isolated;
+    uint64_t *bits, *summ;
+    uint32_t *offsets;
+    DevStats *st, *st_out;
+    uint64_t *visited, *vis_old;
+    unsigned long long hot[BFS_CTRL_HOT_WORDS];
+};
+void bfs_prologue1_node(BfsProArgs *a, void **arg_slot, cudaKernelNodeParams *kp);
 void launch_bfs_prologue(BfsCtrl *c, int64_t n, const uint8_t *deg8, uint64_t *bits, uint64_t *summ,
                          uint32_t *offsets, DevStats *st, uint64_t *visited, uint64_t *vis_old, const Xchg &x,
                          cudaStream_t s);
