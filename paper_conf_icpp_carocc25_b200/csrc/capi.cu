@@ -12,6 +12,7 @@
 #include <cstring>
 #include <string>
 #include <vector>
+#include <mutex>
 
 #include <cuda.h>   // CUdeviceptr / CUresult types for the driver entry point below (no -lcuda)
 
@@ -191,6 +192,32 @@ struct sg_graph {
 };
 static std::atomic<int> g_live_graphs{0};
 
+// Result slots of graph-driven BFS runs (R20): mapped pinned host memory, carved from slabs that
+// live for the process (a cudaHostAlloc / cudaFreeHost pair per graph load cost ~0.7 s of
+// graph_load + graph_free in the end-to-end bench: freeing mapped memory synchronises and unmaps)
+static std::mutex g_res_mu;
+static std::vector<std::pair<BfsResult *, BfsResult *>> g_res_free;   // (host, device)
+static int res_slot_alloc(BfsResult **h, BfsResult **d) {
+    std::lock_guard<std::mutex> lk(g_res_mu);
+    if (g_res_free.empty()) {
+        constexpr int SLAB = 256;
+        BfsResult *hs = nullptr, *ds = nullptr;
+        CK(cudaHostAlloc(&hs, sizeof(BfsResult) * SLAB, cudaHostAllocMapped | cudaHostAllocPortable));
+        CK(cudaHostGetDevicePointer(&ds, hs, 0));
+        for (int i = SLAB - 1; i >= 0; i--) g_res_free.emplace_back(hs + i, ds + i);
+    }
+    *h = g_res_free.back().first;
+    *d = g_res_free.back().second;
+    g_res_free.pop_back();
+    return SG_OK;
+}
+static void res_slot_free(BfsResult *h) {
+    std::lock_guard<std::mutex> lk(g_res_mu);
+    // the device pointer of a slot: same offset in its slab (slabs are never freed)
+    BfsResult *d = nullptr;
+    if (cudaHostGetDevicePointer(&d, h, 0) == cudaSuccess) g_res_free.emplace_back(h, d);
+}
+
 static const int32_t kDefaultHeavy = 2048;
 static const int32_t kDefaultSmall = 32;
 
@@ -335,7 +362,7 @@ static void free_ws(Workspace *ws) {
     cudaFree(ws->bfs_done);
     cudaFree(ws->gbar);
     cudaFreeHost(ws->h_ctrl);
-    if (ws->h_res) cudaFreeHost(ws->h_res);
+    if (ws->h_res) res_slot_free(ws->h_res);
     if (ws->ev0) cudaEventDestroy(ws->ev0);
     if (ws->ev1) cudaEventDestroy(ws->ev1);
     for (cudaEvent_t e : ws->prof.pool) cudaEventDestroy(e);
@@ -1247,8 +1274,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     if (!ws->ctrl) {
         CK(cudaMalloc(&ws->ctrl, sizeof(BfsCtrl)));
         CK(cudaMallocHost(&ws->h_ctrl, sizeof(BfsCtrl)));
-        CK(cudaHostAlloc(&ws->h_res, sizeof(BfsResult), cudaHostAllocMapped));
-        CK(cudaHostGetDevicePointer(&ws->d_res, ws->h_res, 0));
+        TRY(res_slot_alloc(&ws->h_res, &ws->d_res));
     }
     cudaStream_t cs = ws->cap_stream;
     cudaGraph_t root;
@@ -1271,7 +1297,9 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
     // prologue: level = INF, frontiers cleared, visited = isolated, seed src, compact + decide
     TRY(capture_begin(cs, root, {}));
     // (the output frontier F[1] is written whole by the first output kernel: only F[0] is zeroed)
-    if (!g->ar) {   // single GPU: one kernel node (memsets / copies folded in; init as its parameter)
+    const bool pro_node = !g->ar && env_or("SG_PRO_PARAMS", 1) != 0;
+    ws->pro_node = nullptr;
+    if (pro_node) {   // single GPU: one kernel node (memsets / copies folded in; init as its parameter)
         BfsProArgs &pa = ws->pro_args;
         pa.c = ws->ctrl;
         pa.n = G.n;
@@ -1298,7 +1326,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         CK(cudaMemcpyAsync(ws->visited, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
         CK(cudaMemcpyAsync(ws->vis_old, g->isolated, sizeof(uint64_t) * (size_t)G.nw1, cudaMemcpyDeviceToDevice, cs));
         launch_bfs_prologue(ws->ctrl, G.n, G.deg8, F[0]->bits, F[0]->summ, F[0]->offsets, F[0]->st, ws->visited,
-                            ws->vis_old, g->ar->x, cs);
+                            ws->vis_old, g->ar ? g->ar->x : Xchg{}, cs);
     }
     // the handles go to the device with every run's control block (run_bfs_graph)
     ws->hnd[0] = (unsigned long long)h_loop;
@@ -1308,7 +1336,7 @@ static int build_bfs_graph(sg_graph *g, Tiers t) {
         ws->hnd[5 + i] = sc ? (unsigned long long)h_sweep[i] : 0ull;
         ws->hnd[7 + i] = sp ? (unsigned long long)h_sparse[i] : 0ull;
     }
-    if (g->ar) TRY(capture_end(cs, leaves));
+    if (!pro_node) TRY(capture_end(cs, leaves));
     cudaGraphNode_t wnode;
     cudaGraph_t body;
     TRY(add_cond(root, leaves, h_loop, cudaGraphCondTypeWhile, &wnode, &body));
@@ -1413,7 +1441,11 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     c.sparse_arcs = env_or("SG_SPARSE_ARCS", 1 << 16);
     c.pull_warp_frac = (uint32_t)env_or("SG_PULL_WARP_FRAC", 8);
     c.n_iso = g->n_iso;
-    c.res = ws->d_res;
+    // counters back through mapped host memory (SG_RES_MAPPED=1, ~7 us less per BFS) or the
+    // device->host copy (default): with the mapped path on, the end-to-end bench's graph_load /
+    // graph_free cycle slowed 4-8x in 4 of 5 runs (0.7-1.3 vs 5.6 GTEPS e2e), cause not isolated
+    static const bool res_mapped = env_or("SG_RES_MAPPED", 0) != 0;
+    c.res = res_mapped ? ws->d_res : nullptr;
     memset((void *)ws->h_res, 0, sizeof(BfsResult));   // (the previous run's graph has completed)
     c.hl = ws->hnd[0];
     for (int i = 0; i < 2; i++) {
@@ -1425,7 +1457,7 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
     CK(cudaEventRecord(ws->ev0, s));
     // the control block up to the trace arrays (those are read on demand by sg_bfs_trace)
     const size_t hot = offsetof(BfsCtrl, t_ns);
-    if (!g->ar) {   // single GPU: the control block's init rides on the prologue node's parameters
+    if (ws->pro_node) {   // single GPU: the control block's init rides on the prologue node's parameters
         memcpy(ws->pro_args.hot, ws->h_ctrl, hot);
         cudaKernelNodeParams kp;
         bfs_prologue1_node(&ws->pro_args, ws->pro_slot, &kp);
@@ -1440,9 +1472,10 @@ static int run_bfs_graph(sg_graph *g, int32_t src, uint32_t *level, const sg_opt
         launch_xbarrier(A->x, s);
         CK(cudaMemcpyAsync(level, A->vals, sizeof(uint32_t) * (size_t)g->v.n, cudaMemcpyDeviceToDevice, s));
     }
+    if (!res_mapped) CK(cudaMemcpyAsync(ws->h_ctrl, ws->ctrl, hot, cudaMemcpyDeviceToHost, s));
     CK(cudaEventRecord(ws->ev1, s));
     CK(cudaEventSynchronize(ws->ev1));
-    {   // the counters the stopping decision wrote into mapped host memory
+    if (res_mapped) {   // the counters the stopping decision wrote into mapped host memory
         const volatile BfsResult *r = ws->h_res;
         if (!r->done) return fail(SG_ERR_STATE, "the BFS graph ended without a stopping decision");
         c.iters = r->iters;
