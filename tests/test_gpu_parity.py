@@ -641,3 +641,36 @@ def test_bfs_pull_build_variants(sg, name, defines):
     env = dict(os.environ, SYGRAPH_LIB=lib, PYTHONPATH=root)
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, cwd=root)
     assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
+
+
+def _deg8_decoded(d):
+    """The library's 8-bit degree code (exact below 32, 3 mantissa bits above) decoded: the m_f
+    unit of the direction policy (frontier.cu k_deg8 / common.cuh deg8_decode)."""
+    d = np.asarray(d, dtype=np.int64)
+    out = d.copy()
+    big = d >= 32
+    e = np.floor(np.log2(np.maximum(d, 1))).astype(np.int64)
+    m = (d >> np.maximum(e - 3, 0)) & 7
+    code = np.minimum(32 + (e - 5) * 8 + m, 255)
+    e2 = ((code - 32) >> 3) + 5
+    m2 = (code - 32) & 7
+    out[big] = (((8 + m2) << (e2 - 3)) + (1 << (e2 - 4)))[big]
+    return out
+
+
+@pytest.mark.parametrize("direction", DIRS)
+def test_bfs_trace_frontier_statistics(sg, direction):
+    """n_f and m_f of every BFS frontier as the output kernels sum them (quad_mf: the dp4a path
+    for degrees < 32, the table path for coded ones) equal the level sizes and the decoded degree
+    sums of the oracle's levels, on a graph with hubs and low-degree vertices mixed in quads."""
+    g = gen.rmat(14, 16, permute=True)
+    G = load(sg, g)
+    dec = _deg8_decoded(g.degrees())
+    for s in gen.sources(g, 2):
+        ref = oracle.bfs(g, int(s))
+        lv, st = sg.run_bfs(G, int(s), direction=_dir(sg, direction))
+        assert np.array_equal(sg.as_u32(lv), ref)
+        for t in sg.bfs_trace(G):
+            at = ref == t["step"]
+            assert t["nf"] == int(at.sum()), t
+            assert t["mf"] == int(dec[at].sum()), t
