@@ -419,33 +419,58 @@ __global__ void __launch_bounds__(PUSH_THREADS) k_push_words(PushParams p, F f) 
     // sparse: <= 2 active vertices per word on average, of average degree <= 16 (else the
     // warp-tier vertices of 32 words would serialise on one warp)
     const bool sparse = SG_SPARSE_WORDS && p.sparse_ok && p.st->nf <= 2ull * count && p.st->mf <= 16ull * p.st->nf;
-    // Each CTA takes a contiguous share of the word list; its warps take `grab` words at a time,
-    // the first grab static (warp id x grab), later ones from a shared-memory counter.  (One
-    // global counter for all warps serialised a 13 K-word hub level at ~8 K same-address
-    // atomics: 45 % of that k_push_words' stall samples, profiles/r02j_full_l2push.)
-    __shared__ uint32_t s_next;
     if constexpr (F::kSeg) {
         if (lane_id() == 0) s_warp[wid].nhq = 0;
+        __syncwarp();
     }
-    if (threadIdx.x == 0) s_next = 0u;
-    __syncthreads();
     const uint32_t grab = sparse ? 32u : batch;
-    const uint32_t per = (count + gridDim.x - 1) / gridDim.x;
-    const uint32_t c0 = min(blockIdx.x * per, count), c1 = min(c0 + per, count);
-    const uint32_t statics = PUSH_WARPS * grab;
-    for (uint32_t r = wid * grab;;) {
-        const uint32_t b0 = c0 + r;
-        if (b0 >= c1) break;
-        if (sparse) {   // 32 words per grab, one per lane
-            arcs += push_words_sparse(p, f, b0 + lane_id(), c1, seg_on);
-        } else {
-            const uint32_t b1 = min(b0 + grab, c1);
-            for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid], seg_on);
+    if constexpr (F::kSeg) {
+        // BFS: each CTA takes a contiguous share of the word list; its warps take `grab` words at
+        // a time, the first grab static (warp id x grab), later ones from a shared-memory counter.
+        // (One global counter for all warps serialised a 13 K-word hub level at ~8 K same-address
+        // atomics: 45 % of that k_push_words' stall samples, profiles/r02j_full_l2push.  Its hubs
+        // leave the warp as queued chunks, so the per-word work is small and even.)
+        __shared__ uint32_t s_next;
+        if (threadIdx.x == 0) s_next = 0u;
+        __syncthreads();
+        const uint32_t per = (count + gridDim.x - 1) / gridDim.x;
+        const uint32_t c0 = min(blockIdx.x * per, count), c1 = min(c0 + per, count);
+        const uint32_t statics = PUSH_WARPS * grab;
+        for (uint32_t r = wid * grab;;) {
+            const uint32_t b0 = c0 + r;
+            if (b0 >= c1) break;
+            if (sparse) {   // 32 words per grab, one per lane
+                arcs += push_words_sparse(p, f, b0 + lane_id(), c1, seg_on);
+            } else {
+                const uint32_t b1 = min(b0 + grab, c1);
+                for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid], seg_on);
+            }
+            if (c0 + statics >= c1) break;
+            uint32_t nb = 0;
+            if (lane_id() == 0) nb = statics + atomicAdd(&s_next, grab);
+            r = __shfl_sync(0xffffffffu, nb, 0);
         }
-        if (c0 + statics >= c1) break;
-        uint32_t nb = 0;
-        if (lane_id() == 0) nb = statics + atomicAdd(&s_next, grab);
-        r = __shfl_sync(0xffffffffu, nb, 0);
+    } else {
+        // SSSP / CC / BC: grid-wide dynamic grabs (a warp's first grab static, later ones from one
+        // global counter): their words carry uneven warp-tier work that a static CTA share leaves
+        // unbalanced (C2 SSSP 0.90 -> 1.51 ms when it shared the BFS scheme)
+        const uint32_t gwarp = (blockIdx.x * PUSH_THREADS + threadIdx.x) >> 5;
+        const uint32_t nwarps = gridDim.x * PUSH_WARPS;
+        const unsigned long long statics = (unsigned long long)nwarps * grab;
+        for (unsigned long long b0l = (unsigned long long)gwarp * grab;;) {
+            if (b0l >= count) break;
+            const uint32_t b0 = (uint32_t)b0l;
+            if (sparse) {
+                arcs += push_words_sparse(p, f, b0 + lane_id(), count, seg_on);
+            } else {
+                const uint32_t b1 = min(b0 + grab, count);
+                for (uint32_t i = b0; i < b1; i++) arcs += push_word(p, f, p.offsets[i], s_warp[wid], seg_on);
+            }
+            if (statics >= count) break;
+            unsigned long long nb = 0;
+            if (lane_id() == 0) nb = statics + atomicAdd(&p.st->batch, (unsigned long long)grab);
+            b0l = __shfl_sync(0xffffffffu, nb, 0);
+        }
     }
     if constexpr (F::kSeg) flush_hubs(p, s_warp[wid]);
     arcs = warp_sum(arcs);
